@@ -1,0 +1,83 @@
+"""Workload shapes (sizes only; no arithmetic of the method).
+
+Sizes follow BASELINE.json `configs` and PAPER.md Table 2:
+|V|, |E|, d_e, max(t). Bipartite user/item splits follow the JODIE datasets
+the paper uses. Model shape: 2-layer TGAT, 2 heads, k most-recent
+neighbours, batch 200; d_t = d_n.
+"""
+from dataclasses import dataclass, field, replace
+
+
+@dataclass(frozen=True)
+class StreamConfig:
+    name: str
+    n_nodes: int            # |V|; node ids are 1..n_nodes, 0 = padding
+    n_edges: int            # |E|; edge ids are 1..n_edges, 0 = padding
+    d_n: int                # node feature dim
+    d_e: int                # edge feature dim
+    max_t: int              # timestamps are integer seconds in [0, max_t]
+    bipartite: bool
+    n_users: int = 0        # bipartite: ids 1..n_users are users, the rest items
+    seed: int = 0
+    # generator knobs (shape of the stream)
+    p_rep: float = 0.6      # prob. a user re-interacts with its previous item
+    zipf_user: float = 0.8
+    zipf_item: float = 1.2
+    session_mean: float = 6.0
+    gap_scale: float = 30.0  # Pareto scale (s) of intra-session gaps -> power-law dt near 0 (Fig. 4)
+
+
+@dataclass(frozen=True)
+class ModelConfig:
+    n_layers: int = 2       # L
+    n_heads: int = 2        # heads
+    n_neighbors: int = 20   # k most-recent
+    batch: int = 200        # edges per batch
+    cache_limit: int = 2_000_000   # items
+    time_window: int = 10_000      # precomputed dt window
+    param_seed: int = 1234
+
+
+@dataclass(frozen=True)
+class Config:
+    stream: StreamConfig
+    model: ModelConfig = field(default_factory=ModelConfig)
+
+    @property
+    def name(self):
+        return self.stream.name
+
+
+CONFIGS = {
+    # tiny cases for the oracle's own pins (pure-Python brute force finishes fast)
+    "tiny": Config(StreamConfig("tiny", 12, 60, 4, 4, 1000, False, seed=7, gap_scale=3.0),
+                   ModelConfig(n_neighbors=3, batch=10, time_window=50)),
+    "tiny_bip": Config(StreamConfig("tiny_bip", 16, 120, 8, 4, 5000, True, n_users=12, seed=8,
+                                    gap_scale=5.0),
+                       ModelConfig(n_neighbors=4, batch=12, time_window=100)),
+    # configs[0]: synthetic 1k-node / 10k-edge stream, k=10, d_n=100, d_e=172 (oracle in seconds)
+    "config1": Config(StreamConfig("config1", 1000, 10_000, 100, 172, 1_000_000, False, seed=0),
+                      ModelConfig(n_neighbors=10)),
+    # configs[1]: Wikipedia-shaped (jodie-wiki, Table 2: 9,227 / 157,474 / 172 / 2.7e6)
+    "wiki": Config(StreamConfig("wiki", 9227, 157_474, 172, 172, 2_700_000, True, n_users=8227,
+                                seed=2, p_rep=0.75)),
+    # configs[2]: Reddit-shaped (jodie-reddit, Table 2: 10,984 / 672,447 / 172 / 2.7e6)
+    "reddit": Config(StreamConfig("reddit", 10984, 672_447, 172, 172, 2_700_000, True,
+                                  n_users=10000, seed=3, p_rep=0.6)),
+    # configs[3]: LastFM / MOOC-shaped high-repetition streams
+    "lastfm": Config(StreamConfig("lastfm", 1980, 1_293_103, 100, 100, 140_000_000, True,
+                                  n_users=1000, seed=41, p_rep=0.7)),
+    "mooc": Config(StreamConfig("mooc", 7144, 411_749, 4, 4, 2_600_000, True, n_users=7047,
+                                seed=42, p_rep=0.8)),
+    # configs[4]: large Reddit-Posts/GDELT-like stream, batch 2,000
+    "large": Config(StreamConfig("large", 1_000_000, 10_000_000, 172, 172, 100_000_000, True,
+                                 n_users=900_000, seed=5),
+                    ModelConfig(batch=2000)),
+}
+
+
+def get_config(name: str, **model_overrides) -> Config:
+    cfg = CONFIGS[name]
+    if model_overrides:
+        cfg = Config(cfg.stream, replace(cfg.model, **model_overrides))
+    return cfg
