@@ -1,0 +1,219 @@
+// Dense per-target stages of M and the merge FFN (Eqs. 6-7) on CUDA cores
+// (TG_PREC_FP32), LayerNorm (R1), the link-prediction score (R10) and the
+// DedupInvert row copy (Alg. 1 l.20).
+#include "tg_internal.cuh"
+
+namespace tg {
+
+// ----------------------------------------------------------- SIMT fp32 GEMM
+// C[M x N] = epi(A[M x K] . B[N x K]^T); 64x64 tiles, BK = 16, 256 threads,
+// 4x4 outputs per thread, fixed K order (batch-invariant rows).
+constexpr int GBM = 64, GBN = 64, GBK = 16;
+
+__device__ __forceinline__ float4 gemm_load_a(const GemmArgs& g, int row, int M, int c) {
+  if (row >= M || c >= g.K) return make_float4(0.f, 0.f, 0.f, 0.f);
+  const float* p;
+  if (c < g.K0) {
+    p = g.a_rows0 ? g.a_rows0[row] + c : g.a_base0 + (size_t)row * g.lda0 + c;
+  } else {
+    const int cc = c - g.K0;
+    p = g.a_rows1 ? g.a_rows1[row] + cc : g.a_base1 + (size_t)row * g.lda1 + cc;
+  }
+  return *reinterpret_cast<const float4*>(p);
+}
+
+__global__ void __launch_bounds__(256) k_gemm_simt(GemmArgs g) {
+  __shared__ __align__(16) float As[GBK][GBM + 4];
+  __shared__ __align__(16) float Bs[GBK][GBN + 4];
+  const int M = *g.m_dev;
+  const int tiles_m = (M + GBM - 1) / GBM, tiles_n = (g.N + GBN - 1) / GBN;
+  const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
+  const int lr = tid >> 2, lc4 = tid & 3;  // loader: row, float4 column
+  for (int t = blockIdx.x; t < tiles_m * tiles_n; t += gridDim.x) {
+    const int tm = t / tiles_n, tn = t - tm * tiles_n;
+    const int m0 = tm * GBM, n0 = tn * GBN;
+    float acc[4][4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+      for (int j = 0; j < 4; ++j) acc[i][j] = 0.f;
+    for (int k0 = 0; k0 < g.K; k0 += GBK) {
+      const float4 av = gemm_load_a(g, m0 + lr, M, k0 + 4 * lc4);
+      float4 bv = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (n0 + lr < g.N && k0 + 4 * lc4 < g.K)
+        bv = *reinterpret_cast<const float4*>(g.B + (size_t)(n0 + lr) * g.K + k0 + 4 * lc4);
+      As[4 * lc4 + 0][lr] = av.x;
+      As[4 * lc4 + 1][lr] = av.y;
+      As[4 * lc4 + 2][lr] = av.z;
+      As[4 * lc4 + 3][lr] = av.w;
+      Bs[4 * lc4 + 0][lr] = bv.x;
+      Bs[4 * lc4 + 1][lr] = bv.y;
+      Bs[4 * lc4 + 2][lr] = bv.z;
+      Bs[4 * lc4 + 3][lr] = bv.w;
+      __syncthreads();
+#pragma unroll
+      for (int kk = 0; kk < GBK; ++kk) {
+        const float4 a4 = *reinterpret_cast<const float4*>(&As[kk][ty * 4]);
+        const float4 b4 = *reinterpret_cast<const float4*>(&Bs[kk][tx * 4]);
+        const float a[4] = {a4.x, a4.y, a4.z, a4.w};
+        const float b[4] = {b4.x, b4.y, b4.z, b4.w};
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+#pragma unroll
+          for (int j = 0; j < 4; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+      }
+      __syncthreads();
+    }
+    // epilogue: bias, residual q = [hs || 0 || Phi(0)] (Eq. 4), ReLU, store
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int r = m0 + ty * 4 + i;
+      const int c = n0 + tx * 4;
+      if (r >= M || c >= g.N) continue;
+      float v[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        float x = acc[i][j];
+        if (g.bias) x += g.bias[c + j];
+        if (g.q_rows) {
+          const int cc = c + j;
+          if (cc < g.q_dnp) x += g.q_rows[r][cc];
+          else if (cc >= g.q_dnp + g.q_dep) x += g.q_phi0[cc - g.q_dnp - g.q_dep];
+        }
+        if (g.relu) x = fmaxf(x, 0.f);
+        v[j] = x;
+      }
+      float* out = g.c_rows ? g.c_rows[r] + c : g.C + (size_t)r * g.ldc + c;
+      *reinterpret_cast<float4*>(out) = make_float4(v[0], v[1], v[2], v[3]);
+    }
+  }
+}
+
+void launch_gemm_simt(const GemmArgs& g, cudaStream_t st) {
+  const int tiles = ((g.m_max + GBM - 1) / GBM) * ((g.N + GBN - 1) / GBN);
+  int blocks = tiles < 148 * 4 ? tiles : 148 * 4;
+  if (blocks < 1) blocks = 1;
+  k_gemm_simt<<<blocks, 256, 0, st>>>(g);
+}
+
+// ---------------------------------------------------------------- LayerNorm
+__global__ void k_layernorm(const float* __restrict__ y, float* __restrict__ r, int Dp, int dn, int dnp, int de,
+                            int dep, int dt, const float* __restrict__ gamma, const float* __restrict__ beta,
+                            const int* __restrict__ m_dev) {
+  const int M = *m_dev;
+  const int lane = threadIdx.x & 31;
+  const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, nw = (gridDim.x * blockDim.x) >> 5;
+  const int D = dn + de + dt;
+  const int s1 = dnp, s2 = dnp + dep;
+  for (int row = warp; row < M; row += nw) {
+    const float* yr = y + (size_t)row * Dp;
+    float* rr = r + (size_t)row * Dp;
+    float sum = 0.f;
+    for (int c = lane; c < Dp; c += 32) {
+      const bool valid = c < dn || (c >= s1 && c < s1 + de) || (c >= s2 && c < s2 + dt);
+      if (valid) sum += yr[c];
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
+    const float mu = sum / (float)D;
+    float var = 0.f;
+    for (int c = lane; c < Dp; c += 32) {
+      const bool valid = c < dn || (c >= s1 && c < s1 + de) || (c >= s2 && c < s2 + dt);
+      if (valid) {
+        const float d = yr[c] - mu;
+        var = fmaf(d, d, var);
+      }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) var += __shfl_xor_sync(0xffffffffu, var, o);
+    const float rstd = rsqrtf(var / (float)D + 1e-5f);
+    for (int c = lane; c < Dp; c += 32) {
+      const bool valid = c < dn || (c >= s1 && c < s1 + de) || (c >= s2 && c < s2 + dt);
+      rr[c] = valid ? (yr[c] - mu) * rstd * gamma[c] + beta[c] : 0.f;
+    }
+  }
+}
+
+void launch_layernorm(const float* y, float* r, int Dp, int dn, int dnp, int de, int dep, int dt,
+                      const float* gamma, const float* beta, const int* m_dev, int m_max, cudaStream_t st) {
+  int blocks = (m_max * 32 + 255) / 256;
+  if (blocks < 1) blocks = 1;
+  if (blocks > 1184) blocks = 1184;
+  k_layernorm<<<blocks, 256, 0, st>>>(y, r, Dp, dn, dnp, de, dep, dt, gamma, beta, m_dev);
+}
+
+// -------------------------------------------------------------------- score
+__global__ void k_score(const float* __restrict__ HL, int ldh, const int32_t* __restrict__ inv, int64_t n_edges,
+                        int batch, const int* __restrict__ bidx, const float* __restrict__ Wa1,
+                        const float* __restrict__ ba1, const float* __restrict__ Wa2, float ba2, int dn, int dnp,
+                        float* __restrict__ scores) {
+  extern __shared__ float x[];  // [2 dnp]
+  __shared__ float red[32];
+  const int64_t lo = bidx ? (int64_t)(*bidx) * batch : 0;
+  const int64_t rem = n_edges - lo;
+  const int B = (int)(rem < batch ? (rem < 0 ? 0 : rem) : batch);
+  for (int e = blockIdx.x; e < B; e += gridDim.x) {
+    const float* hs = HL + (size_t)inv[e] * ldh;       // DedupInvert (Alg. 1 l.20)
+    const float* hd = HL + (size_t)inv[B + e] * ldh;
+    for (int c = threadIdx.x; c < dnp; c += blockDim.x) {
+      x[c] = hs[c];
+      x[dnp + c] = hd[c];
+    }
+    __syncthreads();
+    float part = 0.f;
+    for (int j = threadIdx.x; j < dn; j += blockDim.x) {
+      const float4* w = reinterpret_cast<const float4*>(Wa1 + (size_t)j * 2 * dnp);
+      const float4* xv = reinterpret_cast<const float4*>(x);
+      float z = 0.f;
+      for (int q = 0; q < (2 * dnp) / 4; ++q) {
+        const float4 a = w[q], b = xv[q];
+        z = fmaf(a.x, b.x, z);
+        z = fmaf(a.y, b.y, z);
+        z = fmaf(a.z, b.z, z);
+        z = fmaf(a.w, b.w, z);
+      }
+      z = fmaxf(z + ba1[j], 0.f);
+      part = fmaf(Wa2[j], z, part);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = part;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      float s = 0.f;
+      for (int w = 0; w < (int)(blockDim.x >> 5); ++w) s += red[w];
+      const float logit = s + ba2;
+      scores[lo + e] = 1.f / (1.f + expf(-logit));
+    }
+    __syncthreads();
+  }
+}
+
+void launch_score(const float* HL, int ldh, const int32_t* inv, int n_edges, int batch, const int* bidx,
+                  const float* Wa1, const float* ba1, const float* Wa2, float ba2, int dn, int dnp,
+                  float* scores, cudaStream_t st) {
+  int blocks = batch < 592 ? batch : 592;
+  if (blocks < 1) blocks = 1;
+  k_score<<<blocks, 128, 2 * dnp * sizeof(float), st>>>(HL, ldh, inv, n_edges, batch, bidx, Wa1, ba1, Wa2, ba2, dn,
+                                                        dnp, scores);
+}
+
+__global__ void k_invert(const float* __restrict__ HL, int ldh, const int32_t* __restrict__ inv, int n, int dn,
+                         float* __restrict__ out) {
+  const long long tot = (long long)n * dn;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < tot; i += (long long)gridDim.x * blockDim.x) {
+    const long long r = i / dn;
+    const int c = (int)(i - r * dn);
+    out[i] = HL[(size_t)inv[r] * ldh + c];
+  }
+}
+
+void launch_invert(const float* HL, int ldh, const int32_t* inv, int n, int dn, float* out, cudaStream_t st) {
+  if (n <= 0) return;
+  long long tot = (long long)n * dn;
+  int blocks = (int)((tot + 255) / 256);
+  if (blocks > 1184) blocks = 1184;
+  k_invert<<<blocks, 256, 0, st>>>(HL, ldh, inv, n, dn, out);
+}
+
+}  // namespace tg

@@ -1,0 +1,946 @@
+// C ABI of libtg (include/tg.h): context, loading, and the per-batch
+// orchestration of Alg. 1 as a chain of stream-ordered sm_100a
+// kernels with device-resident counts (no host sync inside a batch).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <vector>
+
+#include "tg_internal.cuh"
+#include "tg_tc.cuh"
+
+using namespace tg;
+
+namespace {
+
+struct LayerW {
+  float *P = nullptr, *bu = nullptr, *F = nullptr, *bfc = nullptr, *lng = nullptr, *lnb = nullptr;
+  float *W1 = nullptr, *b1 = nullptr, *W2 = nullptr, *b2 = nullptr;
+  TcWeights tcP, tcF, tcW1, tcW2;  // tensor-core operand copies (TG_PREC_TF32X3 / BF16)
+};
+
+}  // namespace
+
+struct tg_ctx {
+  int device = 0;
+  bool broken = false;
+  // graph
+  GraphDev g{};
+  int32_t *rowptr = nullptr, *adj_nbr = nullptr, *adj_eid = nullptr;
+  uint32_t* adj_t = nullptr;
+  float *X = nullptr, *Ef = nullptr;
+  // model
+  bool loaded = false;
+  tg_model_cfg cfg{};
+  int L = 0, H = 0, k = 0, d_n = 0, d_e = 0, d_t = 0, dnp = 0, dep = 0, dtp = 0, Dp = 0, W = 0;
+  LayerW lw[TG_MAX_LAYERS];
+  float *omega = nullptr, *phi = nullptr, *table = nullptr;
+  float *Wa1 = nullptr, *ba1 = nullptr, *Wa2 = nullptr;
+  float ba2 = 0.f;
+  // recursion levels
+  Level I[TG_MAX_LAYERS + 1]{}, U[TG_MAX_LAYERS + 1]{}, C[TG_MAX_LAYERS + 1]{};
+  int capI[TG_MAX_LAYERS + 1]{};
+  int32_t *inv[TG_MAX_LAYERS + 1]{}, *cuidx[TG_MAX_LAYERS + 1]{}, *eid[TG_MAX_LAYERS + 1]{};
+  long long* slot[TG_MAX_LAYERS + 1]{};
+  int* counts = nullptr;  // device: [3*l + 0] |I_l|, [3*l+1] |U_l|, [3*l+2] |C_l|
+  CacheDev cache[TG_MAX_LAYERS]{};
+  long long* cache_state = nullptr;  // [TG_MAX_LAYERS * 4]
+  int64_t limit0 = 0;
+  // compute workspace
+  int maxC = 0, maxRows = 0;
+  float *u = nullptr, *c = nullptr, *y = nullptr, *r = nullptr, *z = nullptr, *HL = nullptr;
+  const float** rows = nullptr;
+  float** dst = nullptr;
+  // counters / flags
+  long long* cnt_total = nullptr;
+  long long* cnt_tmp = nullptr;
+  int* err = nullptr;
+  int* bidx = nullptr;
+  int64_t launches = 0;
+  // per-stage profiling (events around launches)
+  bool prof = false;
+  std::vector<cudaEvent_t> ev_pool;
+  std::vector<int> ev_stage;  // stage of event pair i (events 2i, 2i+1)
+  size_t ev_used = 0;
+  // staging for host buffers
+  void* stage = nullptr;
+  size_t stage_bytes = 0;
+  std::vector<void*> owned;
+};
+
+namespace {
+
+#define CK(x)                                                                                      \
+  do {                                                                                             \
+    cudaError_t e_ = (x);                                                                          \
+    if (e_ != cudaSuccess) {                                                                       \
+      fprintf(stderr, "libtg: CUDA error %s at %s:%d\n", cudaGetErrorString(e_), __FILE__, __LINE__); \
+      return e_ == cudaErrorMemoryAllocation ? TG_ENOMEM : TG_ECUDA;                               \
+    }                                                                                              \
+  } while (0)
+
+template <class T>
+tg_status dalloc(tg_ctx* ctx, T** p, size_t n) {
+  void* q = nullptr;
+  if (n == 0) n = 1;
+  cudaError_t e = cudaMalloc(&q, n * sizeof(T));
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return TG_ENOMEM;
+  }
+  ctx->owned.push_back(q);
+  *p = reinterpret_cast<T*>(q);
+  return TG_OK;
+}
+
+#define TRY(x)                \
+  do {                        \
+    tg_status s_ = (x);       \
+    if (s_ != TG_OK) return s_; \
+  } while (0)
+
+bool is_device_ptr(const void* p) {
+  if (!p) return false;
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+// Bracket the next launch with an event pair when profiling is on.
+struct Prof {
+  tg_ctx* ctx;
+  cudaEvent_t e1 = nullptr;
+  Prof(tg_ctx* c, int stage, cudaStream_t st) : ctx(c) {
+    if (!c->prof) return;
+    if (c->ev_used * 2 + 2 > c->ev_pool.size()) {
+      for (int i = 0; i < 256; ++i) {
+        cudaEvent_t e;
+        cudaEventCreate(&e);
+        c->ev_pool.push_back(e);
+      }
+    }
+    cudaEvent_t e0 = c->ev_pool[2 * c->ev_used];
+    e1 = c->ev_pool[2 * c->ev_used + 1];
+    if (c->ev_stage.size() <= c->ev_used) c->ev_stage.resize(c->ev_used + 1);
+    c->ev_stage[c->ev_used] = stage;
+    ++c->ev_used;
+    cudaEventRecord(e0, st);
+    stream = st;
+  }
+  cudaStream_t stream = nullptr;
+  ~Prof() {
+    if (e1) cudaEventRecord(e1, stream);
+  }
+};
+
+tg_status launched(tg_ctx* ctx, int n = 1) {
+  ctx->launches += n;
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) {
+    fprintf(stderr, "libtg: launch error %s\n", cudaGetErrorString(e));
+    ctx->broken = true;
+    return TG_ECUDA;
+  }
+  return TG_OK;
+}
+
+tg_status ensure_stage(tg_ctx* ctx, size_t bytes) {
+  if (ctx->stage_bytes >= bytes) return TG_OK;
+  if (ctx->stage) cudaFree(ctx->stage);
+  ctx->stage = nullptr;
+  ctx->stage_bytes = 0;
+  CK(cudaMalloc(&ctx->stage, bytes));
+  ctx->stage_bytes = bytes;
+  return TG_OK;
+}
+
+inline int pc(const tg_ctx* ctx, int a) {  // D-space index -> padded kv index
+  if (a < ctx->d_n) return a;
+  if (a < ctx->d_n + ctx->d_e) return ctx->dnp + (a - ctx->d_n);
+  return ctx->dnp + ctx->dep + (a - ctx->d_n - ctx->d_e);
+}
+
+void free_model(tg_ctx* ctx) {
+  // model buffers are in ctx->owned after the graph's; freed with the context
+  (void)ctx;
+}
+
+// ------------------------------------------------------------------------
+// One Embed(L, I_L) pass (Alg. 1), I_L already in ctx->I[L] with its count.
+// ------------------------------------------------------------------------
+tg_status run_embed(tg_ctx* ctx, long long* cnt, cudaStream_t st) {
+  const int L = ctx->L, k = ctx->k;
+  const bool dedup = ctx->cfg.opts & TG_OPT_DEDUP;
+  const bool cache_on = ctx->cfg.opts & TG_OPT_CACHE;
+  int* cnts = ctx->counts;
+  auto nI = [&](int l) { return cnts + 3 * l + 0; };
+  auto nU = [&](int l) { return cnts + 3 * l + 1; };
+  auto nC = [&](int l) { return cnts + 3 * l + 2; };
+  auto cl = [&](int l) { return cnt + l * TG_CNT_PER_LAYER; };
+  // ---- top-down: dedup, lookup, sampling (Alg. 1 l.5-12)
+  for (int l = L; l >= 1; --l) {
+    {
+      Prof pf(ctx, TG_ST_DEDUP, st);
+      launch_dedup(ctx->I[l], nI(l), ctx->capI[l], ctx->U[l], ctx->inv[l], nU(l), cl(l) + 0, cl(l) + 1, dedup,
+                   ctx->err, st);
+    }
+    TRY(launched(ctx));
+    {
+      Prof pf(ctx, TG_ST_LOOKUP, st);
+      if (l == L) {
+        launch_copy_level(ctx->U[l], nU(l), ctx->capI[l], ctx->C[l], ctx->cuidx[l], nC(l), cl(l) + 4, st);
+      } else {
+        launch_probe(ctx->U[l], nU(l), ctx->capI[l], ctx->cache[l], cache_on, ctx->cuidx[l], ctx->C[l], nC(l),
+                     ctx->slot[l], cl(l), ctx->err, st);
+      }
+    }
+    TRY(launched(ctx));
+    {
+      Prof pf(ctx, TG_ST_SAMPLE, st);
+      launch_sample(ctx->g, ctx->C[l], nC(l), ctx->capI[l], k, ctx->I[l - 1], ctx->eid[l], nI(l - 1), ctx->err,
+                    st);
+    }
+    TRY(launched(ctx));
+  }
+  // ---- bottom-up: M and FFN for every computed target (Alg. 1 l.13-18)
+  for (int l = 1; l <= L; ++l) {
+    const LayerW& w = ctx->lw[l - 1];
+    const bool top = (l == L);
+    { Prof pf(ctx, TG_ST_RESOLVE, st);
+    launch_resolve(ctx->g, l == 1, ctx->I[l - 1], nI(l - 1), ctx->capI[l - 1], ctx->inv[l - 1], ctx->slot[l - 1],
+                   l == 1 ? nullptr : ctx->cache[l - 1].ring, 0, ctx->dnp, nC(l), ctx->capI[l], ctx->cuidx[l],
+                   ctx->slot[l], top ? nullptr : ctx->cache[l].ring, 0, ctx->HL, ctx->rows, ctx->dst, ctx->err, st); }
+    TRY(launched(ctx));
+    const int HDp = ctx->H * ctx->Dp;
+    const int mmax = ctx->capI[l];
+    const bool tc = ctx->cfg.precision != TG_PREC_FP32;
+    // G1: u = P hs + bu  (target-side K projection, scale folded)
+    GemmArgs g1{};
+    g1.a_rows0 = ctx->rows;
+    g1.K0 = g1.K = ctx->dnp;
+    g1.B = w.P;
+    g1.N = HDp;
+    g1.bias = w.bu;
+    g1.C = ctx->u;
+    g1.ldc = HDp;
+    g1.m_dev = nC(l);
+    g1.m_max = mmax;
+    { Prof pf(ctx, TG_ST_PROJ_K, st);
+      if (tc) launch_gemm_tc(g1, w.tcP, ctx->cfg.precision, st); else launch_gemm_simt(g1, st); }
+    TRY(launched(ctx));
+    // attention over the k neighbours
+    AttnArgs a{};
+    a.u = ctx->u;
+    a.c = ctx->c;
+    a.rows = ctx->rows;
+    a.prev_node = ctx->I[l - 1].node;
+    a.prev_ts = ctx->I[l - 1].ts;
+    a.eid = ctx->eid[l];
+    a.Ef = ctx->Ef;
+    a.lde = ctx->g.lde;
+    a.omega = ctx->omega;
+    a.phi = ctx->phi;
+    a.table = ctx->table;
+    a.W = ctx->W;
+    a.use_table = (ctx->cfg.opts & TG_OPT_TTABLE) ? 1 : 0;
+    a.dnp = ctx->dnp;
+    a.dep = ctx->dep;
+    a.dtp = ctx->dtp;
+    a.d_t = ctx->d_t;
+    a.Dp = ctx->Dp;
+    a.H = ctx->H;
+    a.k = k;
+    a.nc_dev = nC(l);
+    a.nc_max = mmax;
+    a.cnt_ttable = cnt + TG_CNT_TTABLE;
+    { Prof pf(ctx, TG_ST_ATTN, st); launch_attn(a, st); }
+    TRY(launched(ctx));
+    // G2: y = F c + b_fc + q   (value projection and W_fc folded; residual q, Eq. 4)
+    GemmArgs g2{};
+    g2.a_base0 = ctx->c;
+    g2.lda0 = HDp;
+    g2.K0 = g2.K = HDp;
+    g2.B = w.F;
+    g2.N = ctx->Dp;
+    g2.bias = w.bfc;
+    g2.q_rows = ctx->rows;
+    g2.q_dnp = ctx->dnp;
+    g2.q_dep = ctx->dep;
+    g2.q_phi0 = ctx->table;  // Phi(0): row 0 of the table
+    g2.C = ctx->y;
+    g2.ldc = ctx->Dp;
+    g2.m_dev = nC(l);
+    g2.m_max = mmax;
+    { Prof pf(ctx, TG_ST_PROJ_V, st);
+      if (tc) launch_gemm_tc(g2, w.tcF, ctx->cfg.precision, st); else launch_gemm_simt(g2, st); }
+    TRY(launched(ctx));
+    { Prof pf(ctx, TG_ST_LNORM, st);
+    launch_layernorm(ctx->y, ctx->r, ctx->Dp, ctx->d_n, ctx->dnp, ctx->d_e, ctx->dep, ctx->d_t, w.lng, w.lnb,
+                     nC(l), mmax, st); }
+    TRY(launched(ctx));
+    // G3: z = ReLU(W1 [r || hs] + b1)   (Eq. 7)
+    GemmArgs g3{};
+    g3.a_base0 = ctx->r;
+    g3.lda0 = ctx->Dp;
+    g3.K0 = ctx->Dp;
+    g3.a_rows1 = ctx->rows;
+    g3.K = ctx->Dp + ctx->dnp;
+    g3.B = w.W1;
+    g3.N = ctx->dnp;
+    g3.bias = w.b1;
+    g3.relu = 1;
+    g3.C = ctx->z;
+    g3.ldc = ctx->dnp;
+    g3.m_dev = nC(l);
+    g3.m_max = mmax;
+    { Prof pf(ctx, TG_ST_FFN1, st);
+      if (tc) launch_gemm_tc(g3, w.tcW1, ctx->cfg.precision, st); else launch_gemm_simt(g3, st); }
+    TRY(launched(ctx));
+    // G4: h = W2 z + b2 -> cache ring slot (CacheStore payload, Alg. 3 l.8-10) or H_L
+    GemmArgs g4{};
+    g4.a_base0 = ctx->z;
+    g4.lda0 = ctx->dnp;
+    g4.K0 = g4.K = ctx->dnp;
+    g4.B = w.W2;
+    g4.N = ctx->dnp;
+    g4.bias = w.b2;
+    g4.c_rows = ctx->dst;
+    g4.m_dev = nC(l);
+    g4.m_max = mmax;
+    { Prof pf(ctx, TG_ST_FFN2, st);
+      if (tc) launch_gemm_tc(g4, w.tcW2, ctx->cfg.precision, st); else launch_gemm_simt(g4, st); }
+    TRY(launched(ctx));
+  }
+  return TG_OK;
+}
+
+// level-0 input count: added once the sampler of level 1 has run
+__global__ void k_count_l0(const int* n0, long long* c0) {
+  atomicAdd((unsigned long long*)c0, (unsigned long long)*n0);
+}
+
+tg_status run_embed_counted(tg_ctx* ctx, long long* cnt, cudaStream_t st) {
+  TRY(run_embed(ctx, cnt, st));
+  {
+    Prof pf(ctx, TG_ST_OTHER, st);
+    k_count_l0<<<1, 1, 0, st>>>(ctx->counts + 0, cnt + 0);
+  }
+  return launched(ctx);
+}
+
+__global__ void k_finish_batch(long long* __restrict__ tmp, long long* __restrict__ total,
+                               long long* __restrict__ log, int* __restrict__ bidx, int n) {
+  const int i = threadIdx.x;
+  if (i < n) {
+    const long long v = tmp[i];
+    total[i] += v;
+    if (log) log[(long long)(*bidx) * n + i] = v;
+    tmp[i] = 0;
+  }
+  __syncthreads();
+  if (i == 0) *bidx += 1;
+}
+
+}  // namespace
+
+// =========================================================================
+extern "C" {
+
+const char* tg_strerror(tg_status s) {
+  switch (s) {
+    case TG_OK: return "ok";
+    case TG_EINVAL: return "invalid argument";
+    case TG_ENOMEM: return "out of memory";
+    case TG_ECUDA: return "CUDA error";
+    case TG_ESTATE: return "call out of order";
+    case TG_EORDER: return "timestamps not non-decreasing";
+    case TG_EDEVICE: return "device-side error flag set (id out of range or table full)";
+  }
+  return "unknown";
+}
+
+const char* tg_version(void) { return "libtg 0.1 sm_100a (fp32 SIMT, tf32x3/bf16 tcgen05)"; }
+
+int64_t tg_kernel_launches(tg_ctx* ctx) { return ctx ? ctx->launches : 0; }
+
+tg_status tg_graph_load(int device, const tg_graph_desc* gd, tg_ctx** out) {
+  if (!gd || !out) return TG_EINVAL;
+  *out = nullptr;
+  if (gd->n_nodes < 0 || gd->n_edges < 0 || gd->d_n < 1 || gd->d_e < 1) return TG_EINVAL;
+  if (gd->n_edges > 0 && (!gd->src || !gd->dst || !gd->ts)) return TG_EINVAL;
+  if (!gd->node_feat || !gd->edge_feat) return TG_EINVAL;
+  if (2 * gd->n_edges >= (int64_t)INT32_MAX || gd->n_nodes >= (int64_t)INT32_MAX) return TG_EINVAL;
+  const int64_t V = gd->n_nodes, E = gd->n_edges;
+  for (int64_t i = 0; i < E; ++i) {
+    if (gd->src[i] < 1 || gd->src[i] > V || gd->dst[i] < 1 || gd->dst[i] > V) return TG_EINVAL;
+    if (i && gd->ts[i] < gd->ts[i - 1]) return TG_EORDER;
+  }
+  if (cudaSetDevice(device) != cudaSuccess) return TG_ECUDA;
+  tg_ctx* ctx = new (std::nothrow) tg_ctx();
+  if (!ctx) return TG_ENOMEM;
+  ctx->device = device;
+  // ---- T-CSR on the host: counting sort by node; edges are already in
+  // (t, edge id) order, so appending keeps each adjacency sorted (R6).
+  std::vector<int32_t> rowptr(V + 2, 0);
+  for (int64_t i = 0; i < E; ++i) {
+    rowptr[gd->src[i] + 1]++;
+    rowptr[gd->dst[i] + 1]++;
+  }
+  for (int64_t v = 0; v <= V; ++v) rowptr[v + 1] += rowptr[v];
+  std::vector<int32_t> fill(rowptr.begin(), rowptr.end() - 1);
+  std::vector<int32_t> nbr(2 * E), eid(2 * E);
+  std::vector<uint32_t> tt(2 * E);
+  for (int64_t i = 0; i < E; ++i) {
+    const int32_t s = gd->src[i], d = gd->dst[i];
+    int32_t p = fill[s]++;
+    nbr[p] = d;
+    eid[p] = (int32_t)(i + 1);
+    tt[p] = gd->ts[i];
+    p = fill[d]++;
+    nbr[p] = s;
+    eid[p] = (int32_t)(i + 1);
+    tt[p] = gd->ts[i];
+  }
+  tg_status s;
+#define TRYF(x)       \
+  do {                \
+    s = (x);          \
+    if (s != TG_OK) { \
+      tg_free(ctx);   \
+      return s;       \
+    }                 \
+  } while (0)
+  TRYF(dalloc(ctx, &ctx->rowptr, V + 2));
+  TRYF(dalloc(ctx, &ctx->adj_nbr, 2 * E));
+  TRYF(dalloc(ctx, &ctx->adj_eid, 2 * E));
+  TRYF(dalloc(ctx, &ctx->adj_t, 2 * E));
+  cudaMemcpy(ctx->rowptr, rowptr.data(), (V + 2) * 4, cudaMemcpyHostToDevice);
+  if (E) {
+    cudaMemcpy(ctx->adj_nbr, nbr.data(), 2 * E * 4, cudaMemcpyHostToDevice);
+    cudaMemcpy(ctx->adj_eid, eid.data(), 2 * E * 4, cudaMemcpyHostToDevice);
+    cudaMemcpy(ctx->adj_t, tt.data(), 2 * E * 4, cudaMemcpyHostToDevice);
+  }
+  const int ldn = round4(gd->d_n), lde = round4(gd->d_e);
+  TRYF(dalloc(ctx, &ctx->X, (size_t)(V + 1) * ldn));
+  TRYF(dalloc(ctx, &ctx->Ef, (size_t)(E + 1) * lde));
+  cudaMemset(ctx->X, 0, (size_t)(V + 1) * ldn * 4);
+  cudaMemset(ctx->Ef, 0, (size_t)(E + 1) * lde * 4);
+  // padded row copies; row 0 stays zero
+  if (V > 0)
+    cudaMemcpy2D(ctx->X + ldn, ldn * 4, gd->node_feat + gd->d_n, gd->d_n * 4, gd->d_n * 4, V, cudaMemcpyHostToDevice);
+  if (E > 0)
+    cudaMemcpy2D(ctx->Ef + lde, lde * 4, gd->edge_feat + gd->d_e, gd->d_e * 4, gd->d_e * 4, E,
+                 cudaMemcpyHostToDevice);
+  if (cudaDeviceSynchronize() != cudaSuccess) {
+    tg_free(ctx);
+    return TG_ECUDA;
+  }
+  GraphDev& g = ctx->g;
+  g.V = V;
+  g.E = E;
+  g.rowptr = ctx->rowptr;
+  g.adj_nbr = ctx->adj_nbr;
+  g.adj_eid = ctx->adj_eid;
+  g.adj_t = ctx->adj_t;
+  g.X = ctx->X;
+  g.Ef = ctx->Ef;
+  g.d_n = gd->d_n;
+  g.d_e = gd->d_e;
+  g.ldn = ldn;
+  g.lde = lde;
+  TRYF(dalloc(ctx, &ctx->err, 1));
+  cudaMemset(ctx->err, 0, sizeof(int));
+  *out = ctx;
+  return TG_OK;
+#undef TRYF
+}
+
+tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* params, int64_t n_params) {
+  if (!ctx || !cfg || !params) return TG_EINVAL;
+  if (ctx->broken) return TG_ECUDA;
+  if (ctx->loaded) return TG_ESTATE;  // one model per context (create a new context to replace it)
+  const int L = cfg->n_layers, H = cfg->n_heads, k = cfg->n_neighbors, d_t = cfg->d_t;
+  const int d_n = ctx->g.d_n, d_e = ctx->g.d_e;
+  const int D = d_n + d_e + d_t;
+  if (L < 1 || L > TG_MAX_LAYERS || H < 1 || k < 1 || k > kMaxK || d_t < 1 || D % H) return TG_EINVAL;
+  if (cfg->max_batch_targets < 1 || cfg->cache_limit < 0 || cfg->time_window < 0) return TG_EINVAL;
+  if (cfg->precision < TG_PREC_FP32 || cfg->precision > TG_PREC_BF16) return TG_EINVAL;
+  const int64_t per_layer = 4LL * D * D + 3LL * D + (int64_t)d_n * (D + d_n) + d_n + (int64_t)d_n * d_n + d_n;
+  const int64_t expect = L * per_layer + 2LL * d_t + 2LL * d_n * d_n + d_n + d_n + 1;
+  if (n_params != expect) return TG_EINVAL;
+  // workspace capacities: I_L = targets, I_{l-1} = C_l (k+1) <= I_l (k+1)
+  int64_t cap = cfg->max_batch_targets;
+  int capI[TG_MAX_LAYERS + 1];
+  capI[L] = (int)cap;
+  for (int l = L - 1; l >= 0; --l) {
+    cap = cap * (k + 1);
+    if (cap > (int64_t)1 << 26) return TG_EINVAL;
+    capI[l] = (int)cap;
+  }
+  for (int l = 1; l <= L; ++l) {
+    if (capI[l] > 16 * 10000) return TG_EINVAL;                        // dedup cluster bound
+    if (l < L && capI[l] > kDedupThreads * kDedupIPT) return TG_EINVAL;  // probe CTA bound
+  }
+  if (cudaSetDevice(ctx->device) != cudaSuccess) return TG_ECUDA;
+  ctx->cfg = *cfg;
+  ctx->L = L;
+  ctx->H = H;
+  ctx->k = k;
+  ctx->d_n = d_n;
+  ctx->d_e = d_e;
+  ctx->d_t = d_t;
+  ctx->dnp = round4(d_n);
+  ctx->dep = round4(d_e);
+  ctx->dtp = round4(d_t);
+  ctx->Dp = ctx->dnp + ctx->dep + ctx->dtp;
+  ctx->W = cfg->time_window;
+  const int dnp = ctx->dnp, Dp = ctx->Dp, dk = D / H;
+  const int HDp = H * Dp;
+  // ---- time encoder: Phi table [max(W,1) x dtp] on device; Phi(0) = row 0
+  const float* om = params + L * per_layer;
+  const float* ph = om + d_t;
+  TRY(dalloc(ctx, &ctx->omega, d_t));
+  TRY(dalloc(ctx, &ctx->phi, d_t));
+  const int Wrows = std::max(ctx->W, 1);
+  TRY(dalloc(ctx, &ctx->table, (size_t)Wrows * ctx->dtp));
+  CK(cudaMemcpy(ctx->omega, om, d_t * 4, cudaMemcpyHostToDevice));
+  CK(cudaMemcpy(ctx->phi, ph, d_t * 4, cudaMemcpyHostToDevice));
+  launch_time_table(ctx->omega, ctx->phi, d_t, ctx->dtp, Wrows, ctx->table, 0);
+  CK(cudaGetLastError());
+  std::vector<float> phi0(ctx->dtp);
+  CK(cudaMemcpy(phi0.data(), ctx->table, ctx->dtp * 4, cudaMemcpyDeviceToHost));
+  // ---- per-layer weights, folded in float64 on the host (load time only)
+  const double isq = 1.0 / std::sqrt((double)dk);
+  for (int l = 0; l < L; ++l) {
+    const float* base = params + l * per_layer;
+    const float* Wq = base;
+    const float* Wk = Wq + (size_t)D * D;
+    const float* Wv = Wk + (size_t)D * D;
+    const float* Wfc = Wv + (size_t)D * D;
+    const float* bfc = Wfc + (size_t)D * D;
+    const float* lng = bfc + D;
+    const float* lnb = lng + D;
+    const float* Wm1 = lnb + D;
+    const float* bm1 = Wm1 + (size_t)d_n * (D + d_n);
+    const float* Wm2 = bm1 + d_n;
+    const float* bm2 = Wm2 + (size_t)d_n * d_n;
+    std::vector<double> P((size_t)HDp * dnp, 0.0), bu(HDp, 0.0), F((size_t)Dp * HDp, 0.0);
+    std::vector<double> qc(D, 0.0);  // W_q[:, Phi block] Phi(0)
+    for (int r = 0; r < D; ++r)
+      for (int c = d_n + d_e; c < D; ++c) qc[r] += (double)Wq[(size_t)r * D + c] * phi0[c - d_n - d_e];
+    for (int h = 0; h < H; ++h) {
+      for (int r = h * dk; r < (h + 1) * dk; ++r) {
+        const float* wq = Wq + (size_t)r * D;
+        const float* wk = Wk + (size_t)r * D;
+        for (int a = 0; a < D; ++a) {
+          const double wka = wk[a];
+          double* prow = &P[((size_t)h * Dp + pc(ctx, a)) * dnp];
+          for (int b = 0; b < d_n; ++b) prow[b] += wka * wq[b];
+          bu[(size_t)h * Dp + pc(ctx, a)] += wka * qc[r];
+        }
+      }
+    }
+    for (auto& v : P) v *= isq;
+    for (auto& v : bu) v *= isq;
+    for (int o = 0; o < D; ++o) {
+      double* frow = &F[(size_t)pc(ctx, o) * HDp];
+      for (int h = 0; h < H; ++h)
+        for (int r = h * dk; r < (h + 1) * dk; ++r) {
+          const double w = Wfc[(size_t)o * D + r];
+          const float* wv = Wv + (size_t)r * D;
+          for (int a = 0; a < D; ++a) frow[(size_t)h * Dp + pc(ctx, a)] += w * wv[a];
+        }
+    }
+    std::vector<float> Pf(P.begin(), P.end()), buf(bu.begin(), bu.end()), Ff(F.begin(), F.end());
+    std::vector<float> bfcp(Dp, 0.f), lngp(Dp, 0.f), lnbp(Dp, 0.f);
+    for (int a = 0; a < D; ++a) {
+      bfcp[pc(ctx, a)] = bfc[a];
+      lngp[pc(ctx, a)] = lng[a];
+      lnbp[pc(ctx, a)] = lnb[a];
+    }
+    const int K3 = Dp + dnp;
+    std::vector<float> W1p((size_t)dnp * K3, 0.f), b1p(dnp, 0.f), W2p((size_t)dnp * dnp, 0.f), b2p(dnp, 0.f);
+    for (int j = 0; j < d_n; ++j) {
+      for (int a = 0; a < D; ++a) W1p[(size_t)j * K3 + pc(ctx, a)] = Wm1[(size_t)j * (D + d_n) + a];
+      for (int b = 0; b < d_n; ++b) W1p[(size_t)j * K3 + Dp + b] = Wm1[(size_t)j * (D + d_n) + D + b];
+      b1p[j] = bm1[j];
+      for (int b = 0; b < d_n; ++b) W2p[(size_t)j * dnp + b] = Wm2[(size_t)j * d_n + b];
+      b2p[j] = bm2[j];
+    }
+    LayerW& w = ctx->lw[l];
+    auto up = [&](float** dptr, const std::vector<float>& v) -> tg_status {
+      TRY(dalloc(ctx, dptr, v.size()));
+      CK(cudaMemcpy(*dptr, v.data(), v.size() * 4, cudaMemcpyHostToDevice));
+      return TG_OK;
+    };
+    TRY(up(&w.P, Pf));
+    TRY(up(&w.bu, buf));
+    TRY(up(&w.F, Ff));
+    TRY(up(&w.bfc, bfcp));
+    TRY(up(&w.lng, lngp));
+    TRY(up(&w.lnb, lnbp));
+    TRY(up(&w.W1, W1p));
+    TRY(up(&w.b1, b1p));
+    TRY(up(&w.W2, W2p));
+    TRY(up(&w.b2, b2p));
+    if (cfg->precision != TG_PREC_FP32) {
+      TRY(tc_prepare_weights(w.P, HDp, dnp, cfg->precision, &w.tcP, ctx->owned));
+      TRY(tc_prepare_weights(w.F, Dp, HDp, cfg->precision, &w.tcF, ctx->owned));
+      TRY(tc_prepare_weights(w.W1, dnp, K3, cfg->precision, &w.tcW1, ctx->owned));
+      TRY(tc_prepare_weights(w.W2, dnp, dnp, cfg->precision, &w.tcW2, ctx->owned));
+    }
+  }
+  // ---- affinity score MLP (R10), padded
+  {
+    const float* Wa1 = ph + d_t;
+    const float* ba1 = Wa1 + (size_t)d_n * 2 * d_n;
+    const float* Wa2 = ba1 + d_n;
+    const float* ba2 = Wa2 + d_n;
+    std::vector<float> W((size_t)dnp * 2 * dnp, 0.f), b(dnp, 0.f), w2(dnp, 0.f);
+    for (int j = 0; j < d_n; ++j) {
+      for (int a = 0; a < d_n; ++a) {
+        W[(size_t)j * 2 * dnp + a] = Wa1[(size_t)j * 2 * d_n + a];
+        W[(size_t)j * 2 * dnp + dnp + a] = Wa1[(size_t)j * 2 * d_n + d_n + a];
+      }
+      b[j] = ba1[j];
+      w2[j] = Wa2[j];
+    }
+    TRY(dalloc(ctx, &ctx->Wa1, W.size()));
+    TRY(dalloc(ctx, &ctx->ba1, b.size()));
+    TRY(dalloc(ctx, &ctx->Wa2, w2.size()));
+    CK(cudaMemcpy(ctx->Wa1, W.data(), W.size() * 4, cudaMemcpyHostToDevice));
+    CK(cudaMemcpy(ctx->ba1, b.data(), b.size() * 4, cudaMemcpyHostToDevice));
+    CK(cudaMemcpy(ctx->Wa2, w2.data(), w2.size() * 4, cudaMemcpyHostToDevice));
+    ctx->ba2 = ba2[0];
+  }
+  // ---- recursion-level workspaces
+  for (int l = 0; l <= L; ++l) {
+    ctx->capI[l] = capI[l];
+    TRY(dalloc(ctx, &ctx->I[l].node, capI[l]));
+    TRY(dalloc(ctx, &ctx->I[l].ts, capI[l]));
+    ctx->I[l].cap = capI[l];
+    if (l >= 1) {
+      TRY(dalloc(ctx, &ctx->U[l].node, capI[l]));
+      TRY(dalloc(ctx, &ctx->U[l].ts, capI[l]));
+      TRY(dalloc(ctx, &ctx->C[l].node, capI[l]));
+      TRY(dalloc(ctx, &ctx->C[l].ts, capI[l]));
+      ctx->U[l].cap = ctx->C[l].cap = capI[l];
+      TRY(dalloc(ctx, &ctx->inv[l], capI[l]));
+      TRY(dalloc(ctx, &ctx->cuidx[l], capI[l]));
+      TRY(dalloc(ctx, &ctx->slot[l], capI[l]));
+      TRY(dalloc(ctx, &ctx->eid[l], (size_t)capI[l] * k));
+    }
+  }
+  TRY(dalloc(ctx, &ctx->counts, 3 * (TG_MAX_LAYERS + 1)));
+  CK(cudaMemset(ctx->counts, 0, 3 * (TG_MAX_LAYERS + 1) * sizeof(int)));
+  // ---- caches for layers 1..L-1: index (load <= 1/4 of live items) + FIFO ring
+  TRY(dalloc(ctx, &ctx->cache_state, 4 * TG_MAX_LAYERS));
+  ctx->limit0 = cfg->cache_limit;
+  for (int l = 1; l < L; ++l) {
+    CacheDev& cd = ctx->cache[l];
+    const long long rcap = cfg->cache_limit + 2LL * capI[l] + 16;
+    unsigned long long icap = 1024;
+    while (icap < 4ull * (unsigned long long)(cfg->cache_limit + capI[l])) icap <<= 1;
+    TRY(dalloc(ctx, &cd.ikey, icap));
+    TRY(dalloc(ctx, &cd.ipos, icap));
+    TRY(dalloc(ctx, &cd.ring, (size_t)rcap * dnp));
+    cd.imask = icap - 1;
+    cd.rcap = rcap;
+    cd.state = ctx->cache_state + 4 * l;
+  }
+  // ---- compute workspace
+  int maxC = 0;
+  for (int l = 1; l <= L; ++l) maxC = std::max(maxC, capI[l]);
+  ctx->maxC = maxC;
+  ctx->maxRows = capI[0];
+  for (int l = 1; l <= L; ++l) ctx->maxRows = std::max(ctx->maxRows, capI[l - 1]);
+  TRY(dalloc(ctx, &ctx->u, (size_t)maxC * HDp));
+  TRY(dalloc(ctx, &ctx->c, (size_t)maxC * HDp));
+  TRY(dalloc(ctx, &ctx->y, (size_t)maxC * Dp));
+  TRY(dalloc(ctx, &ctx->r, (size_t)maxC * Dp));
+  TRY(dalloc(ctx, &ctx->z, (size_t)maxC * dnp));
+  TRY(dalloc(ctx, &ctx->HL, (size_t)capI[L] * dnp));
+  TRY(dalloc(ctx, &ctx->rows, ctx->maxRows));
+  TRY(dalloc(ctx, &ctx->dst, maxC));
+  TRY(dalloc(ctx, &ctx->cnt_total, TG_NCOUNTERS));
+  TRY(dalloc(ctx, &ctx->cnt_tmp, TG_NCOUNTERS));
+  TRY(dalloc(ctx, &ctx->bidx, 1));
+  CK(cudaDeviceSynchronize());
+  ctx->loaded = true;
+  return tg_cache_reset(ctx, -1);
+}
+
+tg_status tg_cache_reset(tg_ctx* ctx, int64_t new_limit) {
+  if (!ctx) return TG_EINVAL;
+  if (!ctx->loaded) return TG_ESTATE;
+  if (ctx->broken) return TG_ECUDA;
+  if (new_limit > ctx->limit0) return TG_EINVAL;
+  if (new_limit >= 0) ctx->cfg.cache_limit = new_limit;
+  CK(cudaSetDevice(ctx->device));
+  CK(cudaDeviceSynchronize());
+  for (int l = 1; l < ctx->L; ++l) {
+    CacheDev& cd = ctx->cache[l];
+    CK(cudaMemset(cd.ikey, 0xFF, (cd.imask + 1) * sizeof(unsigned long long)));
+    long long st[4] = {0, 0, ctx->cfg.cache_limit, 0};
+    CK(cudaMemcpy(cd.state, st, sizeof(st), cudaMemcpyHostToDevice));
+  }
+  CK(cudaMemset(ctx->cnt_total, 0, TG_NCOUNTERS * sizeof(long long)));
+  CK(cudaMemset(ctx->cnt_tmp, 0, TG_NCOUNTERS * sizeof(long long)));
+  CK(cudaMemset(ctx->err, 0, sizeof(int)));
+  CK(cudaDeviceSynchronize());
+  ctx->launches = 0;
+  return TG_OK;
+}
+
+tg_status tg_embed_batch(tg_ctx* ctx, const int32_t* nodes, const uint32_t* ts, int64_t n, float* out,
+                         void* cuda_stream) {
+  if (!ctx) return TG_EINVAL;
+  if (!ctx->loaded) return TG_ESTATE;
+  if (ctx->broken) return TG_ECUDA;
+  if (n < 0 || n > ctx->capI[ctx->L] || (n > 0 && (!nodes || !ts || !out))) return TG_EINVAL;
+  cudaStream_t st = (cudaStream_t)cuda_stream;
+  CK(cudaSetDevice(ctx->device));
+  const bool dev_in = n == 0 || is_device_ptr(nodes);
+  const bool dev_out = n == 0 || is_device_ptr(out);
+  const int32_t* dn = nodes;
+  const uint32_t* dt = ts;
+  float* dout = out;
+  size_t need = (size_t)n * 8 + (size_t)n * ctx->d_n * 4 + 64;
+  if (!dev_in || !dev_out) TRY(ensure_stage(ctx, need));
+  char* stg = (char*)ctx->stage;
+  if (!dev_in) {
+    CK(cudaMemcpyAsync(stg, nodes, n * 4, cudaMemcpyHostToDevice, st));
+    CK(cudaMemcpyAsync(stg + n * 4, ts, n * 4, cudaMemcpyHostToDevice, st));
+    dn = (const int32_t*)stg;
+    dt = (const uint32_t*)(stg + n * 4);
+  }
+  if (!dev_out) dout = (float*)(stg + ((n * 8 + 15) & ~15));
+  launch_prep_nodes(dn, dt, (int)n, ctx->I[ctx->L], ctx->counts + 3 * ctx->L, st);
+  TRY(launched(ctx));
+  TRY(run_embed_counted(ctx, ctx->cnt_total, st));
+  launch_invert(ctx->HL, ctx->dnp, ctx->inv[ctx->L], (int)n, ctx->d_n, dout, st);
+  TRY(launched(ctx));
+  if (!dev_out) {
+    CK(cudaMemcpyAsync(out, dout, (size_t)n * ctx->d_n * 4, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+  }
+  return TG_OK;
+}
+
+static tg_status score_edges_dev(tg_ctx* ctx, const int32_t* src, const int32_t* dst, const uint32_t* ts,
+                                 int64_t n_edges, int batch, const int* bidx, float* scores, long long* cnt,
+                                 cudaStream_t st) {
+  {
+    Prof pf(ctx, TG_ST_PREP, st);
+    launch_prep_edges(src, dst, ts, n_edges, batch, bidx, ctx->I[ctx->L], ctx->counts + 3 * ctx->L, st);
+  }
+  TRY(launched(ctx));
+  TRY(run_embed_counted(ctx, cnt, st));
+  Prof pf(ctx, TG_ST_SCORE, st);
+  launch_score(ctx->HL, ctx->dnp, ctx->inv[ctx->L], (int)n_edges, batch, bidx, ctx->Wa1, ctx->ba1, ctx->Wa2,
+               ctx->ba2, ctx->d_n, ctx->dnp, scores, st);
+  return launched(ctx);
+}
+
+tg_status tg_score_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, const uint32_t* ts, int64_t n_edges,
+                         float* scores, void* cuda_stream) {
+  if (!ctx) return TG_EINVAL;
+  if (!ctx->loaded) return TG_ESTATE;
+  if (ctx->broken) return TG_ECUDA;
+  if (n_edges < 0 || 2 * n_edges > ctx->capI[ctx->L] || (n_edges > 0 && (!src || !dst || !ts || !scores)))
+    return TG_EINVAL;
+  cudaStream_t st = (cudaStream_t)cuda_stream;
+  CK(cudaSetDevice(ctx->device));
+  const bool dev_in = n_edges == 0 || is_device_ptr(src);
+  const bool dev_out = n_edges == 0 || is_device_ptr(scores);
+  const int32_t *ds = src, *dd = dst;
+  const uint32_t* dts = ts;
+  float* dsc = scores;
+  if (!dev_in || !dev_out) TRY(ensure_stage(ctx, (size_t)n_edges * 16 + 64));
+  char* stg = (char*)ctx->stage;
+  if (!dev_in) {
+    CK(cudaMemcpyAsync(stg, src, n_edges * 4, cudaMemcpyHostToDevice, st));
+    CK(cudaMemcpyAsync(stg + n_edges * 4, dst, n_edges * 4, cudaMemcpyHostToDevice, st));
+    CK(cudaMemcpyAsync(stg + n_edges * 8, ts, n_edges * 4, cudaMemcpyHostToDevice, st));
+    ds = (const int32_t*)stg;
+    dd = (const int32_t*)(stg + n_edges * 4);
+    dts = (const uint32_t*)(stg + n_edges * 8);
+  }
+  if (!dev_out) dsc = (float*)(stg + n_edges * 12);
+  TRY(score_edges_dev(ctx, ds, dd, dts, n_edges, (int)std::max<int64_t>(n_edges, 1), nullptr, dsc, ctx->cnt_total,
+                      st));
+  if (!dev_out) {
+    CK(cudaMemcpyAsync(scores, dsc, n_edges * 4, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+  }
+  return TG_OK;
+}
+
+tg_status tg_score_stream(tg_ctx* ctx, const int32_t* src, const int32_t* dst, const uint32_t* ts, int64_t n_edges,
+                          int32_t batch, float* scores, int64_t* batch_counters, void* cuda_stream) {
+  if (!ctx) return TG_EINVAL;
+  if (!ctx->loaded) return TG_ESTATE;
+  if (ctx->broken) return TG_ECUDA;
+  if (n_edges < 0 || batch < 1 || 2 * batch > ctx->capI[ctx->L] || (n_edges > 0 && (!src || !dst || !ts || !scores)))
+    return TG_EINVAL;
+  if (n_edges == 0) return TG_OK;
+  cudaStream_t st = (cudaStream_t)cuda_stream;
+  CK(cudaSetDevice(ctx->device));
+  const bool dev_in = is_device_ptr(src);
+  const bool dev_out = is_device_ptr(scores);
+  const int32_t *ds = src, *dd = dst;
+  const uint32_t* dts = ts;
+  float* dsc = scores;
+  if (!dev_in || !dev_out) TRY(ensure_stage(ctx, (size_t)n_edges * 16 + 64));
+  char* stg = (char*)ctx->stage;
+  if (!dev_in) {
+    CK(cudaMemcpyAsync(stg, src, n_edges * 4, cudaMemcpyHostToDevice, st));
+    CK(cudaMemcpyAsync(stg + n_edges * 4, dst, n_edges * 4, cudaMemcpyHostToDevice, st));
+    CK(cudaMemcpyAsync(stg + n_edges * 8, ts, n_edges * 4, cudaMemcpyHostToDevice, st));
+    ds = (const int32_t*)stg;
+    dd = (const int32_t*)(stg + n_edges * 4);
+    dts = (const uint32_t*)(stg + n_edges * 8);
+  }
+  if (!dev_out) dsc = (float*)(stg + n_edges * 12);
+  const int64_t nb = (n_edges + batch - 1) / batch;
+  CK(cudaMemsetAsync(ctx->bidx, 0, sizeof(int), st));
+  CK(cudaMemsetAsync(ctx->cnt_tmp, 0, TG_NCOUNTERS * sizeof(long long), st));
+  for (int64_t b = 0; b < nb; ++b) {
+    TRY(score_edges_dev(ctx, ds, dd, dts, n_edges, batch, ctx->bidx, dsc, ctx->cnt_tmp, st));
+    {
+      Prof pf(ctx, TG_ST_OTHER, st);
+      k_finish_batch<<<1, 64, 0, st>>>(ctx->cnt_tmp, ctx->cnt_total, (long long*)batch_counters, ctx->bidx,
+                                       TG_NCOUNTERS);
+    }
+    TRY(launched(ctx));
+  }
+  if (!dev_out) {
+    CK(cudaMemcpyAsync(scores, dsc, n_edges * 4, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+  }
+  return TG_OK;
+}
+
+tg_status tg_profile_enable(tg_ctx* ctx, int32_t on) {
+  if (!ctx) return TG_EINVAL;
+  CK(cudaSetDevice(ctx->device));
+  CK(cudaDeviceSynchronize());
+  ctx->prof = on != 0;
+  ctx->ev_used = 0;
+  return TG_OK;
+}
+
+tg_status tg_profile_read(tg_ctx* ctx, double* ms, int64_t* launches, int32_t n) {
+  if (!ctx || n < 0) return TG_EINVAL;
+  CK(cudaSetDevice(ctx->device));
+  CK(cudaDeviceSynchronize());
+  std::vector<double> acc(TG_NSTAGES, 0.0);
+  std::vector<int64_t> cnt(TG_NSTAGES, 0);
+  for (size_t i = 0; i < ctx->ev_used; ++i) {
+    float t = 0.f;
+    if (cudaEventElapsedTime(&t, ctx->ev_pool[2 * i], ctx->ev_pool[2 * i + 1]) != cudaSuccess) {
+      cudaGetLastError();
+      continue;
+    }
+    acc[ctx->ev_stage[i]] += t;
+    cnt[ctx->ev_stage[i]] += 1;
+  }
+  for (int i = 0; i < n && i < TG_NSTAGES; ++i) {
+    if (ms) ms[i] = acc[i];
+    if (launches) launches[i] = cnt[i];
+  }
+  return TG_OK;
+}
+
+tg_status tg_counters_read(tg_ctx* ctx, int64_t* host_out, int32_t n) {
+  if (!ctx || !host_out || n < 0) return TG_EINVAL;
+  if (!ctx->loaded) return TG_ESTATE;
+  CK(cudaSetDevice(ctx->device));
+  CK(cudaDeviceSynchronize());
+  long long tmp[TG_NCOUNTERS];
+  CK(cudaMemcpy(tmp, ctx->cnt_total, sizeof(tmp), cudaMemcpyDeviceToHost));
+  for (int i = 0; i < n && i < TG_NCOUNTERS; ++i) host_out[i] = tmp[i];
+  int e = 0;
+  CK(cudaMemcpy(&e, ctx->err, sizeof(int), cudaMemcpyDeviceToHost));
+  return e ? TG_EDEVICE : TG_OK;
+}
+
+tg_status tg_dedup(tg_ctx* ctx, const int32_t* nodes, const uint32_t* ts, int64_t n, int32_t* uniq_nodes,
+                   uint32_t* uniq_ts, int32_t* inv, int32_t* n_uniq, void* cuda_stream) {
+  if (!ctx || n < 0 || n > 16 * 10000) return TG_EINVAL;
+  if (n > 0 && (!nodes || !ts || !uniq_nodes || !uniq_ts || !inv || !n_uniq)) return TG_EINVAL;
+  cudaStream_t st = (cudaStream_t)cuda_stream;
+  CK(cudaSetDevice(ctx->device));
+  int* ndev = nullptr;
+  CK(cudaMalloc(&ndev, sizeof(int)));
+  int nn = (int)n;
+  CK(cudaMemcpyAsync(ndev, &nn, sizeof(int), cudaMemcpyHostToDevice, st));
+  Level in{const_cast<int32_t*>(nodes), const_cast<uint32_t*>(ts), (int)n};
+  Level out{uniq_nodes, uniq_ts, (int)n};
+  launch_dedup(in, ndev, (int)std::max<int64_t>(n, 1), out, inv, n_uniq, nullptr, nullptr, true, ctx->err, st);
+  cudaError_t e = cudaGetLastError();
+  cudaStreamSynchronize(st);
+  cudaFree(ndev);
+  return e == cudaSuccess ? TG_OK : TG_ECUDA;
+}
+
+tg_status tg_sample(tg_ctx* ctx, const int32_t* nodes, const uint32_t* ts, int64_t n, int32_t* nbr, int32_t* eid,
+                    uint32_t* nts, void* cuda_stream) {
+  if (!ctx || n < 0 || !ctx->loaded) return !ctx || n < 0 ? TG_EINVAL : TG_ESTATE;
+  if (n == 0) return TG_OK;
+  if (!nodes || !ts || !nbr || !eid || !nts) return TG_EINVAL;
+  cudaStream_t st = (cudaStream_t)cuda_stream;
+  CK(cudaSetDevice(ctx->device));
+  const int k = ctx->k;
+  int *ndev = nullptr, *nnext = nullptr;
+  int32_t* nx = nullptr;
+  uint32_t* nt = nullptr;
+  CK(cudaMalloc(&ndev, 2 * sizeof(int)));
+  nnext = ndev + 1;
+  CK(cudaMalloc(&nx, (size_t)n * (k + 1) * 4));
+  CK(cudaMalloc(&nt, (size_t)n * (k + 1) * 4));
+  int nn = (int)n;
+  CK(cudaMemcpyAsync(ndev, &nn, sizeof(int), cudaMemcpyHostToDevice, st));
+  Level C{const_cast<int32_t*>(nodes), const_cast<uint32_t*>(ts), (int)n};
+  Level next{nx, nt, (int)(n * (k + 1))};
+  launch_sample(ctx->g, C, ndev, (int)n, k, next, eid, nnext, ctx->err, st);
+  cudaError_t e = cudaGetLastError();
+  cudaMemcpyAsync(nbr, nx + n, (size_t)n * k * 4, cudaMemcpyDeviceToDevice, st);
+  cudaMemcpyAsync(nts, nt + n, (size_t)n * k * 4, cudaMemcpyDeviceToDevice, st);
+  cudaStreamSynchronize(st);
+  cudaFree(ndev);
+  cudaFree(nx);
+  cudaFree(nt);
+  return e == cudaSuccess ? TG_OK : TG_ECUDA;
+}
+
+tg_status tg_time_encode(tg_ctx* ctx, const int64_t* delta, int64_t n, int32_t use_table, float* out,
+                         void* cuda_stream) {
+  if (!ctx || n < 0) return TG_EINVAL;
+  if (!ctx->loaded) return TG_ESTATE;
+  if (n > 0 && (!delta || !out)) return TG_EINVAL;
+  CK(cudaSetDevice(ctx->device));
+  launch_time_encode(ctx->omega, ctx->phi, ctx->table, ctx->d_t, ctx->dtp, ctx->W, use_table, delta, n, out,
+                     (cudaStream_t)cuda_stream);
+  CK(cudaGetLastError());
+  return TG_OK;
+}
+
+void tg_free(tg_ctx* ctx) {
+  if (!ctx) return;
+  cudaSetDevice(ctx->device);
+  cudaDeviceSynchronize();
+  for (void* p : ctx->owned) cudaFree(p);
+  for (cudaEvent_t e : ctx->ev_pool) cudaEventDestroy(e);
+  if (ctx->stage) cudaFree(ctx->stage);
+  delete ctx;
+}
+
+}  // extern "C"

@@ -1,0 +1,262 @@
+"""GPU parity of the CUDA path (through the C ABI) against the oracle.
+
+Integer outputs (dedup keys/inverse, sampled ids, counters) are bit-exact;
+embeddings and scores meet |gpu - oracle| <= 1e-5 + 1e-4 |oracle| (fp32 mode,
+north_star / R17). Inputs are the seeded synthetic streams of synth/.
+"""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+
+from synth import make_stream
+from tests.gpu_helpers import close, setup, make_ctx, make_oracle
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _need_gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_ppopp_wangm23_b200 import lib
+    lib()  # fail loudly if libtg.so is missing
+
+
+def dev(a, dtype=None):
+    t = torch.from_numpy(np.ascontiguousarray(a))
+    if dtype is not None:
+        t = t.to(dtype)
+    return t.cuda()
+
+
+# ----------------------------------------------------------------- dedup
+@pytest.mark.parametrize("n", [0, 1, 7, 400, 8400, 20000, 84000])
+def test_dedup_bitexact(n):
+    from oracle.tgopt import dedup_filter
+    cfg, s, flat = setup("tiny")
+    ctx = make_ctx(s, flat, cfg.model)
+    rng = np.random.default_rng(n)
+    nodes = rng.integers(0, max(2, n // 3), n).astype(np.int32)
+    ts = rng.integers(0, 5, n).astype(np.uint32)
+    un = torch.zeros(max(n, 1), dtype=torch.int32, device="cuda")
+    ut = torch.zeros(max(n, 1), dtype=torch.int32, device="cuda")
+    inv = torch.zeros(max(n, 1), dtype=torch.int32, device="cuda")
+    nu = torch.zeros(1, dtype=torch.int32, device="cuda")
+    ctx.dedup(dev(nodes), dev(ts.view(np.int32)), un, ut, inv, nu)
+    torch.cuda.synchronize()
+    en, et, einv = dedup_filter(nodes, ts)
+    u = int(nu.item())
+    assert u == en.size
+    assert np.array_equal(un[:u].cpu().numpy(), en)
+    assert np.array_equal(ut[:u].cpu().numpy().view(np.uint32), et)
+    assert np.array_equal(inv[:n].cpu().numpy(), einv)
+
+
+def test_dedup_fig1_golden():
+    import json, os
+    gd = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "fig1_dedup.json")))
+    cfg, s, flat = setup("tiny")
+    ctx = make_ctx(s, flat, cfg.model)
+    n = len(gd["nodes"])
+    un = torch.zeros(n, dtype=torch.int32, device="cuda")
+    ut = torch.zeros(n, dtype=torch.int32, device="cuda")
+    inv = torch.zeros(n, dtype=torch.int32, device="cuda")
+    nu = torch.zeros(1, dtype=torch.int32, device="cuda")
+    ctx.dedup(dev(np.array(gd["nodes"], np.int32)), dev(np.array(gd["ts"], np.int32)), un, ut, inv, nu)
+    u = int(nu.item())
+    assert un[:u].tolist() == gd["unique_nodes"] and inv.tolist() == gd["inv_idx"]
+
+
+# --------------------------------------------------------------- sampler
+@pytest.mark.parametrize("name,k", [("config1", 10), ("wiki", 20), ("tiny", 3)])
+def test_sample_bitexact(name, k):
+    cfg, s, flat = setup(name, n_neighbors=k)
+    ctx = make_ctx(s, flat, cfg.model)
+    o = make_oracle(s, flat, cfg.model)
+    rng = np.random.default_rng(1)
+    n = 3000 if name != "tiny" else 200
+    nodes = rng.integers(0, s.n_nodes + 1, n).astype(np.int32)
+    ts = rng.integers(0, int(s.ts.max()) + 2, n).astype(np.int64)
+    ts[:50] = s.ts[rng.integers(0, s.n_edges, 50)]          # exact edge times: strictness t_j < t
+    ts = ts.astype(np.uint32)
+    nbr = torch.zeros(n * k, dtype=torch.int32, device="cuda")
+    eid = torch.zeros(n * k, dtype=torch.int32, device="cuda")
+    nts = torch.zeros(n * k, dtype=torch.int32, device="cuda")
+    ctx.sample(dev(nodes), dev(ts.view(np.int32)), nbr, eid, nts)
+    torch.cuda.synchronize()
+    enb, eed, ets = o.g.sample_many(nodes, ts.astype(np.int64), k)
+    assert np.array_equal(nbr.cpu().numpy().reshape(n, k), enb)
+    assert np.array_equal(eid.cpu().numpy().reshape(n, k), eed)
+    assert np.array_equal(nts.cpu().numpy().view(np.uint32).reshape(n, k).astype(np.int64), ets)
+
+
+def test_sample_fig2_golden():
+    import json, os
+    from paper_conf_ppopp_wangm23_b200 import Context
+    from synth import make_params
+    gd = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "fig2_sampler.json")))
+    e = np.array(gd["edges"])
+    X = np.zeros((6, 4), np.float32)
+    Ef = np.zeros((e.shape[0] + 1, 4), np.float32)
+    ctx = Context(5, e[:, 0], e[:, 1], e[:, 2], X, Ef)
+    ctx.load_model(make_params(1, 2, 4, 4), n_layers=1, n_neighbors=gd["k"], max_batch_targets=8,
+                   cache_limit=10, time_window=10)
+    names = {v: k for k, v in gd["nodes"].items()}
+    for tkey, want in (("t4", gd["expect"]["v@t4"]), ("t6", gd["expect"]["v@t6"])):
+        nbr = torch.zeros(3, dtype=torch.int32, device="cuda")
+        eid = torch.zeros(3, dtype=torch.int32, device="cuda")
+        nts = torch.zeros(3, dtype=torch.int32, device="cuda")
+        ctx.sample(dev(np.array([gd["nodes"]["v"]], np.int32)), dev(np.array([gd["times"][tkey]], np.int32)),
+                   nbr, eid, nts)
+        assert [names[int(j)] for j in nbr.cpu()] == want
+
+
+# ---------------------------------------------------------- time encoding
+def test_time_encode_table_equals_direct_and_oracle():
+    from oracle.tgat import time_encode
+    cfg, s, flat = setup("reddit", n_edges=2000)
+    ctx = make_ctx(s, flat, cfg.model)
+    o = make_oracle(s, flat, cfg.model)
+    rng = np.random.default_rng(2)
+    delta = np.concatenate([np.arange(0, 10_000), rng.integers(0, 3_000_000_000, 20_000),
+                            np.array([2**24 + 1, 2**31 + 5, 0])]).astype(np.int64)
+    n = delta.size
+    d_t = s.d_n
+    a = torch.zeros(n * d_t, dtype=torch.float32, device="cuda")
+    b = torch.zeros(n * d_t, dtype=torch.float32, device="cuda")
+    dd = dev(delta)
+    ctx.time_encode(dd, a, use_table=True)
+    ctx.time_encode(dd, b, use_table=False)
+    torch.cuda.synchronize()
+    assert torch.equal(a, b)              # table == direct bit-for-bit (Sec. 4.3)
+    ref = time_encode(delta, o.m.omega32, o.m.phi32).reshape(-1)
+    assert np.abs(a.cpu().numpy().astype(np.float64) - ref).max() <= 1e-6
+
+
+# ------------------------------------------------------------ embeddings
+def _embed_gpu(ctx, nodes, ts, d_n):
+    out = torch.zeros(len(nodes) * d_n, dtype=torch.float32, device="cuda")
+    ctx.embed_batch(dev(nodes.astype(np.int32)), dev(ts.astype(np.uint32).view(np.int32)), out)
+    torch.cuda.synchronize()
+    return out.cpu().numpy().reshape(len(nodes), d_n)
+
+
+@pytest.mark.parametrize("name,L", [("tiny", 1), ("tiny", 2), ("tiny_bip", 2), ("config1", 2), ("tiny", 3)])
+def test_embed_parity(name, L):
+    cfg, s, flat = setup(name, n_layers=L)
+    mc = cfg.model
+    from synth import make_params
+    flat = make_params(L, mc.n_heads, s.d_n, s.d_e)
+    ctx = make_ctx(s, flat, mc, max_targets=256)
+    o = make_oracle(s, flat, mc)
+    rng = np.random.default_rng(3)
+    n = 256 if name != "config1" else 64
+    nodes = rng.integers(0, s.n_nodes + 1, n)
+    ts = rng.integers(0, int(s.ts.max()) + 2, n)
+    nodes[:5] = 0                                      # padding node: all-masked neighbourhood (R7)
+    nodes[5:9] = nodes[9:13]                           # duplicates inside the batch
+    ts[5:9] = ts[9:13]
+    for rep in range(2):                               # second pass is served by the memo cache
+        got = _embed_gpu(ctx, nodes, ts, s.d_n)
+        ref = o.embed(L, nodes, ts)
+        ok, err, nbad = close(got, ref)
+        assert ok, (rep, err, nbad)
+
+
+def test_embed_empty_and_single():
+    cfg, s, flat = setup("tiny")
+    ctx = make_ctx(s, flat, cfg.model)
+    o = make_oracle(s, flat, cfg.model)
+    out = torch.zeros(1, dtype=torch.float32, device="cuda")
+    ctx.embed_batch(torch.zeros(0, dtype=torch.int32, device="cuda"),
+                    torch.zeros(0, dtype=torch.int32, device="cuda"), out)
+    got = _embed_gpu(ctx, np.array([3]), np.array([600]), s.d_n)
+    assert close(got, o.embed(2, np.array([3]), np.array([600])))[0]
+
+
+# ------------------------------------------------------ stream + counters
+def _stream_gpu(ctx, s, batch, n_edges=None):
+    E = s.n_edges if n_edges is None else n_edges
+    nb = (E + batch - 1) // batch
+    from paper_conf_ppopp_wangm23_b200 import TG_NCOUNTERS
+    scores = torch.zeros(E, dtype=torch.float32, device="cuda")
+    log = torch.zeros(nb * TG_NCOUNTERS, dtype=torch.int64, device="cuda")
+    ctx.score_stream(dev(s.src[:E]), dev(s.dst[:E]), dev(s.ts[:E].view(np.int32)), batch, scores, log)
+    torch.cuda.synchronize()
+    return scores.cpu().numpy(), log.cpu().numpy().reshape(nb, TG_NCOUNTERS)
+
+
+def _sim_counters(s, flat, mc, limit, E=None, opts=(True, True, True)):
+    from oracle.tgopt import TGOptSim
+    o = make_oracle(s, flat, mc)
+    sim = TGOptSim(o, cache_limit=limit, time_window=mc.time_window, dedup=opts[0], cache=opts[1],
+                   ttable=opts[2], compute=False)
+    E = s.n_edges if E is None else E
+    per = []
+    for lo in range(0, E, mc.batch):
+        hi = min(lo + mc.batch, E)
+        sim.reset_counters()
+        sim.infer_batch(s.src[lo:hi], s.dst[lo:hi], s.ts[lo:hi])
+        per.append(sim.counters())
+    return per
+
+
+@pytest.mark.parametrize("name,limit", [("config1", 2_000_000), ("tiny_bip", 20), ("config1", 3000)])
+def test_stream_counters_bitexact(name, limit):
+    from paper_conf_ppopp_wangm23_b200 import counters_dict
+    cfg, s, flat = setup(name)
+    mc = cfg.model
+    ctx = make_ctx(s, flat, mc, cache_limit=limit)
+    _, log = _stream_gpu(ctx, s, mc.batch)
+    want = _sim_counters(s, flat, mc, limit)
+    for b, w in enumerate(want):
+        got = counters_dict(log[b], mc.n_layers)
+        assert got == w, (b, {k: (got[k], w[k]) for k in w if got[k] != w[k]})
+    tot = ctx.counters()
+    assert tot["l1_misses"] == sum(w["l1_misses"] for w in want)
+
+
+@pytest.mark.parametrize("name", ["tiny_bip", "config1"])
+def test_stream_scores_parity(name):
+    cfg, s, flat = setup(name)
+    mc = cfg.model
+    ctx = make_ctx(s, flat, mc)
+    scores, _ = _stream_gpu(ctx, s, mc.batch)
+    o = make_oracle(s, flat, mc)
+    nb = (s.n_edges + mc.batch - 1) // mc.batch
+    picks = sorted(set([0, 1, nb // 2, nb - 1] + ([3, 17, 33] if nb > 33 else [])))
+    for b in picks:
+        lo, hi = b * mc.batch, min((b + 1) * mc.batch, s.n_edges)
+        _, ref = o.infer_batch(s.src[lo:hi], s.dst[lo:hi], s.ts[lo:hi])
+        ok, err, nbad = close(scores[lo:hi], ref)
+        assert ok, (b, err, nbad)
+
+
+def test_opts_invariance_bitexact():
+    cfg, s, flat = setup("config1", n_edges=3000)
+    mc = cfg.model
+    base = None
+    for opts in (7, 6, 5, 3, 1, 0):
+        ctx = make_ctx(s, flat, mc, opts=opts)
+        sc, _ = _stream_gpu(ctx, s, mc.batch)
+        if base is None:
+            base = sc
+        else:
+            assert np.array_equal(sc, base), opts
+        ctx.close()
+
+
+def test_score_edges_host_buffers_match_stream():
+    cfg, s, flat = setup("config1", n_edges=1000)
+    mc = cfg.model
+    a = make_ctx(s, flat, mc)
+    sc, _ = _stream_gpu(a, s, mc.batch)
+    b = make_ctx(s, flat, mc)
+    out = np.zeros(s.n_edges, np.float32)
+    for lo in range(0, s.n_edges, mc.batch):
+        hi = lo + mc.batch
+        tmp = np.zeros(hi - lo, np.float32)
+        b.score_edges(s.src[lo:hi].copy(), s.dst[lo:hi].copy(), s.ts[lo:hi].copy(), tmp)
+        out[lo:hi] = tmp
+    assert np.array_equal(out, sc)
