@@ -94,6 +94,10 @@ typedef struct {
   int32_t time_window;        /* W of the precomputed Phi table (10,000)     */
   uint32_t opts;              /* TG_OPT_* bits                                        */
   int32_t precision;          /* TG_PREC_*                                            */
+  int32_t superbatch;         /* S: batches per launch sequence in tg_score_stream (0 = 16,
+                               * 1 = one batch at a time). Semantics per batch are unchanged:
+                               * dedup scope, cache lookups and FIFO inserts stay per batch
+                               * and in batch order, so outputs and counters do not depend on S. */
 } tg_model_cfg;
 
 /* params: host float32 [n_params] in this order (row-major, Linear = [out x in]),

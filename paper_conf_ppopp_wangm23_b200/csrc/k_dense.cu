@@ -143,18 +143,24 @@ void launch_layernorm(const float* y, float* r, int Dp, int dn, int dnp, int de,
 }
 
 // -------------------------------------------------------------------- score
-__global__ void k_score(const float* __restrict__ HL, int ldh, const int32_t* __restrict__ inv, int64_t n_edges,
-                        int batch, const int* __restrict__ bidx, const float* __restrict__ Wa1,
-                        const float* __restrict__ ba1, const float* __restrict__ Wa2, float ba2, int dn, int dnp,
-                        float* __restrict__ scores) {
+// p_e = sigmoid(W_a2 ReLU(W_a1 [h_src || h_dst] + b_a1) + b_a2) (R10); the
+// targets' rows are reached through the batch's inverse index (DedupInvert).
+__global__ void k_score(const float* __restrict__ HL, int ldh, LevelDev top, int S, EdgeSrc es,
+                        const float* __restrict__ Wa1, const float* __restrict__ ba1, const float* __restrict__ Wa2,
+                        float ba2, int dn, int dnp, float* __restrict__ scores) {
   extern __shared__ float x[];  // [2 dnp]
   __shared__ float red[32];
-  const int64_t lo = bidx ? (int64_t)(*bidx) * batch : 0;
-  const int64_t rem = n_edges - lo;
-  const int B = (int)(rem < batch ? (rem < 0 ? 0 : rem) : batch);
-  for (int e = blockIdx.x; e < B; e += gridDim.x) {
-    const float* hs = HL + (size_t)inv[e] * ldh;       // DedupInvert (Alg. 1 l.20)
-    const float* hd = HL + (size_t)inv[B + e] * ldh;
+  for (int w = blockIdx.x; w < S * es.B; w += gridDim.x) {
+    const int b = w / es.B, e = w - b * es.B;
+    const int64_t lo = es.e0 + (int64_t)b * es.B;
+    const int64_t rem = es.n_edges - lo;
+    const int Bb = (int)(rem < es.B ? (rem < 0 ? 0 : rem) : es.B);
+    if (e >= Bb) continue;  // uniform per block
+    const size_t seg = (size_t)b * top.cap;
+    const int qs = top.c_base[b] + top.inv[seg + e];
+    const int qd = top.c_base[b] + top.inv[seg + Bb + e];
+    const float* hs = HL + (size_t)qs * ldh;
+    const float* hd = HL + (size_t)qd * ldh;
     for (int c = threadIdx.x; c < dnp; c += blockDim.x) {
       x[c] = hs[c];
       x[dnp + c] = hd[c];
@@ -162,15 +168,15 @@ __global__ void k_score(const float* __restrict__ HL, int ldh, const int32_t* __
     __syncthreads();
     float part = 0.f;
     for (int j = threadIdx.x; j < dn; j += blockDim.x) {
-      const float4* w = reinterpret_cast<const float4*>(Wa1 + (size_t)j * 2 * dnp);
+      const float4* wr = reinterpret_cast<const float4*>(Wa1 + (size_t)j * 2 * dnp);
       const float4* xv = reinterpret_cast<const float4*>(x);
       float z = 0.f;
       for (int q = 0; q < (2 * dnp) / 4; ++q) {
-        const float4 a = w[q], b = xv[q];
-        z = fmaf(a.x, b.x, z);
-        z = fmaf(a.y, b.y, z);
-        z = fmaf(a.z, b.z, z);
-        z = fmaf(a.w, b.w, z);
+        const float4 a = wr[q], bb = xv[q];
+        z = fmaf(a.x, bb.x, z);
+        z = fmaf(a.y, bb.y, z);
+        z = fmaf(a.z, bb.z, z);
+        z = fmaf(a.w, bb.w, z);
       }
       z = fmaxf(z + ba1[j], 0.f);
       part = fmaf(Wa2[j], z, part);
@@ -181,39 +187,37 @@ __global__ void k_score(const float* __restrict__ HL, int ldh, const int32_t* __
     __syncthreads();
     if (threadIdx.x == 0) {
       float s = 0.f;
-      for (int w = 0; w < (int)(blockDim.x >> 5); ++w) s += red[w];
-      const float logit = s + ba2;
-      scores[lo + e] = 1.f / (1.f + expf(-logit));
+      for (int ww = 0; ww < (int)(blockDim.x >> 5); ++ww) s += red[ww];
+      scores[lo + e] = 1.f / (1.f + expf(-(s + ba2)));
     }
     __syncthreads();
   }
 }
 
-void launch_score(const float* HL, int ldh, const int32_t* inv, int n_edges, int batch, const int* bidx,
-                  const float* Wa1, const float* ba1, const float* Wa2, float ba2, int dn, int dnp,
-                  float* scores, cudaStream_t st) {
-  int blocks = batch < 592 ? batch : 592;
+void launch_score(const float* HL, int ldh, LevelDev top, int S, EdgeSrc es, const float* Wa1, const float* ba1,
+                  const float* Wa2, float ba2, int dn, int dnp, float* scores, cudaStream_t st) {
+  int blocks = S * es.B;
+  if (blocks > 1184) blocks = 1184;
   if (blocks < 1) blocks = 1;
-  k_score<<<blocks, 128, 2 * dnp * sizeof(float), st>>>(HL, ldh, inv, n_edges, batch, bidx, Wa1, ba1, Wa2, ba2, dn,
-                                                        dnp, scores);
+  k_score<<<blocks, 128, 2 * dnp * sizeof(float), st>>>(HL, ldh, top, S, es, Wa1, ba1, Wa2, ba2, dn, dnp, scores);
 }
 
-__global__ void k_invert(const float* __restrict__ HL, int ldh, const int32_t* __restrict__ inv, int n, int dn,
+__global__ void k_invert(const float* __restrict__ HL, int ldh, LevelDev top, int n, int dn,
                          float* __restrict__ out) {
   const long long tot = (long long)n * dn;
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < tot; i += (long long)gridDim.x * blockDim.x) {
     const long long r = i / dn;
     const int c = (int)(i - r * dn);
-    out[i] = HL[(size_t)inv[r] * ldh + c];
+    out[i] = HL[(size_t)(top.c_base[0] + top.inv[r]) * ldh + c];
   }
 }
 
-void launch_invert(const float* HL, int ldh, const int32_t* inv, int n, int dn, float* out, cudaStream_t st) {
+void launch_invert(const float* HL, int ldh, LevelDev top, int n, int dn, float* out, cudaStream_t st) {
   if (n <= 0) return;
   long long tot = (long long)n * dn;
   int blocks = (int)((tot + 255) / 256);
   if (blocks > 1184) blocks = 1184;
-  k_invert<<<blocks, 256, 0, st>>>(HL, ldh, inv, n, dn, out);
+  k_invert<<<blocks, 256, 0, st>>>(HL, ldh, top, n, dn, out);
 }
 
 }  // namespace tg

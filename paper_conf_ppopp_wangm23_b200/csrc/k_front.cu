@@ -1,8 +1,11 @@
-// Integer front end of the TGOpt hot path on sm_100a: batch -> targets,
-// DedupFilter (Alg. 2) in a thread-block cluster over distributed shared
-// memory, CacheLookup / slot assignment / CacheStore index insert (Alg. 1
-// l.7-10, 17; Alg. 3 with FIFO), NghLookup as a
-// warp-cooperative 32-ary search in the T-CSR, and row-address resolution.
+// Integer front end of the TGOpt hot path on sm_100a, per superbatch:
+//  * DedupFilter (Alg. 2): one thread-block cluster per batch, the
+//    hash table lives in the cluster's distributed shared memory;
+//  * CacheLookup / compaction / CacheStore index insert (Alg. 1 l.7-10, l.17;
+//    Alg. 3 with the FIFO limit of P:L330-332), batch after batch in one CTA so
+//    the per-batch cache semantics are exactly the sequential ones;
+//  * NghLookup: warp per target, 32-ary search in the T-CSR;
+//  * row-address resolution for the dense stages.
 #include <cooperative_groups.h>
 
 #include "tg_internal.cuh"
@@ -11,47 +14,8 @@ namespace cg = cooperative_groups;
 
 namespace tg {
 
-// ---------------------------------------------------------------- batch prep
-__global__ void k_prep_edges(const int32_t* __restrict__ src, const int32_t* __restrict__ dst,
-                             const uint32_t* __restrict__ ts, int64_t n_edges, int batch,
-                             const int* __restrict__ bidx, Level out, int* n_out) {
-  int64_t lo = bidx ? (int64_t)(*bidx) * batch : 0;
-  int64_t rem = n_edges - lo;
-  int B = (int)(rem < batch ? (rem < 0 ? 0 : rem) : batch);
-  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < B; i += gridDim.x * blockDim.x) {
-    // src || dst, both at the edge time
-    out.node[i] = src[lo + i];
-    out.node[B + i] = dst[lo + i];
-    uint32_t t = ts[lo + i];
-    out.ts[i] = t;
-    out.ts[B + i] = t;
-  }
-  if (blockIdx.x == 0 && threadIdx.x == 0) *n_out = 2 * B;
-}
-
-void launch_prep_edges(const int32_t* src, const int32_t* dst, const uint32_t* ts, int64_t n_edges,
-                       int batch, const int* bidx, Level out, int* n_out_dev, cudaStream_t st) {
-  int blocks = (batch + 255) / 256;
-  k_prep_edges<<<blocks, 256, 0, st>>>(src, dst, ts, n_edges, batch, bidx, out, n_out_dev);
-}
-
-__global__ void k_prep_nodes(const int32_t* __restrict__ nodes, const uint32_t* __restrict__ ts, int n,
-                             Level out, int* n_out) {
-  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
-    out.node[i] = nodes[i];
-    out.ts[i] = ts[i];
-  }
-  if (blockIdx.x == 0 && threadIdx.x == 0) *n_out = n;
-}
-
-void launch_prep_nodes(const int32_t* nodes, const uint32_t* ts, int n, Level out, int* n_out_dev,
-                       cudaStream_t st) {
-  int blocks = n > 0 ? (n + 255) / 256 : 1;
-  k_prep_nodes<<<blocks, 256, 0, st>>>(nodes, ts, n, out, n_out_dev);
-}
-
 // -------------------------------------------------- ordered block scan helper
-// Exclusive prefix of `v` over threads in index order; returns block total.
+// Exclusive prefix of `v` over threads in index order; total via `total`.
 __device__ __forceinline__ int block_excl_scan(int v, int* s_warp, int& total) {
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = (blockDim.x + 31) >> 5;
   int x = v;
@@ -78,14 +42,19 @@ __device__ __forceinline__ int block_excl_scan(int v, int* s_warp, int& total) {
   return excl;
 }
 
+__device__ __forceinline__ int batch_edges(const EdgeSrc& es, int b, int64_t& lo) {
+  lo = es.e0 + (int64_t)b * es.B;
+  const int64_t rem = es.n_edges - lo;
+  return (int)(rem < es.B ? (rem < 0 ? 0 : rem) : es.B);
+}
+
 // -------------------------------------------------------------- DedupFilter
-// Alg. 2 with a cluster-wide hash table in distributed shared
-// memory: phase B inserts every (n, t) key and keeps the minimum position;
-// phase C marks first occurrences, ranks them with an ordered scan across the
-// cluster (first-occurrence order, R8) and phase D reads the inverse index.
+// Phase B inserts every (n, t) key into the cluster-wide table (DSMEM) and
+// keeps the minimum position; phase C marks first occurrences and ranks them
+// with an ordered scan across the cluster (first-occurrence order, R8);
+// phase D reads the inverse index.
 __global__ void __launch_bounds__(kDedupThreads, 1)
-k_dedup(Level in, const int* __restrict__ n_dev, Level uniq, int32_t* __restrict__ inv,
-        int* __restrict__ nu_dev, long long* cnt_n, long long* cnt_u, int* err) {
+k_dedup(LevelDev lv, int edge_mode, EdgeSrc es, long long* cnt, int layer, int* err) {
   extern __shared__ __align__(16) unsigned char smem[];
   unsigned long long* skey = reinterpret_cast<unsigned long long*>(smem);
   unsigned int* spos = reinterpret_cast<unsigned int*>(skey + kDedupSlots);
@@ -94,8 +63,27 @@ k_dedup(Level in, const int* __restrict__ n_dev, Level uniq, int32_t* __restrict
   cg::cluster_group cluster = cg::this_cluster();
   const unsigned CL = cluster.num_blocks();
   const unsigned rank = cluster.block_rank();
+  const int b = blockIdx.x / CL;
   const int tid = threadIdx.x;
-  const int n = *n_dev;
+  int64_t elo = 0;
+  int Bb = 0, n;
+  if (edge_mode) {
+    Bb = batch_edges(es, b, elo);
+    n = 2 * Bb;  // targets src || dst at the edge time
+  } else {
+    n = lv.n_in[b];
+  }
+  const size_t seg = (size_t)b * lv.cap;
+  auto item = [&](int i, int32_t& node, uint32_t& t) {
+    if (edge_mode) {
+      const int64_t e = elo + (i < Bb ? i : i - Bb);
+      node = i < Bb ? es.src[e] : es.dst[e];
+      t = es.ts[e];
+    } else {
+      node = lv.in_node[seg + i];
+      t = lv.in_ts[seg + i];
+    }
+  };
   for (int s = tid; s < kDedupSlots; s += blockDim.x) {
     skey[s] = kEmptyKey;
     spos[s] = 0xFFFFFFFFu;
@@ -107,13 +95,16 @@ k_dedup(Level in, const int* __restrict__ n_dev, Level uniq, int32_t* __restrict
   const int tbeg = cbeg + tid * ipt;
   const unsigned long long tmask = (unsigned long long)CL * kDedupSlots - 1ull;
   unsigned slot[kDedupIPT];
-  // ---- phase B: insert keys, keep the minimum position
+  // ---- phase B
 #pragma unroll
   for (int j = 0; j < kDedupIPT; ++j) {
     slot[j] = 0xFFFFFFFFu;
     const int i = tbeg + j;
     if (j < ipt && i < cend) {
-      const unsigned long long key = tkey(in.node[i], in.ts[i]);
+      int32_t node;
+      uint32_t t;
+      item(i, node, t);
+      const unsigned long long key = tkey(node, t);
       unsigned long long h = mix64(key) & tmask;
       for (unsigned long long probe = 0; probe <= tmask; ++probe) {
         const unsigned owner = (unsigned)(h / kDedupSlots), loc = (unsigned)(h % kDedupSlots);
@@ -130,8 +121,8 @@ k_dedup(Level in, const int* __restrict__ n_dev, Level uniq, int32_t* __restrict
     }
   }
   cluster.sync();
-  // ---- phase C1: first occurrences, ordered scan inside the CTA
-  int cnt = 0;
+  // ---- phase C1: first occurrences
+  int c = 0;
   unsigned firstmask = 0;
 #pragma unroll
   for (int j = 0; j < kDedupIPT; ++j) {
@@ -141,14 +132,14 @@ k_dedup(Level in, const int* __restrict__ n_dev, Level uniq, int32_t* __restrict
       const unsigned p = *(cluster.map_shared_rank(spos, h / kDedupSlots) + (h % kDedupSlots));
       if (p == (unsigned)i) {
         firstmask |= 1u << j;
-        ++cnt;
+        ++c;
       }
     }
   }
   int total;
-  const int excl = block_excl_scan(cnt, s_warp, total);
+  const int excl = block_excl_scan(c, s_warp, total);
   if (tid == 0) s_total = total;
-  cluster.sync();  // all first-decisions done; CTA totals visible
+  cluster.sync();
   int base = 0;
   for (unsigned r = 0; r < rank; ++r) base += *cluster.map_shared_rank(&s_total, r);
   // ---- phase C2: unique list in first-occurrence order; slot -> unique id
@@ -157,8 +148,11 @@ k_dedup(Level in, const int* __restrict__ n_dev, Level uniq, int32_t* __restrict
   for (int j = 0; j < kDedupIPT; ++j) {
     if (firstmask & (1u << j)) {
       const int i = tbeg + j;
-      uniq.node[uid] = in.node[i];
-      uniq.ts[uid] = in.ts[i];
+      int32_t node;
+      uint32_t t;
+      item(i, node, t);
+      lv.u_node[seg + uid] = node;
+      lv.u_ts[seg + uid] = t;
       const unsigned h = slot[j];
       *(cluster.map_shared_rank(spos, h / kDedupSlots) + (h % kDedupSlots)) = (unsigned)uid;
       ++uid;
@@ -166,9 +160,10 @@ k_dedup(Level in, const int* __restrict__ n_dev, Level uniq, int32_t* __restrict
   }
   if (rank == CL - 1 && tid == 0) {
     const int u = base + s_total;
-    *nu_dev = u;
-    if (cnt_n) atomicAdd((unsigned long long*)cnt_n, (unsigned long long)n);
-    if (cnt_u) atomicAdd((unsigned long long*)cnt_u, (unsigned long long)u);
+    lv.n_u[b] = u;
+    if (edge_mode) lv.n_in[b] = n;
+    cnt_add(cnt, b, layer * TG_CNT_PER_LAYER + 0, n);
+    cnt_add(cnt, b, layer * TG_CNT_PER_LAYER + 1, u);
   }
   cluster.sync();
   // ---- phase D: inverse index (DedupInvert map, Alg. 1 l.20)
@@ -177,25 +172,45 @@ k_dedup(Level in, const int* __restrict__ n_dev, Level uniq, int32_t* __restrict
     const int i = tbeg + j;
     if (j < ipt && i < cend && slot[j] != 0xFFFFFFFFu) {
       const unsigned h = slot[j];
-      inv[i] = (int32_t) * (cluster.map_shared_rank(spos, h / kDedupSlots) + (h % kDedupSlots));
+      lv.inv[seg + i] = (int32_t) * (cluster.map_shared_rank(spos, h / kDedupSlots) + (h % kDedupSlots));
     }
   }
   cluster.sync();  // peers may still read this CTA's shared memory
 }
 
 // dedup disabled (ablation): identity unique list and inverse index
-__global__ void k_dedup_off(Level in, const int* __restrict__ n_dev, Level uniq, int32_t* __restrict__ inv,
-                            int* __restrict__ nu_dev, long long* cnt_n, long long* cnt_u) {
-  const int n = *n_dev;
-  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
-    uniq.node[i] = in.node[i];
-    uniq.ts[i] = in.ts[i];
-    inv[i] = i;
-  }
-  if (blockIdx.x == 0 && threadIdx.x == 0) {
-    *nu_dev = n;
-    if (cnt_n) atomicAdd((unsigned long long*)cnt_n, (unsigned long long)n);
-    if (cnt_u) atomicAdd((unsigned long long*)cnt_u, (unsigned long long)n);
+__global__ void k_dedup_off(LevelDev lv, int S, int edge_mode, EdgeSrc es, long long* cnt, int layer) {
+  for (int b = blockIdx.y; b < S; b += gridDim.y) {
+    int64_t elo = 0;
+    int Bb = 0, n;
+    if (edge_mode) {
+      Bb = batch_edges(es, b, elo);
+      n = 2 * Bb;
+    } else {
+      n = lv.n_in[b];
+    }
+    const size_t seg = (size_t)b * lv.cap;
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+      int32_t node;
+      uint32_t t;
+      if (edge_mode) {
+        const int64_t e = elo + (i < Bb ? i : i - Bb);
+        node = i < Bb ? es.src[e] : es.dst[e];
+        t = es.ts[e];
+      } else {
+        node = lv.in_node[seg + i];
+        t = lv.in_ts[seg + i];
+      }
+      lv.u_node[seg + i] = node;
+      lv.u_ts[seg + i] = t;
+      lv.inv[seg + i] = i;
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+      lv.n_u[b] = n;
+      if (edge_mode) lv.n_in[b] = n;
+      cnt_add(cnt, b, layer * TG_CNT_PER_LAYER + 0, n);
+      cnt_add(cnt, b, layer * TG_CNT_PER_LAYER + 1, n);
+    }
   }
 }
 
@@ -205,13 +220,13 @@ static int dedup_cluster_size(int n_max) {
   return cl;
 }
 
-void launch_dedup(Level in, const int* n_dev, int n_max, Level uniq, int32_t* inv, int* nu_dev,
-                  long long* cnt_n, long long* cnt_u, bool dedup_on, int* err, cudaStream_t st) {
+void launch_dedup(LevelDev lv, int S, int n_max, bool edge_mode, EdgeSrc es, long long* cnt, int layer,
+                  bool dedup_on, int* err, cudaStream_t st) {
   if (!dedup_on) {
-    int blocks = (n_max + 255) / 256;
-    if (blocks < 1) blocks = 1;
-    if (blocks > 1184) blocks = 1184;
-    k_dedup_off<<<blocks, 256, 0, st>>>(in, n_dev, uniq, inv, nu_dev, cnt_n, cnt_u);
+    int bx = (n_max + 255) / 256;
+    if (bx < 1) bx = 1;
+    if (bx > 64) bx = 64;
+    k_dedup_off<<<dim3(bx, S), 256, 0, st>>>(lv, S, edge_mode ? 1 : 0, es, cnt, layer);
     return;
   }
   const int cl = dedup_cluster_size(n_max);
@@ -223,7 +238,7 @@ void launch_dedup(Level in, const int* n_dev, int n_max, Level uniq, int32_t* in
     attr_done = true;
   }
   cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3(cl);
+  cfg.gridDim = dim3(cl * S);
   cfg.blockDim = dim3(kDedupThreads);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = st;
@@ -234,279 +249,353 @@ void launch_dedup(Level in, const int* n_dev, int n_max, Level uniq, int32_t* in
   attr[0].val.clusterDim.z = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  cudaLaunchKernelEx(&cfg, k_dedup, in, n_dev, uniq, inv, nu_dev, cnt_n, cnt_u, err);
+  cudaLaunchKernelEx(&cfg, k_dedup, lv, edge_mode ? 1 : 0, es, cnt, layer, err);
 }
 
 // ------------------------------------------------------- CacheLookup / Store
-// One CTA: probe every unique key of layer l (Alg. 1 l.7-8), rank the misses
-// in unique-list order (l.10: "shrink ... to only the misses"), give each miss
-// the next FIFO ring position and insert key -> position into the index
-// (CacheStore, Alg. 3). Eviction is logical: the live window is the newest
-// `limit` positions (R11); dead index entries are reclaimed by later inserts.
+// One CTA walks the S batches in order. For each batch: probe every unique
+// key (Alg. 1 l.7-8), rank the misses in unique-list order (l.10), append them
+// to the compute list, give each miss the next FIFO ring position and insert
+// key -> position into the index (CacheStore, Alg. 3). Eviction is logical:
+// the live window is the newest `limit` positions (R11); dead index entries
+// are reclaimed by later inserts. The next batch probes only after this
+// batch's inserts (bar.sync orders the CTA's global writes).
 __device__ __forceinline__ unsigned long long ld_volatile_u64(const unsigned long long* p) {
   return *(const volatile unsigned long long*)p;
 }
 
 __global__ void __launch_bounds__(1024, 1)
-k_probe(Level uniq, const int* __restrict__ nu_dev, CacheDev c, int cache_on, int32_t* __restrict__ c_uidx,
-        Level C, int* __restrict__ nc_dev, long long* __restrict__ slot, long long* cntl, int* err) {
+k_probe(LevelDev lv, int S, CacheDev c, int use_cache, int has_ring, long long* cnt, int layer, int* err) {
   __shared__ int s_warp[32];
-  const int n = *nu_dev;
-  const long long head = c.state[0], size = c.state[1], limit = c.state[2];
-  const long long live_lo = head - size;
+  __shared__ int s_base;
+  __shared__ long long s_head, s_size;
   const int tid = threadIdx.x;
-  const int ipt = (n + (int)blockDim.x - 1) / (int)blockDim.x;
-  const int tbeg = tid * ipt;
-  int cnt = 0;
-  unsigned missmask = 0;
-  // ---- probe (no inserts happen until every probe is done)
+  if (tid == 0) {
+    s_base = 0;
+    s_head = has_ring ? c.state[0] : 0;
+    s_size = has_ring ? c.state[1] : 0;
+  }
+  const long long limit = has_ring ? c.state[2] : 0;
+  for (int b = 0; b < S; ++b) {
+    __syncthreads();
+    const int n = lv.n_u[b];
+    const long long head = s_head, size = s_size;
+    const long long live_lo = head - size;
+    const int base = s_base;
+    const size_t seg = (size_t)b * lv.cap;
+    const int ipt = (n + (int)blockDim.x - 1) / (int)blockDim.x;
+    const int tbeg = tid * ipt;
+    int m_local = 0;
+    unsigned missmask = 0;
 #pragma unroll
-  for (int j = 0; j < kDedupIPT; ++j) {
-    const int i = tbeg + j;
-    if (j < ipt && i < n) {
-      bool hit = false;
-      long long hp = 0;
-      if (cache_on) {
-        const unsigned long long key = tkey(uniq.node[i], uniq.ts[i]);
-        unsigned long long h = mix64(key) & c.imask;
-        for (unsigned long long pr = 0; pr <= c.imask; ++pr) {
-          const unsigned long long k0 = c.ikey[h];
-          if (k0 == kEmptyKey) break;
-          if (k0 == key) {
-            const long long p = c.ipos[h];
-            if (p >= live_lo) {
-              hit = true;
-              hp = p;
-              break;
+    for (int j = 0; j < kProbeIPT; ++j) {
+      const int i = tbeg + j;
+      if (j < ipt && i < n) {
+        bool hit = false;
+        long long hp = 0;
+        if (use_cache) {
+          const unsigned long long key = tkey(lv.u_node[seg + i], lv.u_ts[seg + i]);
+          unsigned long long h = mix64(key) & c.imask;
+          for (unsigned long long pr = 0; pr <= c.imask; ++pr) {
+            const unsigned long long k0 = c.ikey[h];
+            if (k0 == kEmptyKey) break;
+            if (k0 == key) {
+              const long long p = c.ipos[h];
+              if (p >= live_lo) {
+                hit = true;
+                hp = p;
+                break;
+              }
             }
+            h = (h + 1) & c.imask;
           }
-          h = (h + 1) & c.imask;
         }
-      }
-      if (hit) {
-        slot[i] = hp % c.rcap;
-      } else {
-        missmask |= 1u << j;
-        ++cnt;
+        if (hit) {
+          lv.slot[seg + i] = hp % c.rcap;
+        } else {
+          missmask |= 1u << j;
+          ++m_local;
+        }
       }
     }
-  }
-  int m;
-  const int excl = block_excl_scan(cnt, s_warp, m);
-  // ---- misses: ring position, miss list, index insert
-  int r = excl;
+    int m;
+    const int excl = block_excl_scan(m_local, s_warp, m);
+    int r = excl;
 #pragma unroll
-  for (int j = 0; j < kDedupIPT; ++j) {
-    if (missmask & (1u << j)) {
-      const int i = tbeg + j;
-      const long long pos = head + r;
-      slot[i] = pos % c.rcap;
-      c_uidx[r] = i;
-      C.node[r] = uniq.node[i];
-      C.ts[r] = uniq.ts[i];
-      if (cache_on) {
-        const unsigned long long key = tkey(uniq.node[i], uniq.ts[i]);
-        unsigned long long h = mix64(key) & c.imask;
-        bool done = false;
-        for (unsigned long long pr = 0; pr <= 4 * c.imask && !done; ++pr) {
-          const unsigned long long k0 = ld_volatile_u64(c.ikey + h);
-          if (k0 != kLockedKey) {
-            __threadfence();
-            const bool reusable =
-                (k0 == kEmptyKey) || (k0 == key) || (*(volatile long long*)(c.ipos + h) < live_lo);
-            if (reusable) {
-              if (atomicCAS(c.ikey + h, k0, kLockedKey) == k0) {
-                *(volatile long long*)(c.ipos + h) = pos;
+    for (int j = 0; j < kProbeIPT; ++j) {
+      if (missmask & (1u << j)) {
+        const int i = tbeg + j;
+        const int q = base + r;
+        const int32_t node = lv.u_node[seg + i];
+        const uint32_t t = lv.u_ts[seg + i];
+        lv.c_b[q] = b;
+        lv.c_u[q] = i;
+        lv.c_node[q] = node;
+        lv.c_ts[q] = t;
+        if (has_ring) {
+          const long long pos = head + r;
+          lv.slot[seg + i] = pos % c.rcap;
+          if (use_cache) {
+            const unsigned long long key = tkey(node, t);
+            unsigned long long h = mix64(key) & c.imask;
+            bool done = false;
+            for (unsigned long long pr = 0; pr <= 4 * c.imask && !done; ++pr) {
+              const unsigned long long k0 = ld_volatile_u64(c.ikey + h);
+              if (k0 != kLockedKey) {
                 __threadfence();
-                atomicExch(c.ikey + h, key);
-                if (k0 == kEmptyKey) atomicAdd((unsigned long long*)(c.state + 3), 1ull);
-                done = true;
+                const bool reusable =
+                    (k0 == kEmptyKey) || (k0 == key) || (*(volatile long long*)(c.ipos + h) < live_lo);
+                if (reusable) {
+                  if (atomicCAS(c.ikey + h, k0, kLockedKey) == k0) {
+                    *(volatile long long*)(c.ipos + h) = pos;
+                    __threadfence();
+                    atomicExch(c.ikey + h, key);
+                    if (k0 == kEmptyKey) atomicAdd((unsigned long long*)(c.state + 3), 1ull);
+                    done = true;
+                  }
+                  continue;  // lost the race: re-read the same slot
+                }
               }
-              continue;  // lost the race: re-read the same slot
+              h = (h + 1) & c.imask;
             }
+            if (!done) atomicOr(err, kErrIndexFull);
           }
-          h = (h + 1) & c.imask;
         }
-        if (!done) atomicOr(err, kErrIndexFull);
+        ++r;
       }
-      ++r;
+    }
+    __syncthreads();
+    if (tid == 0) {
+      lv.c_base[b] = base;
+      lv.n_c[b] = m;
+      s_base = base + m;
+      const int L6 = layer * TG_CNT_PER_LAYER;
+      if (use_cache) {
+        const long long nsz = size + m < limit ? size + m : limit;
+        const long long ev_total = size + m - nsz;
+        const long long evicted = ev_total < size ? ev_total : size;
+        s_head = head + m;
+        s_size = nsz;
+        cnt_add(cnt, b, L6 + 2, n);      // lookups
+        cnt_add(cnt, b, L6 + 3, n - m);  // hits
+        cnt_add(cnt, b, L6 + 4, m);      // misses = embeddings computed
+        cnt_add(cnt, b, L6 + 5, evicted);
+      } else {
+        if (has_ring) s_head = head + m;  // ring as per-batch scratch
+        cnt_add(cnt, b, L6 + 4, m);
+      }
     }
   }
   __syncthreads();
   if (tid == 0) {
-    *nc_dev = m;
-    if (cache_on) {
-      const long long nsz = size + m < limit ? size + m : limit;
-      const long long ev_total = size + m - nsz;
-      const long long evicted = ev_total < size ? ev_total : size;
-      c.state[0] = head + m;
-      c.state[1] = nsz;
-      if (cntl) {
-        atomicAdd((unsigned long long*)(cntl + 2), (unsigned long long)n);      // lookups
-        atomicAdd((unsigned long long*)(cntl + 3), (unsigned long long)(n - m));  // hits
-        atomicAdd((unsigned long long*)(cntl + 4), (unsigned long long)m);      // misses
-        atomicAdd((unsigned long long*)(cntl + 5), (unsigned long long)evicted);
-      }
-      if (c.state[3] * 10 > (long long)(c.imask + 1) * 9) atomicOr(err, kErrIndexFull);
-    } else {
-      c.state[0] = head + m;  // ring used as per-batch scratch
-      if (cntl) atomicAdd((unsigned long long*)(cntl + 4), (unsigned long long)m);
+    *lv.n_c_total = s_base;
+    if (has_ring) {
+      c.state[0] = s_head;
+      c.state[1] = s_size;
+      if (use_cache && c.state[3] * 10 > (long long)(c.imask + 1) * 9) atomicOr(err, kErrIndexFull);
     }
   }
 }
 
-void launch_probe(Level uniq, const int* nu_dev, int nu_max, CacheDev cache, bool cache_on, int32_t* c_uidx,
-                  Level C, int* nc_dev, long long* slot, long long* cnt_layer, int* err, cudaStream_t st) {
-  (void)nu_max;  // <= 1024 * kDedupIPT, checked by the host
-  k_probe<<<1, 1024, 0, st>>>(uniq, nu_dev, cache, cache_on ? 1 : 0, c_uidx, C, nc_dev, slot, cnt_layer, err);
-}
-
-// Top layer: C_L = U_L (no lookup at l = L, R9).
-__global__ void k_copy_level(Level in, const int* __restrict__ n_dev, Level out, int32_t* __restrict__ c_uidx,
-                             int* __restrict__ n_out, long long* cnt_miss) {
-  const int n = *n_dev;
-  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
-    out.node[i] = in.node[i];
-    out.ts[i] = in.ts[i];
-    c_uidx[i] = i;
+void launch_probe(LevelDev lv, int S, const CacheDev* cache, long long* cnt, int layer, int* err,
+                  cudaStream_t st) {
+  CacheDev c{};
+  int has_ring = 0, use_cache = 0;
+  if (cache) {
+    c = *cache;
+    has_ring = 1;
+    use_cache = c.ikey != nullptr;
   }
-  if (blockIdx.x == 0 && threadIdx.x == 0) {
-    *n_out = n;
-    if (cnt_miss) atomicAdd((unsigned long long*)cnt_miss, (unsigned long long)n);
-  }
-}
-
-void launch_copy_level(Level in, const int* n_dev, int n_max, Level out, int32_t* c_uidx, int* n_out_dev,
-                       long long* cnt_miss, cudaStream_t st) {
-  int blocks = (n_max + 255) / 256;
-  if (blocks < 1) blocks = 1;
-  k_copy_level<<<blocks, 256, 0, st>>>(in, n_dev, out, c_uidx, n_out_dev, cnt_miss);
+  k_probe<<<1, 1024, 0, st>>>(lv, S, c, use_cache, has_ring, cnt, layer, err);
 }
 
 // ------------------------------------------------------------------ NghLookup
-// Warp per target: 32-ary search for the first adjacency entry with t_j >= t
-// (strict t_j < t), then lanes copy the last min(k, p-lo) entries
-// right-aligned (R6), padding (0, 0, 0) on the left (R7).
-__global__ void k_sample(GraphDev g, Level C, const int* __restrict__ nc_dev, int k, Level next,
-                         int32_t* __restrict__ eid, int* __restrict__ n_next, int* err) {
-  const int nC = *nc_dev;
+// Warp per target q: 32-ary search for the first adjacency entry with
+// t_j >= t (strict t_j < t), then lanes copy the last min(k, p-lo)
+// entries right-aligned (R6), padding (0, 0, 0) on the left (R7). Writes the
+// compute-centric neighbour slots and the next level's input list
+// I_{l-1} = [C_l ; N(C_l)] of each batch (Alg. 1 l.12). Also counts, per
+// batch, how many Phi(dt) the precomputed window serves (Sec. 4.3).
+__global__ void k_sample(GraphDev g, LevelDev lv, int S, int k, LevelDev nx, int has_next, int W, int use_table,
+                         long long* cnt, int layer, int* err) {
   const int lane = threadIdx.x & 31;
   const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int nwarps = (gridDim.x * blockDim.x) >> 5;
-  if (warp == 0 && lane == 0) *n_next = nC * (k + 1);
-  for (int p = warp; p < nC; p += nwarps) {
-    int i = C.node[p];
-    const uint32_t t = C.ts[p];
+  if (blockIdx.x == 0 && threadIdx.x < S) {
+    const int b = threadIdx.x;
+    const int nb = lv.n_c[b];
+    if (has_next) nx.n_in[b] = nb * (k + 1);
+    if (layer == 1) cnt_add(cnt, b, 0, (long long)nb * (k + 1));  // h^(0) lookups (l0 n)
+  }
+  const int nC = *lv.n_c_total;
+  for (int q = warp; q < nC; q += nwarps) {
+    const int b = lv.c_b[q];
+    const int p = q - lv.c_base[b];
+    const int nb = lv.n_c[b];
+    int i = lv.c_node[q];
+    const uint32_t t = lv.c_ts[q];
     if (i < 0 || i > g.V) {
       if (lane == 0) atomicOr(err, kErrNodeRange);
       i = 0;
     }
-    int a = g.rowptr[i], b = g.rowptr[i + 1];
-    // invariant: the first entry with t_j >= t lies in [a, b] (b = "none")
-    while (b - a > 31) {
-      const int step = (b - a + 31) >> 5;
+    int a = g.rowptr[i], bnd = g.rowptr[i + 1];
+    const int lo = a;
+    // invariant: the first entry with t_j >= t lies in [a, bnd] (bnd = "none")
+    while (bnd - a > 31) {
+      const int step = (bnd - a + 31) >> 5;
       const int x = a + lane * step;
-      const bool ge = (x < b) ? (g.adj_t[x] >= t) : true;
+      const bool ge = (x < bnd) ? (g.adj_t[x] >= t) : true;
       const unsigned msk = __ballot_sync(0xffffffffu, ge);
-      if (msk == 0) {  // every probe is < t: answer beyond the last probe
+      if (msk == 0) {
         a = a + 31 * step + 1;
         continue;
       }
       const int f = __ffs(msk) - 1;
-      const int nb = a + f * step;
+      const int nbd = a + f * step;
       a = (f == 0) ? a : a + (f - 1) * step + 1;
-      b = nb < b ? nb : b;
+      bnd = nbd < bnd ? nbd : bnd;
     }
     {
-      // b - a <= 31: lane (b - a) probes x == b and votes true, so msk != 0
-      const int x = a + lane;
-      const bool ge = (x < b) ? (g.adj_t[x] >= t) : true;
+      const int x = a + lane;  // bnd - a <= 31: lane (bnd - a) votes true
+      const bool ge = (x < bnd) ? (g.adj_t[x] >= t) : true;
       const unsigned msk = __ballot_sync(0xffffffffu, ge);
       a = a + (__ffs(msk) - 1);
     }
-    const int lo = g.rowptr[i];
-    const int cnt = min(k, a - lo);
-    if (lane < k) {
-      int nb = 0, e = 0;
-      uint32_t tj = 0;
-      if (lane >= k - cnt) {
-        const int x = a - k + lane;
-        nb = g.adj_nbr[x];
-        e = g.adj_eid[x];
-        tj = g.adj_t[x];
-      }
-      next.node[nC + p * k + lane] = nb;
-      next.ts[nC + p * k + lane] = tj;
-      eid[p * k + lane] = e;
+    const int c = min(k, a - lo);
+    int nbr = 0, e = 0;
+    uint32_t tj = 0;
+    if (lane < k && lane >= k - c) {
+      const int x = a - k + lane;
+      nbr = g.adj_nbr[x];
+      e = g.adj_eid[x];
+      tj = g.adj_t[x];
     }
+    if (lane < k) {
+      const size_t o = (size_t)q * k + lane;
+      lv.nb_node[o] = nbr;
+      lv.nb_ts[o] = tj;
+      lv.nb_eid[o] = e;
+      if (has_next) {
+        const size_t seg = (size_t)b * nx.cap;
+        nx.in_node[seg + nb + (size_t)p * k + lane] = nbr;
+        nx.in_ts[seg + nb + (size_t)p * k + lane] = tj;
+      }
+    }
+    if (lane == 0 && has_next) {
+      const size_t seg = (size_t)b * nx.cap;
+      nx.in_node[seg + p] = lv.c_node[q];
+      nx.in_ts[seg + p] = t;
+    }
+    // Phi(t - t_j) source per slot: table if dt < W (padding: t_j = 0, dt = t)
+    const long long dt = (long long)t - (long long)tj;
+    const unsigned tab = __ballot_sync(0xffffffffu, lane < k && use_table && dt < W);
     if (lane == 0) {
-      next.node[p] = C.node[p];
-      next.ts[p] = t;
+      const int nt = __popc(tab);
+      cnt_add(cnt, b, TG_CNT_TTABLE, nt);
+      cnt_add(cnt, b, TG_CNT_TDIRECT, k - nt);
     }
   }
 }
 
-void launch_sample(const GraphDev& g, Level C, const int* nc_dev, int nc_max, int k, Level next, int32_t* eid,
-                   int* n_next_dev, int* err, cudaStream_t st) {
-  int blocks = (nc_max * 32 + 255) / 256;
+void launch_sample(const GraphDev& g, LevelDev lv, int S, int k, const LevelDev* next, int W, int use_table,
+                   long long* cnt, int layer, int* err, cudaStream_t st) {
+  int blocks = (lv.c_cap * 32 + 255) / 256;
   if (blocks < 1) blocks = 1;
   if (blocks > 148 * 8) blocks = 148 * 8;
-  k_sample<<<blocks, 256, 0, st>>>(g, C, nc_dev, k, next, eid, n_next_dev, err);
+  LevelDev nx{};
+  if (next) nx = *next;
+  k_sample<<<blocks, 256, 0, st>>>(g, lv, S, k, nx, next ? 1 : 0, W, use_table, cnt, layer, err);
 }
 
 // ---------------------------------------------------------------- row lookup
-__global__ void k_resolve(const float* __restrict__ X, int ldn, int64_t V, int lm1_is_zero, Level prev,
-                          const int* __restrict__ nprev_dev, const int32_t* __restrict__ inv_prev,
-                          const long long* __restrict__ slot_prev, const float* __restrict__ ring_prev,
-                          const int* __restrict__ nc_dev, const int32_t* __restrict__ c_uidx,
-                          const long long* __restrict__ slot_cur, float* ring_cur, float* hl_out,
-                          const float** __restrict__ rows, float** __restrict__ dst, int* err) {
-  const int np = *nprev_dev, nC = *nc_dev;
-  const int tid = blockIdx.x * blockDim.x + threadIdx.x, nt = gridDim.x * blockDim.x;
-  for (int j = tid; j < np; j += nt) {
-    const float* r;
-    if (lm1_is_zero) {
-      int node = prev.node[j];
-      if (node < 0 || node > V) {
-        atomicOr(err, kErrNodeRange);
-        node = 0;
+// Layer l reads h^(l-1): x_i at l = 1 (Alg. 1 l.2-3), else the ring
+// slot of the target's unique entry at level l-1 (through inv, Alg. 1 l.20).
+__global__ void k_resolve(ResolveArgs a, int* err) {
+  const int l = blockIdx.y + 1;
+  const LevelDev& lv = a.lv[l];
+  const LevelDev& pv = a.lv[l - 1];
+  const int k = a.k;
+  const int n = *lv.n_c_total;
+  const long long tot = (long long)n * (k + 1);
+  for (long long idx = blockIdx.x * (long long)blockDim.x + threadIdx.x; idx < tot;
+       idx += (long long)gridDim.x * blockDim.x) {
+    const int q = (int)(idx / (k + 1));
+    const int m = (int)(idx - (long long)q * (k + 1)) - 1;
+    const int b = lv.c_b[q];
+    const int p = q - lv.c_base[b];
+    if (m < 0) {
+      const float* hs;
+      if (l == 1) {
+        int node = lv.c_node[q];
+        if (node < 0) {
+          atomicOr(err, kErrNodeRange);
+          node = 0;
+        }
+        hs = a.X + (size_t)node * a.ldn;
+      } else {
+        const size_t seg = (size_t)b * pv.cap;
+        hs = a.ring[l - 1] + (size_t)pv.slot[seg + pv.inv[seg + p]] * a.ldn;
       }
-      r = X + (size_t)node * ldn;  // h^(0) = x_i (Alg. 1 l.2-3)
+      lv.hs_row[q] = hs;
+      lv.dst_row[q] = (l < a.L) ? a.ring[l] + (size_t)lv.slot[(size_t)b * lv.cap + lv.c_u[q]] * a.ldn
+                                : a.HL + (size_t)q * a.ldn;
     } else {
-      r = ring_prev + (size_t)slot_prev[inv_prev[j]] * ldn;  // H^(l-1) via inv (l.20)
+      const size_t o = (size_t)q * k + m;
+      const float* r;
+      if (l == 1) {
+        int node = lv.nb_node[o];
+        if (node < 0) {
+          atomicOr(err, kErrNodeRange);
+          node = 0;
+        }
+        r = a.X + (size_t)node * a.ldn;
+      } else {
+        const int nb = lv.n_c[b];
+        const size_t seg = (size_t)b * pv.cap;
+        r = a.ring[l - 1] + (size_t)pv.slot[seg + pv.inv[seg + nb + (size_t)p * k + m]] * a.ldn;
+      }
+      lv.nb_row[o] = r;
     }
-    rows[j] = r;
   }
-  for (int p = tid; p < nC; p += nt)
-    dst[p] = ring_cur ? ring_cur + (size_t)slot_cur[c_uidx[p]] * ldn : hl_out + (size_t)p * ldn;
 }
 
-void launch_resolve(const GraphDev& g, int lm1_is_zero, Level prev, const int* nprev_dev, int nprev_max,
-                    const int32_t* inv_prev, const long long* slot_prev, const float* ring_prev,
-                    long long rcap_prev, int ld, const int* nc_dev, int nc_max, const int32_t* c_uidx,
-                    const long long* slot_cur, float* ring_cur, long long rcap_cur, float* hl_out,
-                    const float** rows, float** dst, int* err, cudaStream_t st) {
-  (void)rcap_prev;
-  (void)rcap_cur;
-  (void)ld;
-  int mx = nprev_max > nc_max ? nprev_max : nc_max;
-  int blocks = (mx + 255) / 256;
-  if (blocks < 1) blocks = 1;
-  if (blocks > 592) blocks = 592;
-  k_resolve<<<blocks, 256, 0, st>>>(g.X, g.ldn, g.V, lm1_is_zero, prev, nprev_dev, inv_prev, slot_prev,
-                                    ring_prev, nc_dev, c_uidx, slot_cur, ring_cur, hl_out, rows, dst, err);
+void launch_resolve(const ResolveArgs& a, int* err, cudaStream_t st) {
+  long long mx = (long long)a.c_cap_max * (a.k + 1);
+  int bx = (int)((mx + 255) / 256);
+  if (bx < 1) bx = 1;
+  if (bx > 592) bx = 592;
+  k_resolve<<<dim3(bx, a.L), 256, 0, st>>>(a, err);
 }
 
 // ------------------------------------------------------------------- misc
-__global__ void k_bump(int* b) { *b += 1; }
-void launch_bump(int* bidx, cudaStream_t st) { k_bump<<<1, 1, 0, st>>>(bidx); }
-
-__global__ void k_add_counters(const long long* __restrict__ src, long long* __restrict__ dst, int n) {
-  int i = threadIdx.x;
-  if (i < n) dst[i] += src[i];
+__global__ void k_prep_nodes(const int32_t* __restrict__ nodes, const uint32_t* __restrict__ ts, int n,
+                             LevelDev top) {
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    top.in_node[i] = nodes[i];
+    top.in_ts[i] = ts[i];
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) top.n_in[0] = n;
 }
-void launch_add_counters(const long long* src, long long* dst, int n, cudaStream_t st) {
-  k_add_counters<<<1, 128, 0, st>>>(src, dst, n);
+
+void launch_prep_nodes(const int32_t* nodes, const uint32_t* ts, int n, LevelDev top, cudaStream_t st) {
+  int blocks = n > 0 ? (n + 255) / 256 : 1;
+  if (blocks > 592) blocks = 592;
+  k_prep_nodes<<<blocks, 256, 0, st>>>(nodes, ts, n, top);
+}
+
+__global__ void k_finish(long long* __restrict__ cnt_sb, int S, long long* __restrict__ total,
+                         long long* __restrict__ log, int64_t row0) {
+  for (int i = threadIdx.x; i < S * TG_NCOUNTERS; i += blockDim.x) {
+    const long long v = cnt_sb[i];
+    if (v) atomicAdd((unsigned long long*)(total + i % TG_NCOUNTERS), (unsigned long long)v);
+    if (log) log[row0 * TG_NCOUNTERS + i] = v;
+    cnt_sb[i] = 0;
+  }
+}
+
+void launch_finish(long long* cnt_sb, int S, long long* total, long long* log, int64_t log_row0,
+                   cudaStream_t st) {
+  k_finish<<<1, 1024, 0, st>>>(cnt_sb, S, total, log, log_row0);
 }
 
 }  // namespace tg

@@ -1,6 +1,7 @@
-// C ABI of libtg (include/tg.h): context, loading, and the per-batch
-// orchestration of Alg. 1 as a chain of stream-ordered sm_100a
-// kernels with device-resident counts (no host sync inside a batch).
+// C ABI of libtg (include/tg.h): context, loading, and the orchestration of
+// Alg. 1 over a superbatch of S chronological batches as one
+// chain of stream-ordered sm_100a kernels with device-resident counts (no
+// host sync inside the chain).
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -36,35 +37,29 @@ struct tg_ctx {
   // model
   bool loaded = false;
   tg_model_cfg cfg{};
-  int L = 0, H = 0, k = 0, d_n = 0, d_e = 0, d_t = 0, dnp = 0, dep = 0, dtp = 0, Dp = 0, W = 0;
+  int L = 0, H = 0, k = 0, d_n = 0, d_e = 0, d_t = 0, dnp = 0, dep = 0, dtp = 0, Dp = 0, W = 0, S = 1;
   LayerW lw[TG_MAX_LAYERS];
   float *omega = nullptr, *phi = nullptr, *table = nullptr;
   float *Wa1 = nullptr, *ba1 = nullptr, *Wa2 = nullptr;
   float ba2 = 0.f;
-  // recursion levels
-  Level I[TG_MAX_LAYERS + 1]{}, U[TG_MAX_LAYERS + 1]{}, C[TG_MAX_LAYERS + 1]{};
-  int capI[TG_MAX_LAYERS + 1]{};
-  int32_t *inv[TG_MAX_LAYERS + 1]{}, *cuidx[TG_MAX_LAYERS + 1]{}, *eid[TG_MAX_LAYERS + 1]{};
-  long long* slot[TG_MAX_LAYERS + 1]{};
-  int* counts = nullptr;  // device: [3*l + 0] |I_l|, [3*l+1] |U_l|, [3*l+2] |C_l|
+  // recursion levels (index l = 1..L), caches for l = 1..L-1
+  LevelDev lv[TG_MAX_LAYERS + 1]{};
+  int cap[TG_MAX_LAYERS + 1]{};
   CacheDev cache[TG_MAX_LAYERS]{};
-  long long* cache_state = nullptr;  // [TG_MAX_LAYERS * 4]
+  long long* cache_state = nullptr;
   int64_t limit0 = 0;
   // compute workspace
-  int maxC = 0, maxRows = 0;
+  int maxC = 0;
   float *u = nullptr, *c = nullptr, *y = nullptr, *r = nullptr, *z = nullptr, *HL = nullptr;
-  const float** rows = nullptr;
-  float** dst = nullptr;
   // counters / flags
   long long* cnt_total = nullptr;
-  long long* cnt_tmp = nullptr;
+  long long* cnt_sb = nullptr;  // [kMaxS x TG_NCOUNTERS]
   int* err = nullptr;
-  int* bidx = nullptr;
   int64_t launches = 0;
   // per-stage profiling (events around launches)
   bool prof = false;
   std::vector<cudaEvent_t> ev_pool;
-  std::vector<int> ev_stage;  // stage of event pair i (events 2i, 2i+1)
+  std::vector<int> ev_stage;
   size_t ev_used = 0;
   // staging for host buffers
   void* stage = nullptr;
@@ -74,13 +69,19 @@ struct tg_ctx {
 
 namespace {
 
-#define CK(x)                                                                                      \
-  do {                                                                                             \
-    cudaError_t e_ = (x);                                                                          \
-    if (e_ != cudaSuccess) {                                                                       \
+#define CK(x)                                                                                         \
+  do {                                                                                                \
+    cudaError_t e_ = (x);                                                                             \
+    if (e_ != cudaSuccess) {                                                                          \
       fprintf(stderr, "libtg: CUDA error %s at %s:%d\n", cudaGetErrorString(e_), __FILE__, __LINE__); \
-      return e_ == cudaErrorMemoryAllocation ? TG_ENOMEM : TG_ECUDA;                               \
-    }                                                                                              \
+      return e_ == cudaErrorMemoryAllocation ? TG_ENOMEM : TG_ECUDA;                                  \
+    }                                                                                                 \
+  } while (0)
+
+#define TRY(x)                  \
+  do {                          \
+    tg_status s_ = (x);         \
+    if (s_ != TG_OK) return s_; \
   } while (0)
 
 template <class T>
@@ -97,12 +98,6 @@ tg_status dalloc(tg_ctx* ctx, T** p, size_t n) {
   return TG_OK;
 }
 
-#define TRY(x)                \
-  do {                        \
-    tg_status s_ = (x);       \
-    if (s_ != TG_OK) return s_; \
-  } while (0)
-
 bool is_device_ptr(const void* p) {
   if (!p) return false;
   cudaPointerAttributes a;
@@ -113,10 +108,11 @@ bool is_device_ptr(const void* p) {
   return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
 }
 
-// Bracket the next launch with an event pair when profiling is on.
+// Bracket a launch with an event pair when profiling is on (Table 3 style breakdown).
 struct Prof {
   tg_ctx* ctx;
   cudaEvent_t e1 = nullptr;
+  cudaStream_t stream = nullptr;
   Prof(tg_ctx* c, int stage, cudaStream_t st) : ctx(c) {
     if (!c->prof) return;
     if (c->ev_used * 2 + 2 > c->ev_pool.size()) {
@@ -131,10 +127,9 @@ struct Prof {
     if (c->ev_stage.size() <= c->ev_used) c->ev_stage.resize(c->ev_used + 1);
     c->ev_stage[c->ev_used] = stage;
     ++c->ev_used;
-    cudaEventRecord(e0, st);
     stream = st;
+    cudaEventRecord(e0, st);
   }
-  cudaStream_t stream = nullptr;
   ~Prof() {
     if (e1) cudaEventRecord(e1, stream);
   }
@@ -167,186 +162,226 @@ inline int pc(const tg_ctx* ctx, int a) {  // D-space index -> padded kv index
   return ctx->dnp + ctx->dep + (a - ctx->d_n - ctx->d_e);
 }
 
-void free_model(tg_ctx* ctx) {
-  // model buffers are in ctx->owned after the graph's; freed with the context
-  (void)ctx;
-}
-
 // ------------------------------------------------------------------------
-// One Embed(L, I_L) pass (Alg. 1), I_L already in ctx->I[L] with its count.
+// Dense stages of layer l over its compute list (Eqs. 4-7).
 // ------------------------------------------------------------------------
-tg_status run_embed(tg_ctx* ctx, long long* cnt, cudaStream_t st) {
-  const int L = ctx->L, k = ctx->k;
-  const bool dedup = ctx->cfg.opts & TG_OPT_DEDUP;
-  const bool cache_on = ctx->cfg.opts & TG_OPT_CACHE;
-  int* cnts = ctx->counts;
-  auto nI = [&](int l) { return cnts + 3 * l + 0; };
-  auto nU = [&](int l) { return cnts + 3 * l + 1; };
-  auto nC = [&](int l) { return cnts + 3 * l + 2; };
-  auto cl = [&](int l) { return cnt + l * TG_CNT_PER_LAYER; };
-  // ---- top-down: dedup, lookup, sampling (Alg. 1 l.5-12)
-  for (int l = L; l >= 1; --l) {
-    {
-      Prof pf(ctx, TG_ST_DEDUP, st);
-      launch_dedup(ctx->I[l], nI(l), ctx->capI[l], ctx->U[l], ctx->inv[l], nU(l), cl(l) + 0, cl(l) + 1, dedup,
-                   ctx->err, st);
-    }
-    TRY(launched(ctx));
-    {
-      Prof pf(ctx, TG_ST_LOOKUP, st);
-      if (l == L) {
-        launch_copy_level(ctx->U[l], nU(l), ctx->capI[l], ctx->C[l], ctx->cuidx[l], nC(l), cl(l) + 4, st);
-      } else {
-        launch_probe(ctx->U[l], nU(l), ctx->capI[l], ctx->cache[l], cache_on, ctx->cuidx[l], ctx->C[l], nC(l),
-                     ctx->slot[l], cl(l), ctx->err, st);
-      }
-    }
-    TRY(launched(ctx));
-    {
-      Prof pf(ctx, TG_ST_SAMPLE, st);
-      launch_sample(ctx->g, ctx->C[l], nC(l), ctx->capI[l], k, ctx->I[l - 1], ctx->eid[l], nI(l - 1), ctx->err,
-                    st);
-    }
-    TRY(launched(ctx));
-  }
-  // ---- bottom-up: M and FFN for every computed target (Alg. 1 l.13-18)
-  for (int l = 1; l <= L; ++l) {
-    const LayerW& w = ctx->lw[l - 1];
-    const bool top = (l == L);
-    { Prof pf(ctx, TG_ST_RESOLVE, st);
-    launch_resolve(ctx->g, l == 1, ctx->I[l - 1], nI(l - 1), ctx->capI[l - 1], ctx->inv[l - 1], ctx->slot[l - 1],
-                   l == 1 ? nullptr : ctx->cache[l - 1].ring, 0, ctx->dnp, nC(l), ctx->capI[l], ctx->cuidx[l],
-                   ctx->slot[l], top ? nullptr : ctx->cache[l].ring, 0, ctx->HL, ctx->rows, ctx->dst, ctx->err, st); }
-    TRY(launched(ctx));
-    const int HDp = ctx->H * ctx->Dp;
-    const int mmax = ctx->capI[l];
-    const bool tc = ctx->cfg.precision != TG_PREC_FP32;
-    // G1: u = P hs + bu  (target-side K projection, scale folded)
-    GemmArgs g1{};
-    g1.a_rows0 = ctx->rows;
-    g1.K0 = g1.K = ctx->dnp;
-    g1.B = w.P;
-    g1.N = HDp;
-    g1.bias = w.bu;
-    g1.C = ctx->u;
-    g1.ldc = HDp;
-    g1.m_dev = nC(l);
-    g1.m_max = mmax;
-    { Prof pf(ctx, TG_ST_PROJ_K, st);
-      if (tc) launch_gemm_tc(g1, w.tcP, ctx->cfg.precision, st); else launch_gemm_simt(g1, st); }
-    TRY(launched(ctx));
-    // attention over the k neighbours
-    AttnArgs a{};
-    a.u = ctx->u;
-    a.c = ctx->c;
-    a.rows = ctx->rows;
-    a.prev_node = ctx->I[l - 1].node;
-    a.prev_ts = ctx->I[l - 1].ts;
-    a.eid = ctx->eid[l];
-    a.Ef = ctx->Ef;
-    a.lde = ctx->g.lde;
-    a.omega = ctx->omega;
-    a.phi = ctx->phi;
-    a.table = ctx->table;
-    a.W = ctx->W;
-    a.use_table = (ctx->cfg.opts & TG_OPT_TTABLE) ? 1 : 0;
-    a.dnp = ctx->dnp;
-    a.dep = ctx->dep;
-    a.dtp = ctx->dtp;
-    a.d_t = ctx->d_t;
-    a.Dp = ctx->Dp;
-    a.H = ctx->H;
-    a.k = k;
-    a.nc_dev = nC(l);
-    a.nc_max = mmax;
-    a.cnt_ttable = cnt + TG_CNT_TTABLE;
-    { Prof pf(ctx, TG_ST_ATTN, st); launch_attn(a, st); }
-    TRY(launched(ctx));
-    // G2: y = F c + b_fc + q   (value projection and W_fc folded; residual q, Eq. 4)
-    GemmArgs g2{};
-    g2.a_base0 = ctx->c;
-    g2.lda0 = HDp;
-    g2.K0 = g2.K = HDp;
-    g2.B = w.F;
-    g2.N = ctx->Dp;
-    g2.bias = w.bfc;
-    g2.q_rows = ctx->rows;
-    g2.q_dnp = ctx->dnp;
-    g2.q_dep = ctx->dep;
-    g2.q_phi0 = ctx->table;  // Phi(0): row 0 of the table
-    g2.C = ctx->y;
-    g2.ldc = ctx->Dp;
-    g2.m_dev = nC(l);
-    g2.m_max = mmax;
-    { Prof pf(ctx, TG_ST_PROJ_V, st);
-      if (tc) launch_gemm_tc(g2, w.tcF, ctx->cfg.precision, st); else launch_gemm_simt(g2, st); }
-    TRY(launched(ctx));
-    { Prof pf(ctx, TG_ST_LNORM, st);
-    launch_layernorm(ctx->y, ctx->r, ctx->Dp, ctx->d_n, ctx->dnp, ctx->d_e, ctx->dep, ctx->d_t, w.lng, w.lnb,
-                     nC(l), mmax, st); }
-    TRY(launched(ctx));
-    // G3: z = ReLU(W1 [r || hs] + b1)   (Eq. 7)
-    GemmArgs g3{};
-    g3.a_base0 = ctx->r;
-    g3.lda0 = ctx->Dp;
-    g3.K0 = ctx->Dp;
-    g3.a_rows1 = ctx->rows;
-    g3.K = ctx->Dp + ctx->dnp;
-    g3.B = w.W1;
-    g3.N = ctx->dnp;
-    g3.bias = w.b1;
-    g3.relu = 1;
-    g3.C = ctx->z;
-    g3.ldc = ctx->dnp;
-    g3.m_dev = nC(l);
-    g3.m_max = mmax;
-    { Prof pf(ctx, TG_ST_FFN1, st);
-      if (tc) launch_gemm_tc(g3, w.tcW1, ctx->cfg.precision, st); else launch_gemm_simt(g3, st); }
-    TRY(launched(ctx));
-    // G4: h = W2 z + b2 -> cache ring slot (CacheStore payload, Alg. 3 l.8-10) or H_L
-    GemmArgs g4{};
-    g4.a_base0 = ctx->z;
-    g4.lda0 = ctx->dnp;
-    g4.K0 = g4.K = ctx->dnp;
-    g4.B = w.W2;
-    g4.N = ctx->dnp;
-    g4.bias = w.b2;
-    g4.c_rows = ctx->dst;
-    g4.m_dev = nC(l);
-    g4.m_max = mmax;
-    { Prof pf(ctx, TG_ST_FFN2, st);
-      if (tc) launch_gemm_tc(g4, w.tcW2, ctx->cfg.precision, st); else launch_gemm_simt(g4, st); }
-    TRY(launched(ctx));
-  }
-  return TG_OK;
-}
-
-// level-0 input count: added once the sampler of level 1 has run
-__global__ void k_count_l0(const int* n0, long long* c0) {
-  atomicAdd((unsigned long long*)c0, (unsigned long long)*n0);
-}
-
-tg_status run_embed_counted(tg_ctx* ctx, long long* cnt, cudaStream_t st) {
-  TRY(run_embed(ctx, cnt, st));
+tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
+  const LayerW& w = ctx->lw[l - 1];
+  const LevelDev& lv = ctx->lv[l];
+  const int HDp = ctx->H * ctx->Dp;
+  const int mmax = lv.c_cap;
+  const bool tc = ctx->cfg.precision != TG_PREC_FP32;
+  const int* m_dev = lv.n_c_total;
+  // G1: u = P h^(l-1) + bu  (target-side K projection with W_q and 1/sqrt(d_k) folded)
+  GemmArgs g1{};
+  g1.a_rows0 = lv.hs_row;
+  g1.K0 = g1.K = ctx->dnp;
+  g1.B = w.P;
+  g1.N = HDp;
+  g1.bias = w.bu;
+  g1.C = ctx->u;
+  g1.ldc = HDp;
+  g1.m_dev = m_dev;
+  g1.m_max = mmax;
   {
-    Prof pf(ctx, TG_ST_OTHER, st);
-    k_count_l0<<<1, 1, 0, st>>>(ctx->counts + 0, cnt + 0);
+    Prof pf(ctx, TG_ST_PROJ_K, st);
+    if (tc) launch_gemm_tc(g1, w.tcP, ctx->cfg.precision, st);
+    else launch_gemm_simt(g1, st);
+  }
+  TRY(launched(ctx));
+  // attention over the k sampled neighbours
+  AttnArgs a{};
+  a.u = ctx->u;
+  a.c = ctx->c;
+  a.nb_row = lv.nb_row;
+  a.nb_node = lv.nb_node;
+  a.nb_ts = lv.nb_ts;
+  a.nb_eid = lv.nb_eid;
+  a.c_ts = lv.c_ts;
+  a.Ef = ctx->Ef;
+  a.lde = ctx->g.lde;
+  a.omega = ctx->omega;
+  a.phi = ctx->phi;
+  a.table = ctx->table;
+  a.W = ctx->W;
+  a.use_table = (ctx->cfg.opts & TG_OPT_TTABLE) ? 1 : 0;
+  a.dnp = ctx->dnp;
+  a.dep = ctx->dep;
+  a.dtp = ctx->dtp;
+  a.d_t = ctx->d_t;
+  a.Dp = ctx->Dp;
+  a.H = ctx->H;
+  a.k = ctx->k;
+  a.nc_dev = m_dev;
+  a.nc_max = mmax;
+  {
+    Prof pf(ctx, TG_ST_ATTN, st);
+    launch_attn(a, st);
+  }
+  TRY(launched(ctx));
+  // G2: y = F c + b_fc + q  (W_v and W_fc folded; residual q of Eq. 4)
+  GemmArgs g2{};
+  g2.a_base0 = ctx->c;
+  g2.lda0 = HDp;
+  g2.K0 = g2.K = HDp;
+  g2.B = w.F;
+  g2.N = ctx->Dp;
+  g2.bias = w.bfc;
+  g2.q_rows = lv.hs_row;
+  g2.q_dnp = ctx->dnp;
+  g2.q_dep = ctx->dep;
+  g2.q_phi0 = ctx->table;  // Phi(0): row 0 of the table
+  g2.C = ctx->y;
+  g2.ldc = ctx->Dp;
+  g2.m_dev = m_dev;
+  g2.m_max = mmax;
+  {
+    Prof pf(ctx, TG_ST_PROJ_V, st);
+    if (tc) launch_gemm_tc(g2, w.tcF, ctx->cfg.precision, st);
+    else launch_gemm_simt(g2, st);
+  }
+  TRY(launched(ctx));
+  {
+    Prof pf(ctx, TG_ST_LNORM, st);
+    launch_layernorm(ctx->y, ctx->r, ctx->Dp, ctx->d_n, ctx->dnp, ctx->d_e, ctx->dep, ctx->d_t, w.lng, w.lnb, m_dev,
+                     mmax, st);
+  }
+  TRY(launched(ctx));
+  // G3: z = ReLU(W1 [r || h^(l-1)] + b1)  (Eq. 7)
+  GemmArgs g3{};
+  g3.a_base0 = ctx->r;
+  g3.lda0 = ctx->Dp;
+  g3.K0 = ctx->Dp;
+  g3.a_rows1 = lv.hs_row;
+  g3.K = ctx->Dp + ctx->dnp;
+  g3.B = w.W1;
+  g3.N = ctx->dnp;
+  g3.bias = w.b1;
+  g3.relu = 1;
+  g3.C = ctx->z;
+  g3.ldc = ctx->dnp;
+  g3.m_dev = m_dev;
+  g3.m_max = mmax;
+  {
+    Prof pf(ctx, TG_ST_FFN1, st);
+    if (tc) launch_gemm_tc(g3, w.tcW1, ctx->cfg.precision, st);
+    else launch_gemm_simt(g3, st);
+  }
+  TRY(launched(ctx));
+  // G4: h = W2 z + b2 -> ring slot (CacheStore payload, Alg. 3 l.8-10) or H_L
+  GemmArgs g4{};
+  g4.a_base0 = ctx->z;
+  g4.lda0 = ctx->dnp;
+  g4.K0 = g4.K = ctx->dnp;
+  g4.B = w.W2;
+  g4.N = ctx->dnp;
+  g4.bias = w.b2;
+  g4.c_rows = lv.dst_row;
+  g4.m_dev = m_dev;
+  g4.m_max = mmax;
+  {
+    Prof pf(ctx, TG_ST_FFN2, st);
+    if (tc) launch_gemm_tc(g4, w.tcW2, ctx->cfg.precision, st);
+    else launch_gemm_simt(g4, st);
   }
   return launched(ctx);
 }
 
-__global__ void k_finish_batch(long long* __restrict__ tmp, long long* __restrict__ total,
-                               long long* __restrict__ log, int* __restrict__ bidx, int n) {
-  const int i = threadIdx.x;
-  if (i < n) {
-    const long long v = tmp[i];
-    total[i] += v;
-    if (log) log[(long long)(*bidx) * n + i] = v;
-    tmp[i] = 0;
+// ------------------------------------------------------------------------
+// Embed(L, .) for S batches (Alg. 1): edge_mode -> batches of the stream
+// (targets src || dst), else one batch of explicit targets (prepared in lv[L]).
+// ------------------------------------------------------------------------
+tg_status run_superbatch(tg_ctx* ctx, int S, bool edge_mode, const EdgeSrc& es, int n_max_top, cudaStream_t st) {
+  const int L = ctx->L, k = ctx->k;
+  const bool dedup = ctx->cfg.opts & TG_OPT_DEDUP;
+  const bool cache_on = ctx->cfg.opts & TG_OPT_CACHE;
+  const int use_table = (ctx->cfg.opts & TG_OPT_TTABLE) ? 1 : 0;
+  long long* cnt = ctx->cnt_sb;
+  // ---- top-down (Alg. 1 l.5-12): dedup, lookup/compaction, sampling
+  {
+    Prof pf(ctx, TG_ST_DEDUP, st);
+    launch_dedup(ctx->lv[L], S, n_max_top, edge_mode, es, cnt, L, dedup, ctx->err, st);
   }
-  __syncthreads();
-  if (i == 0) *bidx += 1;
+  TRY(launched(ctx));
+  {
+    Prof pf(ctx, TG_ST_LOOKUP, st);
+    launch_probe(ctx->lv[L], S, nullptr, cnt, L, ctx->err, st);  // no lookup at l = L
+  }
+  TRY(launched(ctx));
+  for (int l = L; l >= 1; --l) {
+    {
+      Prof pf(ctx, TG_ST_SAMPLE, st);
+      launch_sample(ctx->g, ctx->lv[l], S, k, l >= 2 ? &ctx->lv[l - 1] : nullptr, ctx->W, use_table, cnt, l,
+                    ctx->err, st);
+    }
+    TRY(launched(ctx));
+    if (l >= 2) {
+      {
+        Prof pf(ctx, TG_ST_DEDUP, st);
+        launch_dedup(ctx->lv[l - 1], S, ctx->cap[l - 1], false, es, cnt, l - 1, dedup, ctx->err, st);
+      }
+      TRY(launched(ctx));
+      CacheDev cd = ctx->cache[l - 1];
+      if (!cache_on) cd.ikey = nullptr;  // ring used as scratch only
+      {
+        Prof pf(ctx, TG_ST_LOOKUP, st);
+        launch_probe(ctx->lv[l - 1], S, &cd, cnt, l - 1, ctx->err, st);
+      }
+      TRY(launched(ctx));
+    }
+  }
+  // ---- row addresses for every layer
+  ResolveArgs ra{};
+  for (int l = 0; l <= L; ++l) ra.lv[l] = ctx->lv[l];
+  for (int l = 1; l < L; ++l) ra.ring[l] = ctx->cache[l].ring;
+  ra.HL = ctx->HL;
+  ra.X = ctx->X;
+  ra.ldn = ctx->dnp;
+  ra.k = k;
+  ra.L = L;
+  ra.c_cap_max = ctx->maxC;
+  {
+    Prof pf(ctx, TG_ST_RESOLVE, st);
+    launch_resolve(ra, ctx->err, st);
+  }
+  TRY(launched(ctx));
+  // ---- bottom-up (Alg. 1 l.13-18): M and FFN, layer by layer over all S batches
+  for (int l = 1; l <= L; ++l) TRY(run_layer(ctx, l, st));
+  return TG_OK;
 }
+
+tg_status finish(tg_ctx* ctx, int S, long long* log, int64_t row0, cudaStream_t st) {
+  {
+    Prof pf(ctx, TG_ST_OTHER, st);
+    launch_finish(ctx->cnt_sb, S, ctx->cnt_total, log, row0, st);
+  }
+  return launched(ctx);
+}
+
+tg_status stream_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, const uint32_t* ts, int64_t n_edges,
+                       int batch, float* scores, long long* log, cudaStream_t st) {
+  const int64_t nb = (n_edges + batch - 1) / batch;
+  for (int64_t b0 = 0; b0 < nb; b0 += ctx->S) {
+    const int S = (int)std::min<int64_t>(ctx->S, nb - b0);
+    EdgeSrc es{src, dst, ts, n_edges, b0 * batch, batch};
+    TRY(run_superbatch(ctx, S, true, es, 2 * batch, st));
+    {
+      Prof pf(ctx, TG_ST_SCORE, st);
+      launch_score(ctx->HL, ctx->dnp, ctx->lv[ctx->L], S, es, ctx->Wa1, ctx->ba1, ctx->Wa2, ctx->ba2, ctx->d_n,
+                   ctx->dnp, scores, st);
+    }
+    TRY(launched(ctx));
+    TRY(finish(ctx, S, log, b0, st));
+  }
+  return TG_OK;
+}
+
+struct Staged {
+  const int32_t *src = nullptr, *dst = nullptr;
+  const uint32_t* ts = nullptr;
+  float* out = nullptr;
+  bool host_out = false;
+};
 
 }  // namespace
 
@@ -366,7 +401,7 @@ const char* tg_strerror(tg_status s) {
   return "unknown";
 }
 
-const char* tg_version(void) { return "libtg 0.1 sm_100a (fp32 SIMT, tf32x3/bf16 tcgen05)"; }
+const char* tg_version(void) { return "libtg 0.2 sm_100a (fp32 SIMT, tf32x3/bf16 tcgen05; superbatch schedule)"; }
 
 int64_t tg_kernel_launches(tg_ctx* ctx) { return ctx ? ctx->launches : 0; }
 
@@ -386,8 +421,8 @@ tg_status tg_graph_load(int device, const tg_graph_desc* gd, tg_ctx** out) {
   tg_ctx* ctx = new (std::nothrow) tg_ctx();
   if (!ctx) return TG_ENOMEM;
   ctx->device = device;
-  // ---- T-CSR on the host: counting sort by node; edges are already in
-  // (t, edge id) order, so appending keeps each adjacency sorted (R6).
+  // T-CSR on the host: counting sort by node; edges are already in (t, edge
+  // id) order, so appending keeps each adjacency sorted (R6).
   std::vector<int32_t> rowptr(V + 2, 0);
   for (int64_t i = 0; i < E; ++i) {
     rowptr[gd->src[i] + 1]++;
@@ -432,7 +467,6 @@ tg_status tg_graph_load(int device, const tg_graph_desc* gd, tg_ctx** out) {
   TRYF(dalloc(ctx, &ctx->Ef, (size_t)(E + 1) * lde));
   cudaMemset(ctx->X, 0, (size_t)(V + 1) * ldn * 4);
   cudaMemset(ctx->Ef, 0, (size_t)(E + 1) * lde * 4);
-  // padded row copies; row 0 stays zero
   if (V > 0)
     cudaMemcpy2D(ctx->X + ldn, ldn * 4, gd->node_feat + gd->d_n, gd->d_n * 4, gd->d_n * 4, V, cudaMemcpyHostToDevice);
   if (E > 0)
@@ -465,31 +499,34 @@ tg_status tg_graph_load(int device, const tg_graph_desc* gd, tg_ctx** out) {
 tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* params, int64_t n_params) {
   if (!ctx || !cfg || !params) return TG_EINVAL;
   if (ctx->broken) return TG_ECUDA;
-  if (ctx->loaded) return TG_ESTATE;  // one model per context (create a new context to replace it)
+  if (ctx->loaded) return TG_ESTATE;  // one model per context
   const int L = cfg->n_layers, H = cfg->n_heads, k = cfg->n_neighbors, d_t = cfg->d_t;
   const int d_n = ctx->g.d_n, d_e = ctx->g.d_e;
   const int D = d_n + d_e + d_t;
   if (L < 1 || L > TG_MAX_LAYERS || H < 1 || k < 1 || k > kMaxK || d_t < 1 || D % H) return TG_EINVAL;
   if (cfg->max_batch_targets < 1 || cfg->cache_limit < 0 || cfg->time_window < 0) return TG_EINVAL;
   if (cfg->precision < TG_PREC_FP32 || cfg->precision > TG_PREC_BF16) return TG_EINVAL;
+  if (cfg->superbatch < 0 || cfg->superbatch > kMaxS) return TG_EINVAL;
   const int64_t per_layer = 4LL * D * D + 3LL * D + (int64_t)d_n * (D + d_n) + d_n + (int64_t)d_n * d_n + d_n;
   const int64_t expect = L * per_layer + 2LL * d_t + 2LL * d_n * d_n + d_n + d_n + 1;
   if (n_params != expect) return TG_EINVAL;
-  // workspace capacities: I_L = targets, I_{l-1} = C_l (k+1) <= I_l (k+1)
-  int64_t cap = cfg->max_batch_targets;
-  int capI[TG_MAX_LAYERS + 1];
-  capI[L] = (int)cap;
-  for (int l = L - 1; l >= 0; --l) {
-    cap = cap * (k + 1);
-    if (cap > (int64_t)1 << 26) return TG_EINVAL;
-    capI[l] = (int)cap;
+  const int S = cfg->superbatch ? cfg->superbatch : 16;
+  // per-batch capacities: I_L = targets; I_{l-1} = C_l (k+1) <= I_l (k+1)
+  int cap[TG_MAX_LAYERS + 1];
+  int64_t cc = cfg->max_batch_targets;
+  cap[L] = (int)cc;
+  for (int l = L - 1; l >= 1; --l) {
+    cc = cc * (k + 1);
+    if (cc * S > ((int64_t)1 << 26)) return TG_EINVAL;
+    cap[l] = (int)cc;
   }
   for (int l = 1; l <= L; ++l) {
-    if (capI[l] > 16 * 10000) return TG_EINVAL;                        // dedup cluster bound
-    if (l < L && capI[l] > kDedupThreads * kDedupIPT) return TG_EINVAL;  // probe CTA bound
+    if (cap[l] > 16 * 10000) return TG_EINVAL;                   // dedup cluster bound
+    if (cap[l] > 1024 * kProbeIPT) return TG_EINVAL;             // probe CTA bound
   }
   if (cudaSetDevice(ctx->device) != cudaSuccess) return TG_ECUDA;
   ctx->cfg = *cfg;
+  ctx->S = S;
   ctx->L = L;
   ctx->H = H;
   ctx->k = k;
@@ -603,51 +640,67 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     const float* ba1 = Wa1 + (size_t)d_n * 2 * d_n;
     const float* Wa2 = ba1 + d_n;
     const float* ba2 = Wa2 + d_n;
-    std::vector<float> W((size_t)dnp * 2 * dnp, 0.f), b(dnp, 0.f), w2(dnp, 0.f);
+    std::vector<float> Wv((size_t)dnp * 2 * dnp, 0.f), b(dnp, 0.f), w2(dnp, 0.f);
     for (int j = 0; j < d_n; ++j) {
       for (int a = 0; a < d_n; ++a) {
-        W[(size_t)j * 2 * dnp + a] = Wa1[(size_t)j * 2 * d_n + a];
-        W[(size_t)j * 2 * dnp + dnp + a] = Wa1[(size_t)j * 2 * d_n + d_n + a];
+        Wv[(size_t)j * 2 * dnp + a] = Wa1[(size_t)j * 2 * d_n + a];
+        Wv[(size_t)j * 2 * dnp + dnp + a] = Wa1[(size_t)j * 2 * d_n + d_n + a];
       }
       b[j] = ba1[j];
       w2[j] = Wa2[j];
     }
-    TRY(dalloc(ctx, &ctx->Wa1, W.size()));
+    TRY(dalloc(ctx, &ctx->Wa1, Wv.size()));
     TRY(dalloc(ctx, &ctx->ba1, b.size()));
     TRY(dalloc(ctx, &ctx->Wa2, w2.size()));
-    CK(cudaMemcpy(ctx->Wa1, W.data(), W.size() * 4, cudaMemcpyHostToDevice));
+    CK(cudaMemcpy(ctx->Wa1, Wv.data(), Wv.size() * 4, cudaMemcpyHostToDevice));
     CK(cudaMemcpy(ctx->ba1, b.data(), b.size() * 4, cudaMemcpyHostToDevice));
     CK(cudaMemcpy(ctx->Wa2, w2.data(), w2.size() * 4, cudaMemcpyHostToDevice));
     ctx->ba2 = ba2[0];
   }
-  // ---- recursion-level workspaces
-  for (int l = 0; l <= L; ++l) {
-    ctx->capI[l] = capI[l];
-    TRY(dalloc(ctx, &ctx->I[l].node, capI[l]));
-    TRY(dalloc(ctx, &ctx->I[l].ts, capI[l]));
-    ctx->I[l].cap = capI[l];
-    if (l >= 1) {
-      TRY(dalloc(ctx, &ctx->U[l].node, capI[l]));
-      TRY(dalloc(ctx, &ctx->U[l].ts, capI[l]));
-      TRY(dalloc(ctx, &ctx->C[l].node, capI[l]));
-      TRY(dalloc(ctx, &ctx->C[l].ts, capI[l]));
-      ctx->U[l].cap = ctx->C[l].cap = capI[l];
-      TRY(dalloc(ctx, &ctx->inv[l], capI[l]));
-      TRY(dalloc(ctx, &ctx->cuidx[l], capI[l]));
-      TRY(dalloc(ctx, &ctx->slot[l], capI[l]));
-      TRY(dalloc(ctx, &ctx->eid[l], (size_t)capI[l] * k));
-    }
+  // ---- recursion levels: batch-segmented lists + superbatch compute lists
+  int maxC = 0;
+  for (int l = 1; l <= L; ++l) {
+    LevelDev& v = ctx->lv[l];
+    const size_t n = (size_t)S * cap[l];
+    ctx->cap[l] = cap[l];
+    v.cap = cap[l];
+    v.c_cap = (int)n;
+    maxC = std::max(maxC, (int)n);
+    TRY(dalloc(ctx, &v.in_node, n));
+    TRY(dalloc(ctx, &v.in_ts, n));
+    TRY(dalloc(ctx, &v.n_in, kMaxS));
+    TRY(dalloc(ctx, &v.u_node, n));
+    TRY(dalloc(ctx, &v.u_ts, n));
+    TRY(dalloc(ctx, &v.n_u, kMaxS));
+    TRY(dalloc(ctx, &v.inv, n));
+    TRY(dalloc(ctx, &v.slot, n));
+    TRY(dalloc(ctx, &v.c_b, n));
+    TRY(dalloc(ctx, &v.c_u, n));
+    TRY(dalloc(ctx, &v.c_node, n));
+    TRY(dalloc(ctx, &v.c_ts, n));
+    TRY(dalloc(ctx, &v.c_base, kMaxS));
+    TRY(dalloc(ctx, &v.n_c, kMaxS));
+    TRY(dalloc(ctx, &v.n_c_total, 1));
+    TRY(dalloc(ctx, &v.nb_node, n * k));
+    TRY(dalloc(ctx, &v.nb_ts, n * k));
+    TRY(dalloc(ctx, &v.nb_eid, n * k));
+    TRY(dalloc(ctx, &v.hs_row, n));
+    TRY(dalloc(ctx, &v.nb_row, n * k));
+    TRY(dalloc(ctx, &v.dst_row, n));
+    CK(cudaMemset(v.n_c_total, 0, sizeof(int)));
+    CK(cudaMemset(v.n_in, 0, kMaxS * sizeof(int)));
   }
-  TRY(dalloc(ctx, &ctx->counts, 3 * (TG_MAX_LAYERS + 1)));
-  CK(cudaMemset(ctx->counts, 0, 3 * (TG_MAX_LAYERS + 1) * sizeof(int)));
-  // ---- caches for layers 1..L-1: index (load <= 1/4 of live items) + FIFO ring
+  ctx->maxC = maxC;
+  // ---- caches for layers 1..L-1: index (load <= 1/4 of live items) + FIFO ring.
+  // Ring capacity limit + (S+2) cap: a superbatch never overwrites a slot that
+  // one of its own batches still reads.
   TRY(dalloc(ctx, &ctx->cache_state, 4 * TG_MAX_LAYERS));
   ctx->limit0 = cfg->cache_limit;
   for (int l = 1; l < L; ++l) {
     CacheDev& cd = ctx->cache[l];
-    const long long rcap = cfg->cache_limit + 2LL * capI[l] + 16;
+    const long long rcap = cfg->cache_limit + (long long)(S + 2) * cap[l] + 16;
     unsigned long long icap = 1024;
-    while (icap < 4ull * (unsigned long long)(cfg->cache_limit + capI[l])) icap <<= 1;
+    while (icap < 4ull * (unsigned long long)(cfg->cache_limit + (long long)S * cap[l])) icap <<= 1;
     TRY(dalloc(ctx, &cd.ikey, icap));
     TRY(dalloc(ctx, &cd.ipos, icap));
     TRY(dalloc(ctx, &cd.ring, (size_t)rcap * dnp));
@@ -656,22 +709,15 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     cd.state = ctx->cache_state + 4 * l;
   }
   // ---- compute workspace
-  int maxC = 0;
-  for (int l = 1; l <= L; ++l) maxC = std::max(maxC, capI[l]);
-  ctx->maxC = maxC;
-  ctx->maxRows = capI[0];
-  for (int l = 1; l <= L; ++l) ctx->maxRows = std::max(ctx->maxRows, capI[l - 1]);
   TRY(dalloc(ctx, &ctx->u, (size_t)maxC * HDp));
   TRY(dalloc(ctx, &ctx->c, (size_t)maxC * HDp));
   TRY(dalloc(ctx, &ctx->y, (size_t)maxC * Dp));
   TRY(dalloc(ctx, &ctx->r, (size_t)maxC * Dp));
   TRY(dalloc(ctx, &ctx->z, (size_t)maxC * dnp));
-  TRY(dalloc(ctx, &ctx->HL, (size_t)capI[L] * dnp));
-  TRY(dalloc(ctx, &ctx->rows, ctx->maxRows));
-  TRY(dalloc(ctx, &ctx->dst, maxC));
+  TRY(dalloc(ctx, &ctx->HL, (size_t)S * cap[L] * dnp));
   TRY(dalloc(ctx, &ctx->cnt_total, TG_NCOUNTERS));
-  TRY(dalloc(ctx, &ctx->cnt_tmp, TG_NCOUNTERS));
-  TRY(dalloc(ctx, &ctx->bidx, 1));
+  TRY(dalloc(ctx, &ctx->cnt_sb, (size_t)kMaxS * TG_NCOUNTERS));
+  CK(cudaMemset(ctx->cnt_sb, 0, (size_t)kMaxS * TG_NCOUNTERS * sizeof(long long)));
   CK(cudaDeviceSynchronize());
   ctx->loaded = true;
   return tg_cache_reset(ctx, -1);
@@ -692,7 +738,7 @@ tg_status tg_cache_reset(tg_ctx* ctx, int64_t new_limit) {
     CK(cudaMemcpy(cd.state, st, sizeof(st), cudaMemcpyHostToDevice));
   }
   CK(cudaMemset(ctx->cnt_total, 0, TG_NCOUNTERS * sizeof(long long)));
-  CK(cudaMemset(ctx->cnt_tmp, 0, TG_NCOUNTERS * sizeof(long long)));
+  CK(cudaMemset(ctx->cnt_sb, 0, (size_t)kMaxS * TG_NCOUNTERS * sizeof(long long)));
   CK(cudaMemset(ctx->err, 0, sizeof(int)));
   CK(cudaDeviceSynchronize());
   ctx->launches = 0;
@@ -704,7 +750,7 @@ tg_status tg_embed_batch(tg_ctx* ctx, const int32_t* nodes, const uint32_t* ts, 
   if (!ctx) return TG_EINVAL;
   if (!ctx->loaded) return TG_ESTATE;
   if (ctx->broken) return TG_ECUDA;
-  if (n < 0 || n > ctx->capI[ctx->L] || (n > 0 && (!nodes || !ts || !out))) return TG_EINVAL;
+  if (n < 0 || n > ctx->cap[ctx->L] || (n > 0 && (!nodes || !ts || !out))) return TG_EINVAL;
   cudaStream_t st = (cudaStream_t)cuda_stream;
   CK(cudaSetDevice(ctx->device));
   const bool dev_in = n == 0 || is_device_ptr(nodes);
@@ -712,7 +758,7 @@ tg_status tg_embed_batch(tg_ctx* ctx, const int32_t* nodes, const uint32_t* ts, 
   const int32_t* dn = nodes;
   const uint32_t* dt = ts;
   float* dout = out;
-  size_t need = (size_t)n * 8 + (size_t)n * ctx->d_n * 4 + 64;
+  const size_t need = (size_t)n * 8 + (size_t)n * ctx->d_n * 4 + 64;
   if (!dev_in || !dev_out) TRY(ensure_stage(ctx, need));
   char* stg = (char*)ctx->stage;
   if (!dev_in) {
@@ -722,11 +768,13 @@ tg_status tg_embed_batch(tg_ctx* ctx, const int32_t* nodes, const uint32_t* ts, 
     dt = (const uint32_t*)(stg + n * 4);
   }
   if (!dev_out) dout = (float*)(stg + ((n * 8 + 15) & ~15));
-  launch_prep_nodes(dn, dt, (int)n, ctx->I[ctx->L], ctx->counts + 3 * ctx->L, st);
+  launch_prep_nodes(dn, dt, (int)n, ctx->lv[ctx->L], st);
   TRY(launched(ctx));
-  TRY(run_embed_counted(ctx, ctx->cnt_total, st));
-  launch_invert(ctx->HL, ctx->dnp, ctx->inv[ctx->L], (int)n, ctx->d_n, dout, st);
+  EdgeSrc none{};
+  TRY(run_superbatch(ctx, 1, false, none, (int)std::max<int64_t>(n, 1), st));
+  launch_invert(ctx->HL, ctx->dnp, ctx->lv[ctx->L], (int)n, ctx->d_n, dout, st);
   TRY(launched(ctx));
+  TRY(finish(ctx, 1, nullptr, 0, st));
   if (!dev_out) {
     CK(cudaMemcpyAsync(out, dout, (size_t)n * ctx->d_n * 4, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
@@ -734,19 +782,28 @@ tg_status tg_embed_batch(tg_ctx* ctx, const int32_t* nodes, const uint32_t* ts, 
   return TG_OK;
 }
 
-static tg_status score_edges_dev(tg_ctx* ctx, const int32_t* src, const int32_t* dst, const uint32_t* ts,
-                                 int64_t n_edges, int batch, const int* bidx, float* scores, long long* cnt,
-                                 cudaStream_t st) {
-  {
-    Prof pf(ctx, TG_ST_PREP, st);
-    launch_prep_edges(src, dst, ts, n_edges, batch, bidx, ctx->I[ctx->L], ctx->counts + 3 * ctx->L, st);
+static tg_status stage_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, const uint32_t* ts,
+                             int64_t n_edges, float* scores, cudaStream_t st, Staged& o) {
+  const bool dev_in = is_device_ptr(src);
+  const bool dev_out = is_device_ptr(scores);
+  o.src = src;
+  o.dst = dst;
+  o.ts = ts;
+  o.out = scores;
+  o.host_out = !dev_out;
+  if (dev_in && dev_out) return TG_OK;
+  TRY(ensure_stage(ctx, (size_t)n_edges * 16 + 64));
+  char* stg = (char*)ctx->stage;
+  if (!dev_in) {  // host -> device copies of this call's inputs (H2D)
+    CK(cudaMemcpyAsync(stg, src, n_edges * 4, cudaMemcpyHostToDevice, st));
+    CK(cudaMemcpyAsync(stg + n_edges * 4, dst, n_edges * 4, cudaMemcpyHostToDevice, st));
+    CK(cudaMemcpyAsync(stg + n_edges * 8, ts, n_edges * 4, cudaMemcpyHostToDevice, st));
+    o.src = (const int32_t*)stg;
+    o.dst = (const int32_t*)(stg + n_edges * 4);
+    o.ts = (const uint32_t*)(stg + n_edges * 8);
   }
-  TRY(launched(ctx));
-  TRY(run_embed_counted(ctx, cnt, st));
-  Prof pf(ctx, TG_ST_SCORE, st);
-  launch_score(ctx->HL, ctx->dnp, ctx->inv[ctx->L], (int)n_edges, batch, bidx, ctx->Wa1, ctx->ba1, ctx->Wa2,
-               ctx->ba2, ctx->d_n, ctx->dnp, scores, st);
-  return launched(ctx);
+  if (!dev_out) o.out = (float*)(stg + n_edges * 12);
+  return TG_OK;
 }
 
 tg_status tg_score_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, const uint32_t* ts, int64_t n_edges,
@@ -754,30 +811,16 @@ tg_status tg_score_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, co
   if (!ctx) return TG_EINVAL;
   if (!ctx->loaded) return TG_ESTATE;
   if (ctx->broken) return TG_ECUDA;
-  if (n_edges < 0 || 2 * n_edges > ctx->capI[ctx->L] || (n_edges > 0 && (!src || !dst || !ts || !scores)))
+  if (n_edges < 0 || 2 * n_edges > ctx->cap[ctx->L] || (n_edges > 0 && (!src || !dst || !ts || !scores)))
     return TG_EINVAL;
+  if (n_edges == 0) return TG_OK;
   cudaStream_t st = (cudaStream_t)cuda_stream;
   CK(cudaSetDevice(ctx->device));
-  const bool dev_in = n_edges == 0 || is_device_ptr(src);
-  const bool dev_out = n_edges == 0 || is_device_ptr(scores);
-  const int32_t *ds = src, *dd = dst;
-  const uint32_t* dts = ts;
-  float* dsc = scores;
-  if (!dev_in || !dev_out) TRY(ensure_stage(ctx, (size_t)n_edges * 16 + 64));
-  char* stg = (char*)ctx->stage;
-  if (!dev_in) {
-    CK(cudaMemcpyAsync(stg, src, n_edges * 4, cudaMemcpyHostToDevice, st));
-    CK(cudaMemcpyAsync(stg + n_edges * 4, dst, n_edges * 4, cudaMemcpyHostToDevice, st));
-    CK(cudaMemcpyAsync(stg + n_edges * 8, ts, n_edges * 4, cudaMemcpyHostToDevice, st));
-    ds = (const int32_t*)stg;
-    dd = (const int32_t*)(stg + n_edges * 4);
-    dts = (const uint32_t*)(stg + n_edges * 8);
-  }
-  if (!dev_out) dsc = (float*)(stg + n_edges * 12);
-  TRY(score_edges_dev(ctx, ds, dd, dts, n_edges, (int)std::max<int64_t>(n_edges, 1), nullptr, dsc, ctx->cnt_total,
-                      st));
-  if (!dev_out) {
-    CK(cudaMemcpyAsync(scores, dsc, n_edges * 4, cudaMemcpyDeviceToHost, st));
+  Staged o;
+  TRY(stage_edges(ctx, src, dst, ts, n_edges, scores, st, o));
+  TRY(stream_edges(ctx, o.src, o.dst, o.ts, n_edges, (int)n_edges, o.out, nullptr, st));
+  if (o.host_out) {
+    CK(cudaMemcpyAsync(scores, o.out, n_edges * 4, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
   }
   return TG_OK;
@@ -788,41 +831,16 @@ tg_status tg_score_stream(tg_ctx* ctx, const int32_t* src, const int32_t* dst, c
   if (!ctx) return TG_EINVAL;
   if (!ctx->loaded) return TG_ESTATE;
   if (ctx->broken) return TG_ECUDA;
-  if (n_edges < 0 || batch < 1 || 2 * batch > ctx->capI[ctx->L] || (n_edges > 0 && (!src || !dst || !ts || !scores)))
+  if (n_edges < 0 || batch < 1 || 2 * batch > ctx->cap[ctx->L] || (n_edges > 0 && (!src || !dst || !ts || !scores)))
     return TG_EINVAL;
   if (n_edges == 0) return TG_OK;
   cudaStream_t st = (cudaStream_t)cuda_stream;
   CK(cudaSetDevice(ctx->device));
-  const bool dev_in = is_device_ptr(src);
-  const bool dev_out = is_device_ptr(scores);
-  const int32_t *ds = src, *dd = dst;
-  const uint32_t* dts = ts;
-  float* dsc = scores;
-  if (!dev_in || !dev_out) TRY(ensure_stage(ctx, (size_t)n_edges * 16 + 64));
-  char* stg = (char*)ctx->stage;
-  if (!dev_in) {
-    CK(cudaMemcpyAsync(stg, src, n_edges * 4, cudaMemcpyHostToDevice, st));
-    CK(cudaMemcpyAsync(stg + n_edges * 4, dst, n_edges * 4, cudaMemcpyHostToDevice, st));
-    CK(cudaMemcpyAsync(stg + n_edges * 8, ts, n_edges * 4, cudaMemcpyHostToDevice, st));
-    ds = (const int32_t*)stg;
-    dd = (const int32_t*)(stg + n_edges * 4);
-    dts = (const uint32_t*)(stg + n_edges * 8);
-  }
-  if (!dev_out) dsc = (float*)(stg + n_edges * 12);
-  const int64_t nb = (n_edges + batch - 1) / batch;
-  CK(cudaMemsetAsync(ctx->bidx, 0, sizeof(int), st));
-  CK(cudaMemsetAsync(ctx->cnt_tmp, 0, TG_NCOUNTERS * sizeof(long long), st));
-  for (int64_t b = 0; b < nb; ++b) {
-    TRY(score_edges_dev(ctx, ds, dd, dts, n_edges, batch, ctx->bidx, dsc, ctx->cnt_tmp, st));
-    {
-      Prof pf(ctx, TG_ST_OTHER, st);
-      k_finish_batch<<<1, 64, 0, st>>>(ctx->cnt_tmp, ctx->cnt_total, (long long*)batch_counters, ctx->bidx,
-                                       TG_NCOUNTERS);
-    }
-    TRY(launched(ctx));
-  }
-  if (!dev_out) {
-    CK(cudaMemcpyAsync(scores, dsc, n_edges * 4, cudaMemcpyDeviceToHost, st));
+  Staged o;
+  TRY(stage_edges(ctx, src, dst, ts, n_edges, scores, st, o));
+  TRY(stream_edges(ctx, o.src, o.dst, o.ts, n_edges, batch, o.out, (long long*)batch_counters, st));
+  if (o.host_out) {  // device -> host read of the results (D2H)
+    CK(cudaMemcpyAsync(scores, o.out, n_edges * 4, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
   }
   return TG_OK;
@@ -882,9 +900,17 @@ tg_status tg_dedup(tg_ctx* ctx, const int32_t* nodes, const uint32_t* ts, int64_
   CK(cudaMalloc(&ndev, sizeof(int)));
   int nn = (int)n;
   CK(cudaMemcpyAsync(ndev, &nn, sizeof(int), cudaMemcpyHostToDevice, st));
-  Level in{const_cast<int32_t*>(nodes), const_cast<uint32_t*>(ts), (int)n};
-  Level out{uniq_nodes, uniq_ts, (int)n};
-  launch_dedup(in, ndev, (int)std::max<int64_t>(n, 1), out, inv, n_uniq, nullptr, nullptr, true, ctx->err, st);
+  LevelDev v{};
+  v.cap = (int)std::max<int64_t>(n, 1);
+  v.in_node = const_cast<int32_t*>(nodes);
+  v.in_ts = const_cast<uint32_t*>(ts);
+  v.n_in = ndev;
+  v.u_node = uniq_nodes;
+  v.u_ts = uniq_ts;
+  v.n_u = n_uniq;
+  v.inv = inv;
+  EdgeSrc none{};
+  launch_dedup(v, 1, v.cap, false, none, nullptr, 0, true, ctx->err, st);
   cudaError_t e = cudaGetLastError();
   cudaStreamSynchronize(st);
   cudaFree(ndev);
@@ -893,31 +919,37 @@ tg_status tg_dedup(tg_ctx* ctx, const int32_t* nodes, const uint32_t* ts, int64_
 
 tg_status tg_sample(tg_ctx* ctx, const int32_t* nodes, const uint32_t* ts, int64_t n, int32_t* nbr, int32_t* eid,
                     uint32_t* nts, void* cuda_stream) {
-  if (!ctx || n < 0 || !ctx->loaded) return !ctx || n < 0 ? TG_EINVAL : TG_ESTATE;
+  if (!ctx || n < 0) return TG_EINVAL;
+  if (!ctx->loaded) return TG_ESTATE;
   if (n == 0) return TG_OK;
   if (!nodes || !ts || !nbr || !eid || !nts) return TG_EINVAL;
   cudaStream_t st = (cudaStream_t)cuda_stream;
   CK(cudaSetDevice(ctx->device));
-  const int k = ctx->k;
-  int *ndev = nullptr, *nnext = nullptr;
-  int32_t* nx = nullptr;
-  uint32_t* nt = nullptr;
-  CK(cudaMalloc(&ndev, 2 * sizeof(int)));
-  nnext = ndev + 1;
-  CK(cudaMalloc(&nx, (size_t)n * (k + 1) * 4));
-  CK(cudaMalloc(&nt, (size_t)n * (k + 1) * 4));
-  int nn = (int)n;
-  CK(cudaMemcpyAsync(ndev, &nn, sizeof(int), cudaMemcpyHostToDevice, st));
-  Level C{const_cast<int32_t*>(nodes), const_cast<uint32_t*>(ts), (int)n};
-  Level next{nx, nt, (int)(n * (k + 1))};
-  launch_sample(ctx->g, C, ndev, (int)n, k, next, eid, nnext, ctx->err, st);
+  // a one-batch compute list over the caller's targets
+  int* meta = nullptr;
+  int32_t* cb = nullptr;
+  CK(cudaMalloc(&meta, 4 * sizeof(int)));
+  CK(cudaMalloc(&cb, (size_t)n * sizeof(int32_t)));
+  CK(cudaMemsetAsync(cb, 0, (size_t)n * sizeof(int32_t), st));
+  int h[4] = {0, (int)n, (int)n, 0};  // c_base[0], n_c[0], n_c_total
+  CK(cudaMemcpyAsync(meta, h, sizeof(h), cudaMemcpyHostToDevice, st));
+  LevelDev v{};
+  v.cap = (int)n;
+  v.c_cap = (int)n;
+  v.c_b = cb;
+  v.c_node = const_cast<int32_t*>(nodes);
+  v.c_ts = const_cast<uint32_t*>(ts);
+  v.c_base = meta;
+  v.n_c = meta + 1;
+  v.n_c_total = meta + 2;
+  v.nb_node = nbr;
+  v.nb_ts = nts;
+  v.nb_eid = eid;
+  launch_sample(ctx->g, v, 1, ctx->k, nullptr, ctx->W, 0, nullptr, 0, ctx->err, st);
   cudaError_t e = cudaGetLastError();
-  cudaMemcpyAsync(nbr, nx + n, (size_t)n * k * 4, cudaMemcpyDeviceToDevice, st);
-  cudaMemcpyAsync(nts, nt + n, (size_t)n * k * 4, cudaMemcpyDeviceToDevice, st);
   cudaStreamSynchronize(st);
-  cudaFree(ndev);
-  cudaFree(nx);
-  cudaFree(nt);
+  cudaFree(meta);
+  cudaFree(cb);
   return e == cudaSuccess ? TG_OK : TG_ECUDA;
 }
 

@@ -8,6 +8,13 @@
 //   kv rows    [hn (dnp) | ef (dep) | Phi (dtp)] = Dp floats, dXp = round4(dX)
 //   ring_l     float [C x ldn] FIFO ring of cached layer-l embeddings
 //   index_l    {u64 key, i64 logical pos} open addressing, linear probing
+//
+// Superbatch: S consecutive batches share one launch
+// sequence. Per recursion level l the *dedup lists* (I_l, U_l, inv_l, slot_l)
+// are batch-segmented with a fixed per-batch stride `cap`; the *compute list*
+// C_l (targets whose embedding is computed at layer l) is compacted over the
+// superbatch in (batch, unique-list) order, with its neighbour slots stored
+// compute-centric at [q*k + m].
 #pragma once
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -19,9 +26,11 @@ namespace tg {
 constexpr unsigned long long kEmptyKey = 0xFFFFFFFFFFFFFFFFull;
 constexpr unsigned long long kLockedKey = 0xFFFFFFFFFFFFFFFEull;
 constexpr int kMaxK = 32;          // neighbours per target (warp lanes)
+constexpr int kMaxS = 64;          // batches per superbatch
 constexpr int kDedupThreads = 1024;
 constexpr int kDedupIPT = 16;      // items per thread per CTA (ordered scan)
-constexpr int kDedupSlots = 16384; // smem hash slots per CTA (load <= 0.5 target)
+constexpr int kDedupSlots = 16384; // smem hash slots per CTA (load <= ~0.6)
+constexpr int kProbeIPT = 16;
 
 // device error bits (sticky)
 enum : int { kErrNodeRange = 1, kErrIndexFull = 2, kErrDedupFull = 4, kErrEidRange = 8 };
@@ -53,13 +62,6 @@ struct GraphDev {
   int d_n, d_e, ldn, lde;
 };
 
-// Target list of one recursion level: I_l = [C_{l+1} ; N(C_{l+1})] (Alg. 1 l.12).
-struct Level {
-  int32_t* node;   // [cap]
-  uint32_t* ts;    // [cap]
-  int cap;
-};
-
 struct CacheDev {
   unsigned long long* ikey;  // [icap]
   long long* ipos;           // [icap]
@@ -69,40 +71,78 @@ struct CacheDev {
   long long* state;          // device [4]: head, size, limit, occupied index slots
 };
 
+// One recursion level l >= 1 of a superbatch.
+struct LevelDev {
+  int cap;                   // per-batch stride of the segmented lists
+  // batch-segmented (stride cap): input I_l, unique U_l, inverse, ring slot per U entry
+  int32_t* in_node;
+  uint32_t* in_ts;
+  int* n_in;                 // [S]
+  int32_t* u_node;
+  uint32_t* u_ts;
+  int* n_u;                  // [S]
+  int32_t* inv;
+  long long* slot;
+  // compute list C_l, compacted over the superbatch (q = 0..n_c_total-1)
+  int32_t* c_b;              // batch of q
+  int32_t* c_u;              // unique-list index of q inside its batch
+  int32_t* c_node;
+  uint32_t* c_ts;
+  int* c_base;               // [S] first q of each batch
+  int* n_c;                  // [S]
+  int* n_c_total;            // [1]
+  int c_cap;                 // S * cap
+  // sampled neighbours of each q (compute-centric [q*k + m])
+  int32_t* nb_node;
+  uint32_t* nb_ts;
+  int32_t* nb_eid;
+  // row addresses resolved for the layer-l compute
+  const float** hs_row;      // [c_cap]     h^(l-1) of the target
+  const float** nb_row;      // [c_cap * k] h^(l-1) of each neighbour
+  float** dst_row;           // [c_cap]     where h^(l) goes (ring slot or H_L)
+};
+
+// per-superbatch counter rows: cnt[b * TG_NCOUNTERS + c]
+__device__ __forceinline__ void cnt_add(long long* cnt, int b, int c, long long v) {
+  if (cnt && v) atomicAdd((unsigned long long*)(cnt + (size_t)b * TG_NCOUNTERS + c), (unsigned long long)v);
+}
+
 // -------------------------------------------------------------- launchers
-// All launchers are stream-ordered; counts marked *_dev are device scalars.
+struct EdgeSrc {            // batch b of the superbatch = edges [e0 + b*B, +B) clipped to n_edges
+  const int32_t* src;
+  const int32_t* dst;
+  const uint32_t* ts;
+  int64_t n_edges;
+  int64_t e0;
+  int B;
+};
 
-// targets = src || dst at the batch's edge times; batch picked by *bidx
-void launch_prep_edges(const int32_t* src, const int32_t* dst, const uint32_t* ts, int64_t n_edges,
-                       int batch, const int* bidx, Level out, int* n_out_dev, cudaStream_t st);
-void launch_prep_nodes(const int32_t* nodes, const uint32_t* ts, int n, Level out, int* n_out_dev,
-                       cudaStream_t st);
+// DedupFilter (Alg. 2) of every batch segment of level `lv`, one cluster per batch.
+// edge_mode: the level-L input is src || dst of the batch, read from `es`.
+void launch_dedup(LevelDev lv, int S, int n_max, bool edge_mode, EdgeSrc es, long long* cnt, int layer,
+                  bool dedup_on, int* err, cudaStream_t st);
 
-// DedupFilter (Alg. 2); n from *n_dev (<= n_max). Writes U, inv, *nu_dev; adds counters.
-void launch_dedup(Level in, const int* n_dev, int n_max, Level uniq, int32_t* inv, int* nu_dev,
-                  long long* cnt_n, long long* cnt_u, bool dedup_on, int* err, cudaStream_t st);
+// CacheLookup + compaction + slot assignment + index insert, sequential over
+// the S batches (Alg. 1 l.7-10 and CacheStore, Alg. 3, in batch order).
+// cache == nullptr: no lookup (top layer, R9, or cache disabled).
+void launch_probe(LevelDev lv, int S, const CacheDev* cache, long long* cnt, int layer, int* err,
+                  cudaStream_t st);
 
-// CacheLookup + slot assignment + index insert (Alg. 1 l.7-10, 17; Alg. 3).
-// Writes the miss list C (as U indices and node/ts), slot[u] for every u.
-void launch_probe(Level uniq, const int* nu_dev, int nu_max, CacheDev cache, bool cache_on,
-                  int32_t* c_uidx, Level C, int* nc_dev, long long* slot, long long* cnt_layer,
-                  int* err, cudaStream_t st);
+// NghLookup for every q of level `lv`; writes lv.nb_* and,
+// if next != nullptr, the batch-segmented input list of level l-1 (Alg. 1 l.12).
+void launch_sample(const GraphDev& g, LevelDev lv, int S, int k, const LevelDev* next, int W, int use_table,
+                   long long* cnt, int layer, int* err, cudaStream_t st);
 
-// C_L = U_L (top layer: no lookup): identity miss list.
-void launch_copy_level(Level in, const int* n_dev, int n_max, Level out, int32_t* c_uidx, int* n_out_dev,
-                       long long* cnt_lookup_miss, cudaStream_t st);
-
-// NghLookup: k most recent with t_j < t; writes I_{l-1} =
-// [C ; N(C)] plus eid[p*k+m]; *n_next_dev = nC*(k+1).
-void launch_sample(const GraphDev& g, Level C, const int* nc_dev, int nc_max, int k, Level next,
-                   int32_t* eid, int* n_next_dev, int* err, cudaStream_t st);
-
-// Row addresses for layer l: rows[j] for j in I_{l-1}; dst[p] for p in C_l.
-void launch_resolve(const GraphDev& g, int lm1_is_zero, Level prev, const int* nprev_dev, int nprev_max,
-                    const int32_t* inv_prev, const long long* slot_prev, const float* ring_prev,
-                    long long rcap_prev, int ld, const int* nc_dev, int nc_max, const int32_t* c_uidx,
-                    const long long* slot_cur, float* ring_cur, long long rcap_cur, float* hl_out,
-                    const float** rows, float** dst, int* err, cudaStream_t st);
+// Row addresses for the layer-l compute of every level (one launch).
+struct ResolveArgs {
+  LevelDev lv[TG_MAX_LAYERS + 1];
+  float* ring[TG_MAX_LAYERS + 1];   // ring of level l (null for l = L)
+  float* HL;
+  const float* X;
+  int ldn, k, L;
+  int c_cap_max;
+};
+void launch_resolve(const ResolveArgs& a, int* err, cudaStream_t st);
 
 // Phi table [W x dtp] built on device with the same function as the direct path.
 void launch_time_table(const float* omega, const float* phi, int d_t, int dtp, int W, float* table,
@@ -111,12 +151,13 @@ void launch_time_encode(const float* omega, const float* phi, const float* table
                         int use_table, const int64_t* delta, int64_t n, float* out, cudaStream_t st);
 
 struct AttnArgs {
-  const float* u;          // [nc x 2Dp] (H*Dp)
+  const float* u;          // [nc x H*Dp]
   float* c;                // [nc x H*Dp]
-  const float** rows;      // I_{l-1} row addresses
-  const int32_t* prev_node;   // I_{l-1} nodes (mask: node == 0)
-  const uint32_t* prev_ts;    // I_{l-1} times
-  const int32_t* eid;      // [nc x k]
+  const float* const* nb_row;
+  const int32_t* nb_node;  // mask: node == 0 (R7)
+  const uint32_t* nb_ts;
+  const int32_t* nb_eid;
+  const uint32_t* c_ts;
   const float* Ef;
   int lde;
   const float* omega;
@@ -126,7 +167,6 @@ struct AttnArgs {
   int dnp, dep, dtp, d_t, Dp, H, k;
   const int* nc_dev;
   int nc_max;
-  long long* cnt_ttable;   // [2] table, direct
 };
 void launch_attn(const AttnArgs& a, cudaStream_t st);
 
@@ -161,13 +201,15 @@ void launch_gemm_simt(const GemmArgs& g, cudaStream_t st);
 void launch_layernorm(const float* y, float* r, int Dp, int dn, int dnp, int de, int dep, int dt,
                       const float* gamma, const float* beta, const int* m_dev, int m_max, cudaStream_t st);
 
-// Scores p_e = sigmoid(MLP(h_src, h_dst)) (R10) and inversion out[i] = H_L[inv[i]].
-void launch_score(const float* HL, int ldh, const int32_t* inv, int n_edges, int batch, const int* bidx,
-                  const float* Wa1, const float* ba1, const float* Wa2, float ba2, int dn, int dnp,
-                  float* scores, cudaStream_t st);
-void launch_invert(const float* HL, int ldh, const int32_t* inv, int n, int dn, float* out, cudaStream_t st);
+// Scores p_e = sigmoid(MLP(h_src, h_dst)) (R10) for every edge of the superbatch.
+void launch_score(const float* HL, int ldh, LevelDev top, int S, EdgeSrc es, const float* Wa1, const float* ba1,
+                  const float* Wa2, float ba2, int dn, int dnp, float* scores, cudaStream_t st);
+// out[i] = H_L[q(i)] for a single-batch embed call (DedupInvert, Alg. 1 l.20).
+void launch_invert(const float* HL, int ldh, LevelDev top, int n, int dn, float* out, cudaStream_t st);
+void launch_prep_nodes(const int32_t* nodes, const uint32_t* ts, int n, LevelDev top, cudaStream_t st);
 
-void launch_bump(int* bidx, cudaStream_t st);
-void launch_add_counters(const long long* src, long long* dst, int n, cudaStream_t st);
+// fold the superbatch counter rows into the totals and the per-batch log
+void launch_finish(long long* cnt_sb, int S, long long* total, long long* log, int64_t log_row0,
+                   cudaStream_t st);
 
 }  // namespace tg

@@ -45,7 +45,7 @@ class ModelCfg(ctypes.Structure):
     _fields_ = [("n_layers", ctypes.c_int32), ("n_heads", ctypes.c_int32), ("n_neighbors", ctypes.c_int32),
                 ("d_t", ctypes.c_int32), ("max_batch_targets", ctypes.c_int32),
                 ("cache_limit", ctypes.c_int64), ("time_window", ctypes.c_int32),
-                ("opts", ctypes.c_uint32), ("precision", ctypes.c_int32)]
+                ("opts", ctypes.c_uint32), ("precision", ctypes.c_int32), ("superbatch", ctypes.c_int32)]
 
 
 _lib = None
@@ -142,11 +142,12 @@ class Context:
         return cls(stream.n_nodes, stream.src, stream.dst, stream.ts, stream.node_feat, stream.edge_feat, device)
 
     def load_model(self, params, n_layers=2, n_heads=2, n_neighbors=20, d_t=None, max_batch_targets=400,
-                   cache_limit=2_000_000, time_window=10_000, opts=TG_OPT_ALL, precision=TG_PREC_FP32):
+                   cache_limit=2_000_000, time_window=10_000, opts=TG_OPT_ALL, precision=TG_PREC_FP32,
+                   superbatch=0):
         d_t = self.d_n if d_t is None else d_t
         p = np.ascontiguousarray(params, np.float32)
         cfg = ModelCfg(n_layers, n_heads, n_neighbors, d_t, max_batch_targets, cache_limit, time_window,
-                       opts, precision)
+                       opts, precision, superbatch)
         _check(lib().tg_model_load(self.h, ctypes.byref(cfg), _ptr(p), p.size), "tg_model_load")
         self.cfg = cfg
         return self

@@ -22,13 +22,13 @@ def setup(name, n_edges=None, **model_over):
     return cfg, s, flat
 
 
-def make_ctx(s, flat, mc, precision=0, opts=7, cache_limit=None, max_targets=None, device=0):
+def make_ctx(s, flat, mc, precision=0, opts=7, cache_limit=None, max_targets=None, device=0, superbatch=0):
     from paper_conf_ppopp_wangm23_b200 import Context
     ctx = Context.from_stream(s, device=device)
     ctx.load_model(flat, n_layers=mc.n_layers, n_heads=mc.n_heads, n_neighbors=mc.n_neighbors,
                    max_batch_targets=max_targets or 2 * mc.batch,
                    cache_limit=mc.cache_limit if cache_limit is None else cache_limit,
-                   time_window=mc.time_window, opts=opts, precision=precision)
+                   time_window=mc.time_window, opts=opts, precision=precision, superbatch=superbatch)
     return ctx
 
 

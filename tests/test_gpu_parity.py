@@ -260,3 +260,24 @@ def test_score_edges_host_buffers_match_stream():
         b.score_edges(s.src[lo:hi].copy(), s.dst[lo:hi].copy(), s.ts[lo:hi].copy(), tmp)
         out[lo:hi] = tmp
     assert np.array_equal(out, sc)
+
+
+@pytest.mark.parametrize("limit", [2_000_000, 700])
+def test_superbatch_invariance_bitexact(limit):
+    """S batches per launch sequence change neither outputs nor per-batch counters."""
+    cfg, s, flat = setup("config1", n_edges=4000)
+    mc = cfg.model
+    ref_sc = ref_log = None
+    for S in (1, 3, 16):
+        ctx = make_ctx(s, flat, mc, cache_limit=limit, superbatch=S)
+        sc, log = _stream_gpu(ctx, s, mc.batch)
+        if ref_sc is None:
+            ref_sc, ref_log = sc, log
+        else:
+            assert np.array_equal(sc, ref_sc), S
+            assert np.array_equal(log, ref_log), S
+        ctx.close()
+    want = _sim_counters(s, flat, mc, limit)
+    from paper_conf_ppopp_wangm23_b200 import counters_dict
+    for b, w in enumerate(want):
+        assert counters_dict(ref_log[b], mc.n_layers) == w, b
