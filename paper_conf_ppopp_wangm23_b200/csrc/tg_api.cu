@@ -965,6 +965,48 @@ tg_status tg_time_encode(tg_ctx* ctx, const int64_t* delta, int64_t n, int32_t u
   return TG_OK;
 }
 
+tg_status tg_gemm(tg_ctx* ctx, int32_t precision, int32_t M, int32_t N, int32_t K, const float* A,
+                  const float* B, const float* bias, int32_t relu, float* C, void* cuda_stream) {
+  if (!ctx || M < 0 || N < 4 || K < 4 || (N & 3) || (K & 3) || !A || !B || !C) return TG_EINVAL;
+  if (precision < TG_PREC_FP32 || precision > TG_PREC_BF16) return TG_EINVAL;
+  cudaStream_t st = (cudaStream_t)cuda_stream;
+  CK(cudaSetDevice(ctx->device));
+  int* mdev = nullptr;
+  CK(cudaMalloc(&mdev, sizeof(int)));
+  CK(cudaMemcpy(mdev, &M, sizeof(int), cudaMemcpyHostToDevice));
+  GemmArgs g{};
+  g.a_base0 = A;
+  g.lda0 = K;
+  g.K0 = g.K = K;
+  g.B = B;
+  g.N = N;
+  g.bias = bias;
+  g.relu = relu;
+  g.C = C;
+  g.ldc = N;
+  g.m_dev = mdev;
+  g.m_max = std::max(M, 1);
+  tg_status s = TG_OK;
+  if (precision == TG_PREC_FP32) {
+    launch_gemm_simt(g, st);
+  } else {
+    std::vector<void*> owned;
+    TcWeights w;
+    s = tc_prepare_weights(B, N, K, precision, &w, owned);
+    if (s == TG_OK) launch_gemm_tc(g, w, precision, st);
+    cudaStreamSynchronize(st);
+    for (void* p : owned) cudaFree(p);
+  }
+  cudaError_t e = cudaGetLastError();
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  cudaFree(mdev);
+  if (e != cudaSuccess) {
+    fprintf(stderr, "libtg: tg_gemm %s\n", cudaGetErrorString(e));
+    return TG_ECUDA;
+  }
+  return s;
+}
+
 void tg_free(tg_ctx* ctx) {
   if (!ctx) return;
   cudaSetDevice(ctx->device);

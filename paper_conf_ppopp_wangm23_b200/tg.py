@@ -25,7 +25,7 @@ COUNTER_FIELDS = ("n", "unique", "lookups", "hits", "misses", "evicted")
 EXPORTS = ("tg_graph_load", "tg_model_load", "tg_embed_batch", "tg_score_edges", "tg_score_stream",
            "tg_cache_reset", "tg_counters_read", "tg_dedup", "tg_sample", "tg_time_encode",
            "tg_kernel_launches", "tg_free", "tg_strerror", "tg_version", "tg_profile_enable",
-           "tg_profile_read")
+           "tg_profile_read", "tg_gemm")
 STAGES = ("prep", "dedup", "lookup", "sample", "resolve", "proj_k", "attn", "proj_v", "lnorm", "ffn1", "ffn2",
           "score", "other")
 
@@ -71,6 +71,7 @@ def lib():
         L.tg_time_encode.argtypes = [vp, vp, i64, i32, vp, vp]
         L.tg_profile_enable.argtypes = [vp, i32]
         L.tg_profile_read.argtypes = [vp, vp, vp, i32]
+        L.tg_gemm.argtypes = [vp, i32, i32, i32, i32, vp, vp, vp, i32, vp, vp]
         L.tg_kernel_launches.argtypes = [vp]
         L.tg_kernel_launches.restype = i64
         L.tg_free.argtypes = [vp]
@@ -80,7 +81,7 @@ def lib():
         L.tg_version.restype = ctypes.c_char_p
         for f in ("tg_graph_load", "tg_model_load", "tg_embed_batch", "tg_score_edges", "tg_score_stream",
                   "tg_cache_reset", "tg_counters_read", "tg_dedup", "tg_sample", "tg_time_encode",
-                  "tg_profile_enable", "tg_profile_read"):
+                  "tg_profile_enable", "tg_profile_read", "tg_gemm"):
             getattr(L, f).restype = ctypes.c_int
         _lib = L
     return _lib
@@ -198,6 +199,14 @@ class Context:
         cnt = np.zeros(len(STAGES), np.int64)
         _check(lib().tg_profile_read(self.h, ms.ctypes.data, cnt.ctypes.data, len(STAGES)), "tg_profile_read")
         return {s: (float(m), int(c)) for s, m, c in zip(STAGES, ms, cnt)}
+
+    def gemm(self, A, B, C, bias=None, relu=False, precision=TG_PREC_FP32, stream=None):
+        """C = A B^T (+bias, ReLU) with the library's dense-projection kernels (unit entry)."""
+        M, K = A.shape
+        N = B.shape[0]
+        _check(lib().tg_gemm(self.h, int(precision), int(M), int(N), int(K), _ptr(A), _ptr(B), _ptr(bias),
+                             int(bool(relu)), _ptr(C), _stream(stream)), "tg_gemm")
+        return C
 
     def kernel_launches(self):
         return int(lib().tg_kernel_launches(self.h))

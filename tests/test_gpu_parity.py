@@ -13,6 +13,7 @@ from synth import make_stream
 from tests.gpu_helpers import close, setup, make_ctx, make_oracle
 
 pytestmark = pytest.mark.gpu
+TOL = {0: (1e-4, 1e-5), 1: (1e-4, 1e-5), 2: (2e-2, 2e-2)}   # fp32 / tf32x3 / bf16: (rtol, atol)
 
 
 @pytest.fixture(scope="module", autouse=True)
@@ -142,13 +143,14 @@ def _embed_gpu(ctx, nodes, ts, d_n):
     return out.cpu().numpy().reshape(len(nodes), d_n)
 
 
+@pytest.mark.parametrize("prec", [0, 1, 2])
 @pytest.mark.parametrize("name,L", [("tiny", 1), ("tiny", 2), ("tiny_bip", 2), ("config1", 2), ("tiny", 3)])
-def test_embed_parity(name, L):
+def test_embed_parity(name, L, prec):
     cfg, s, flat = setup(name, n_layers=L)
     mc = cfg.model
     from synth import make_params
     flat = make_params(L, mc.n_heads, s.d_n, s.d_e)
-    ctx = make_ctx(s, flat, mc, max_targets=256)
+    ctx = make_ctx(s, flat, mc, max_targets=256, precision=prec)
     o = make_oracle(s, flat, mc)
     rng = np.random.default_rng(3)
     n = 256 if name != "config1" else 64
@@ -160,7 +162,7 @@ def test_embed_parity(name, L):
     for rep in range(2):                               # second pass is served by the memo cache
         got = _embed_gpu(ctx, nodes, ts, s.d_n)
         ref = o.embed(L, nodes, ts)
-        ok, err, nbad = close(got, ref)
+        ok, err, nbad = close(got, ref, *TOL[prec])
         assert ok, (rep, err, nbad)
 
 
@@ -217,11 +219,12 @@ def test_stream_counters_bitexact(name, limit):
     assert tot["l1_misses"] == sum(w["l1_misses"] for w in want)
 
 
+@pytest.mark.parametrize("prec", [0, 1, 2])
 @pytest.mark.parametrize("name", ["tiny_bip", "config1"])
-def test_stream_scores_parity(name):
+def test_stream_scores_parity(name, prec):
     cfg, s, flat = setup(name)
     mc = cfg.model
-    ctx = make_ctx(s, flat, mc)
+    ctx = make_ctx(s, flat, mc, precision=prec)
     scores, _ = _stream_gpu(ctx, s, mc.batch)
     o = make_oracle(s, flat, mc)
     nb = (s.n_edges + mc.batch - 1) // mc.batch
@@ -229,7 +232,7 @@ def test_stream_scores_parity(name):
     for b in picks:
         lo, hi = b * mc.batch, min((b + 1) * mc.batch, s.n_edges)
         _, ref = o.infer_batch(s.src[lo:hi], s.dst[lo:hi], s.ts[lo:hi])
-        ok, err, nbad = close(scores[lo:hi], ref)
+        ok, err, nbad = close(scores[lo:hi], ref, *TOL[prec])
         assert ok, (b, err, nbad)
 
 
@@ -281,3 +284,22 @@ def test_superbatch_invariance_bitexact(limit):
     from paper_conf_ppopp_wangm23_b200 import counters_dict
     for b, w in enumerate(want):
         assert counters_dict(ref_log[b], mc.n_layers) == w, b
+
+
+# ------------------------------------------------------------- GEMM kernels
+@pytest.mark.parametrize("prec,rtol,atol", [(0, 1e-5, 1e-5), (1, 1e-5, 1e-4), (2, 2e-2, 2e-2)])
+@pytest.mark.parametrize("M,N,K", [(1, 16, 8), (130, 176, 172), (6400, 1032, 172), (700, 516, 1032),
+                                   (257, 172, 688)])
+def test_gemm_kernels_vs_torch_float64(prec, rtol, atol, M, N, K):
+    cfg, s, flat = setup("tiny")
+    ctx = make_ctx(s, flat, cfg.model)
+    g = torch.Generator(device="cpu").manual_seed(M + N + K)
+    A = torch.randn(M, K, generator=g).cuda()
+    B = (torch.randn(N, K, generator=g) / K ** 0.5).cuda()
+    bias = torch.randn(N, generator=g).cuda()
+    C = torch.zeros(M, N, device="cuda")
+    ctx.gemm(A, B, C, bias=bias, relu=True, precision=prec)
+    ref = torch.relu(A.double() @ B.double().T + bias.double())
+    err = (C.double() - ref).abs()
+    bound = atol + rtol * ref.abs()
+    assert bool((err <= bound).all()), (prec, float(err.max()))
