@@ -397,6 +397,382 @@ k_probe(LevelDev lv, int S, CacheDev c, int use_cache, int has_ring, long long* 
   }
 }
 
+// ---------------------------------------------- cached levels, in parallel
+// The same CacheLookup/CacheStore semantics as k_probe, in three launches:
+//  (1) k_probe_pre: read-only lookup of every key of the superbatch in the
+//      global index (state at superbatch start) -- fully parallel;
+//  (2) k_probe_seq: one thread-block cluster walks the batches in order and
+//      decides hit / miss per batch against (a) keys first missed earlier in
+//      this superbatch, kept in a DSMEM hash, else (b) the pre-looked-up
+//      position; misses get FIFO positions head0 + q (q = rank in the
+//      superbatch's compute list, since positions are handed out in order);
+//  (3) k_probe_ins: parallel insert of the superbatch's misses into the
+//      global index (key -> head0 + q), skipping keys re-missed later.
+// The newest copy of a key is always first on its probe chain (an insert
+// takes the first dead or empty slot), so lookups stop at the first match.
+__global__ void k_probe_pre(LevelDev lv, int S, CacheDev c) {
+  const int tot = S * lv.cap;
+  for (int idx = blockIdx.x * blockDim.x + threadIdx.x; idx < tot; idx += gridDim.x * blockDim.x) {
+    const int b = idx / lv.cap, i = idx - b * lv.cap;
+    if (i >= lv.n_u[b]) continue;
+    const unsigned long long key = tkey(lv.u_node[idx], lv.u_ts[idx]);
+    unsigned long long h = mix64(key) & c.imask;
+    long long p = -1;
+    for (unsigned long long pr = 0; pr <= c.imask; ++pr) {
+      const unsigned long long k0 = c.ikey[h];
+      if (k0 == kEmptyKey) break;
+      if (k0 == key) {
+        p = c.ipos[h];
+        break;
+      }
+      h = (h + 1) & c.imask;
+    }
+    lv.p0[idx] = p;
+  }
+}
+
+constexpr int kSeqCL = 16;        // cluster CTAs of the ordered pass
+constexpr int kSeqThreads = 1024;
+constexpr int kSeqSlots = 16384;  // DSMEM hash slots per CTA
+
+__global__ void __launch_bounds__(kSeqThreads, 1)
+k_probe_seq(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  unsigned long long* skey = reinterpret_cast<unsigned long long*>(smem);
+  int* sq = reinterpret_cast<int*>(skey + kSeqSlots);  // key -> q of its latest miss in this SB
+  __shared__ int s_warp[32];
+  __shared__ int s_total;
+  __shared__ long long s_head, s_size;
+  __shared__ int s_base;
+  cg::cluster_group cluster = cg::this_cluster();
+  const unsigned CL = cluster.num_blocks();
+  const unsigned rank = cluster.block_rank();
+  const int tid = threadIdx.x;
+  if (c.state[5] == 1) return;  // the eviction-free parallel pass handled this superbatch
+  for (int s = tid; s < kSeqSlots; s += blockDim.x) skey[s] = kEmptyKey;
+  if (rank == 0 && tid == 0) {
+    s_head = c.state[0];
+    s_size = c.state[1];
+    s_base = 0;
+    c.state[4] = c.state[0];  // head0 for the insert pass
+  }
+  const long long limit = c.state[2];
+  const long long head0 = c.state[0];
+  const unsigned long long tmask = (unsigned long long)CL * kSeqSlots - 1ull;
+  cluster.sync();
+  for (int b = 0; b < S; ++b) {
+    const long long head = *cluster.map_shared_rank(&s_head, 0);
+    const long long size = *cluster.map_shared_rank(&s_size, 0);
+    const int cbase = *cluster.map_shared_rank(&s_base, 0);
+    const long long live_lo = head - size;
+    const int n = lv.n_u[b];
+    const size_t seg = (size_t)b * lv.cap;
+    const int chunk = (n + (int)CL - 1) / (int)CL;
+    const int cbeg = min(n, (int)rank * chunk), cend = min(n, cbeg + chunk);
+    const int ipt = (chunk + (int)blockDim.x - 1) / (int)blockDim.x;
+    const int tbeg = cbeg + tid * ipt;
+    int m_local = 0;
+    unsigned missmask = 0;
+    unsigned sbslot[kProbeIPT];
+#pragma unroll
+    for (int j = 0; j < kProbeIPT; ++j) {
+      sbslot[j] = 0xFFFFFFFFu;
+      const int i = tbeg + j;
+      if (j < ipt && i < cend) {
+        const unsigned long long key = tkey(lv.u_node[seg + i], lv.u_ts[seg + i]);
+        long long p = -1;
+        unsigned long long h = mix64(key) & tmask;
+        for (unsigned long long pr = 0; pr <= tmask; ++pr) {
+          const unsigned long long k0 = *(cluster.map_shared_rank(skey, (unsigned)(h / kSeqSlots)) + (h % kSeqSlots));
+          if (k0 == kEmptyKey) break;
+          if (k0 == key) {
+            sbslot[j] = (unsigned)h;
+            p = head0 + *(cluster.map_shared_rank(sq, (unsigned)(h / kSeqSlots)) + (h % kSeqSlots));
+            break;
+          }
+          h = (h + 1) & tmask;
+        }
+        if (sbslot[j] == 0xFFFFFFFFu) p = lv.p0[seg + i];
+        if (p >= 0 && p >= live_lo) {
+          lv.slot[seg + i] = p % c.rcap;  // hit (Alg. 1 l.8)
+        } else {
+          missmask |= 1u << j;
+          ++m_local;
+        }
+      }
+    }
+    int tot_cta;
+    const int excl = block_excl_scan(m_local, s_warp, tot_cta);
+    if (tid == 0) s_total = tot_cta;
+    cluster.sync();
+    int before = 0, m = 0;
+    for (unsigned r = 0; r < CL; ++r) {
+      const int v = *cluster.map_shared_rank(&s_total, r);
+      if (r < rank) before += v;
+      m += v;
+    }
+    int rr = before + excl;
+#pragma unroll
+    for (int j = 0; j < kProbeIPT; ++j) {
+      if (missmask & (1u << j)) {
+        const int i = tbeg + j;
+        const int q = cbase + rr;
+        const int32_t node = lv.u_node[seg + i];
+        const uint32_t t = lv.u_ts[seg + i];
+        lv.c_b[q] = b;
+        lv.c_u[q] = i;
+        lv.c_node[q] = node;
+        lv.c_ts[q] = t;
+        lv.sup[q] = 0;
+        lv.slot[seg + i] = (head + rr) % c.rcap;  // == (head0 + q) % rcap
+        const unsigned long long key = tkey(node, t);
+        if (sbslot[j] != 0xFFFFFFFFu) {  // evicted and missed again inside this SB
+          const unsigned h = sbslot[j];
+          int* qp = cluster.map_shared_rank(sq, h / kSeqSlots) + (h % kSeqSlots);
+          lv.sup[*qp] = 1;
+          *qp = q;
+        } else {
+          unsigned long long h = mix64(key) & tmask;
+          for (unsigned long long pr = 0; pr <= tmask; ++pr) {
+            unsigned long long* kp = cluster.map_shared_rank(skey, (unsigned)(h / kSeqSlots)) + (h % kSeqSlots);
+            const unsigned long long old = atomicCAS(kp, kEmptyKey, key);
+            if (old == kEmptyKey || old == key) {
+              *(cluster.map_shared_rank(sq, (unsigned)(h / kSeqSlots)) + (h % kSeqSlots)) = q;
+              break;
+            }
+            h = (h + 1) & tmask;
+          }
+        }
+        ++rr;
+      }
+    }
+    if (rank == 0 && tid == 0) {
+      const long long nsz = size + m < limit ? size + m : limit;
+      const long long ev_total = size + m - nsz;
+      const long long evicted = ev_total < size ? ev_total : size;
+      s_head = head + m;
+      s_size = nsz;
+      s_base = cbase + m;
+      lv.c_base[b] = cbase;
+      lv.n_c[b] = m;
+      const int L6 = layer * TG_CNT_PER_LAYER;
+      cnt_add(cnt, b, L6 + 2, n);      // lookups
+      cnt_add(cnt, b, L6 + 3, n - m);  // hits
+      cnt_add(cnt, b, L6 + 4, m);      // misses = embeddings computed
+      cnt_add(cnt, b, L6 + 5, evicted);
+    }
+    cluster.sync();
+  }
+  if (rank == 0 && tid == 0) {
+    *lv.n_c_total = s_base;
+    c.state[0] = s_head;
+    c.state[1] = s_size;
+  }
+  cluster.sync();
+}
+
+// Eviction-free superbatch (size0 + sum_b |U_b| <= limit): nothing live at
+// the start or inserted during the superbatch can leave the FIFO window, so
+// the sequential outcome is closed-form: the occurrence of a key in batch b
+// hits iff an earlier batch of the superbatch holds the same key, or the key
+// is live in the index at superbatch start. One cluster pass over the
+// concatenated unique lists (j = batch-major order, the order of Alg. 1's
+// lookups) finds first occurrences (DSMEM hash, min position), ranks the
+// misses with an ordered scan (their FIFO positions are head0 + q) and hands
+// every later occurrence the ring slot of its first one.
+__global__ void __launch_bounds__(kSeqThreads, 1)
+k_probe_par(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  unsigned long long* skey = reinterpret_cast<unsigned long long*>(smem);
+  unsigned* sval = reinterpret_cast<unsigned*>(skey + kSeqSlots);  // min j, later: ring slot
+  __shared__ int s_pre[kMaxS + 1];
+  __shared__ int s_warp[32];
+  __shared__ int s_total;
+  cg::cluster_group cluster = cg::this_cluster();
+  const unsigned CL = cluster.num_blocks();
+  const unsigned rank = cluster.block_rank();
+  const int tid = threadIdx.x;
+  const long long head0 = c.state[0], size0 = c.state[1], limit = c.state[2];
+  if (tid == 0) {
+    int a = 0;
+    for (int b = 0; b < S; ++b) {
+      s_pre[b] = a;
+      a += lv.n_u[b];
+    }
+    s_pre[S] = a;
+  }
+  __syncthreads();
+  const int NT = s_pre[S];
+  if (size0 + NT > limit) {  // eviction possible: the ordered pass handles this superbatch
+    if (rank == 0 && tid == 0) c.state[5] = 0;
+    return;                  // uniform over the cluster (same inputs everywhere)
+  }
+  for (int s = tid; s < kSeqSlots; s += blockDim.x) {
+    skey[s] = kEmptyKey;
+    sval[s] = 0xFFFFFFFFu;
+  }
+  const long long live_lo = head0 - size0;
+  const unsigned long long tmask = (unsigned long long)CL * kSeqSlots - 1ull;
+  cluster.sync();
+  const int chunk = (NT + (int)CL - 1) / (int)CL;
+  const int cbeg = min(NT, (int)rank * chunk), cend = min(NT, cbeg + chunk);
+  const int ipt = (chunk + (int)blockDim.x - 1) / (int)blockDim.x;
+  const int tbeg = cbeg + tid * ipt;
+  unsigned hs[kDedupIPT];
+  int jb[kDedupIPT];
+  // ---- first occurrences (min j per key)
+#pragma unroll
+  for (int j = 0; j < kDedupIPT; ++j) {
+    hs[j] = 0xFFFFFFFFu;
+    jb[j] = 0;
+    const int i = tbeg + j;
+    if (j < ipt && i < cend) {
+      int b = 0;
+      while (b + 1 < S && s_pre[b + 1] <= i) ++b;
+      jb[j] = b;
+      const size_t idx = (size_t)b * lv.cap + (i - s_pre[b]);
+      const unsigned long long key = tkey(lv.u_node[idx], lv.u_ts[idx]);
+      unsigned long long h = mix64(key) & tmask;
+      for (unsigned long long pr = 0; pr <= tmask; ++pr) {
+        unsigned long long* kp = cluster.map_shared_rank(skey, (unsigned)(h / kSeqSlots)) + (h % kSeqSlots);
+        const unsigned long long old = atomicCAS(kp, kEmptyKey, key);
+        if (old == kEmptyKey || old == key) {
+          atomicMin(cluster.map_shared_rank(sval, (unsigned)(h / kSeqSlots)) + (h % kSeqSlots), (unsigned)i);
+          hs[j] = (unsigned)h;
+          break;
+        }
+        h = (h + 1) & tmask;
+      }
+      if (hs[j] == 0xFFFFFFFFu) atomicOr(err, kErrDedupFull);
+    }
+  }
+  cluster.sync();
+  // ---- misses = first occurrences not live at superbatch start; ordered rank
+  unsigned firstmask = 0, missmask = 0;
+  int m_local = 0;
+#pragma unroll
+  for (int j = 0; j < kDedupIPT; ++j) {
+    const int i = tbeg + j;
+    if (j < ipt && i < cend && hs[j] != 0xFFFFFFFFu) {
+      const unsigned h = hs[j];
+      if (*(cluster.map_shared_rank(sval, h / kSeqSlots) + (h % kSeqSlots)) == (unsigned)i) {
+        firstmask |= 1u << j;
+        const size_t idx = (size_t)jb[j] * lv.cap + (i - s_pre[jb[j]]);
+        const long long p = lv.p0[idx];
+        if (!(p >= 0 && p >= live_lo)) {
+          missmask |= 1u << j;
+          ++m_local;
+        }
+      }
+    }
+  }
+  int tot_cta;
+  const int excl = block_excl_scan(m_local, s_warp, tot_cta);
+  if (tid == 0) s_total = tot_cta;
+  cluster.sync();  // first-decisions done everywhere (sval may be overwritten now)
+  int before = 0;
+  for (unsigned r = 0; r < rank; ++r) before += *cluster.map_shared_rank(&s_total, r);
+  int q = before + excl;
+#pragma unroll
+  for (int j = 0; j < kDedupIPT; ++j) {
+    if (firstmask & (1u << j)) {
+      const int i = tbeg + j;
+      const int b = jb[j];
+      const int u = i - s_pre[b];
+      const size_t idx = (size_t)b * lv.cap + u;
+      long long sl;
+      if (missmask & (1u << j)) {
+        lv.c_b[q] = b;
+        lv.c_u[q] = u;
+        lv.c_node[q] = lv.u_node[idx];
+        lv.c_ts[q] = lv.u_ts[idx];
+        lv.sup[q] = 0;
+        sl = (head0 + q) % c.rcap;
+        ++q;
+      } else {
+        sl = lv.p0[idx] % c.rcap;
+      }
+      lv.slot[idx] = sl;
+      const unsigned h = hs[j];
+      *(cluster.map_shared_rank(sval, h / kSeqSlots) + (h % kSeqSlots)) = (unsigned)sl;
+    }
+  }
+  cluster.sync();
+  // ---- later occurrences: the slot of the first one; per-batch bookkeeping
+#pragma unroll
+  for (int j = 0; j < kDedupIPT; ++j) {
+    const int i = tbeg + j;
+    if (j < ipt && i < cend && hs[j] != 0xFFFFFFFFu && !(firstmask & (1u << j))) {
+      const unsigned h = hs[j];
+      const size_t idx = (size_t)jb[j] * lv.cap + (i - s_pre[jb[j]]);
+      lv.slot[idx] = *(cluster.map_shared_rank(sval, h / kSeqSlots) + (h % kSeqSlots));
+    }
+  }
+  if (rank == CL - 1 && tid == 0) {
+    const int M = before + tot_cta;  // last CTA: total misses
+    *lv.n_c_total = M;
+    c.state[4] = head0;
+    c.state[0] = head0 + M;
+    c.state[1] = size0 + M;
+    c.state[5] = 1;
+  }
+  cluster.sync();  // remote smem reads done; n_c per batch needs every miss counted
+  if (rank == 0 && tid < S) {
+    // misses of batch b = misses with j in [pre[b], pre[b+1]); recount from the compute list
+    const int b = tid;
+    const int M = *lv.n_c_total;
+    int lo = 0, hi = M;  // first q with c_b[q] >= b
+    while (lo < hi) {
+      const int mid = (lo + hi) >> 1;
+      if (lv.c_b[mid] < b) lo = mid + 1; else hi = mid;
+    }
+    int lo2 = lo, hi2 = M;  // first q with c_b[q] > b
+    while (lo2 < hi2) {
+      const int mid = (lo2 + hi2) >> 1;
+      if (lv.c_b[mid] <= b) lo2 = mid + 1; else hi2 = mid;
+    }
+    const int n = s_pre[b + 1] - s_pre[b], m = lo2 - lo;
+    lv.c_base[b] = lo;
+    lv.n_c[b] = m;
+    const int L6 = layer * TG_CNT_PER_LAYER;
+    cnt_add(cnt, b, L6 + 2, n);      // lookups
+    cnt_add(cnt, b, L6 + 3, n - m);  // hits
+    cnt_add(cnt, b, L6 + 4, m);      // misses
+  }
+}
+
+__global__ void k_probe_ins(LevelDev lv, CacheDev c, int* err) {
+  const int n = *lv.n_c_total;
+  const long long head0 = c.state[4];
+  const long long live_lo = c.state[0] - c.state[1];
+  for (int q = blockIdx.x * blockDim.x + threadIdx.x; q < n; q += gridDim.x * blockDim.x) {
+    if (lv.sup[q]) continue;
+    const unsigned long long key = tkey(lv.c_node[q], lv.c_ts[q]);
+    const long long pos = head0 + q;
+    unsigned long long h = mix64(key) & c.imask;
+    bool done = false;
+    for (unsigned long long pr = 0; pr <= 4 * c.imask && !done; ++pr) {
+      const unsigned long long k0 = ld_volatile_u64(c.ikey + h);
+      if (k0 != kLockedKey) {
+        __threadfence();
+        const bool reusable = (k0 == kEmptyKey) || (k0 == key) || (*(volatile long long*)(c.ipos + h) < live_lo);
+        if (reusable) {
+          if (atomicCAS(c.ikey + h, k0, kLockedKey) == k0) {
+            *(volatile long long*)(c.ipos + h) = pos;
+            __threadfence();
+            atomicExch(c.ikey + h, key);
+            if (k0 == kEmptyKey) atomicAdd((unsigned long long*)(c.state + 3), 1ull);
+            done = true;
+          }
+          continue;
+        }
+      }
+      h = (h + 1) & c.imask;
+    }
+    if (!done) atomicOr(err, kErrIndexFull);
+  }
+}
+
 void launch_probe(LevelDev lv, int S, const CacheDev* cache, long long* cnt, int layer, int* err,
                   cudaStream_t st) {
   CacheDev c{};
@@ -406,7 +782,46 @@ void launch_probe(LevelDev lv, int S, const CacheDev* cache, long long* cnt, int
     has_ring = 1;
     use_cache = c.ikey != nullptr;
   }
-  k_probe<<<1, 1024, 0, st>>>(lv, S, c, use_cache, has_ring, cnt, layer, err);
+  if (!use_cache) {  // top layer (no lookup, R9) or cache disabled: ordered compaction only
+    k_probe<<<1, 1024, 0, st>>>(lv, S, c, 0, has_ring, cnt, layer, err);
+    return;
+  }
+  int blocks = (S * lv.cap + 255) / 256;
+  if (blocks > 148 * 8) blocks = 148 * 8;
+  k_probe_pre<<<blocks, 256, 0, st>>>(lv, S, c);
+  const size_t smem = (size_t)kSeqSlots * (sizeof(unsigned long long) + sizeof(int));
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(k_probe_seq, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(k_probe_seq, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+    attr = true;
+  }
+  // cluster large enough for every key of the superbatch to be an in-SB miss (load <= 0.6)
+  int cl = 1;
+  while (cl < kSeqCL && (long long)cl * kSeqSlots * 6 / 10 < (long long)S * lv.cap) cl <<= 1;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(cl);
+  cfg.blockDim = dim3(kSeqThreads);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = cl;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  static bool attr2 = false;
+  if (!attr2) {
+    cudaFuncSetAttribute(k_probe_par, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(k_probe_par, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+    attr2 = true;
+  }
+  cudaLaunchKernelEx(&cfg, k_probe_par, lv, S, c, cnt, layer, err);
+  cudaLaunchKernelEx(&cfg, k_probe_seq, lv, S, c, cnt, layer, err);
+  int ib = (S * lv.cap + 255) / 256;
+  if (ib > 148 * 4) ib = 148 * 4;
+  k_probe_ins<<<ib, 256, 0, st>>>(lv, c, err);
 }
 
 // ------------------------------------------------------------------ NghLookup

@@ -327,7 +327,7 @@ tg_status run_superbatch(tg_ctx* ctx, int S, bool edge_mode, const EdgeSrc& es, 
         Prof pf(ctx, TG_ST_LOOKUP, st);
         launch_probe(ctx->lv[l - 1], S, &cd, cnt, l - 1, ctx->err, st);
       }
-      TRY(launched(ctx));
+      TRY(launched(ctx, cache_on ? 3 : 1));
     }
   }
   // ---- row addresses for every layer
@@ -674,6 +674,8 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     TRY(dalloc(ctx, &v.n_u, kMaxS));
     TRY(dalloc(ctx, &v.inv, n));
     TRY(dalloc(ctx, &v.slot, n));
+    TRY(dalloc(ctx, &v.p0, n));
+    TRY(dalloc(ctx, &v.sup, n));
     TRY(dalloc(ctx, &v.c_b, n));
     TRY(dalloc(ctx, &v.c_u, n));
     TRY(dalloc(ctx, &v.c_node, n));
@@ -694,7 +696,7 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
   // ---- caches for layers 1..L-1: index (load <= 1/4 of live items) + FIFO ring.
   // Ring capacity limit + (S+2) cap: a superbatch never overwrites a slot that
   // one of its own batches still reads.
-  TRY(dalloc(ctx, &ctx->cache_state, 4 * TG_MAX_LAYERS));
+  TRY(dalloc(ctx, &ctx->cache_state, 8 * TG_MAX_LAYERS));
   ctx->limit0 = cfg->cache_limit;
   for (int l = 1; l < L; ++l) {
     CacheDev& cd = ctx->cache[l];
@@ -706,7 +708,7 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     TRY(dalloc(ctx, &cd.ring, (size_t)rcap * dnp));
     cd.imask = icap - 1;
     cd.rcap = rcap;
-    cd.state = ctx->cache_state + 4 * l;
+    cd.state = ctx->cache_state + 8 * l;
   }
   // ---- compute workspace
   TRY(dalloc(ctx, &ctx->u, (size_t)maxC * HDp));
@@ -734,7 +736,7 @@ tg_status tg_cache_reset(tg_ctx* ctx, int64_t new_limit) {
   for (int l = 1; l < ctx->L; ++l) {
     CacheDev& cd = ctx->cache[l];
     CK(cudaMemset(cd.ikey, 0xFF, (cd.imask + 1) * sizeof(unsigned long long)));
-    long long st[4] = {0, 0, ctx->cfg.cache_limit, 0};
+    long long st[8] = {0, 0, ctx->cfg.cache_limit, 0, 0, 0, 0, 0};
     CK(cudaMemcpy(cd.state, st, sizeof(st), cudaMemcpyHostToDevice));
   }
   CK(cudaMemset(ctx->cnt_total, 0, TG_NCOUNTERS * sizeof(long long)));

@@ -68,7 +68,7 @@ struct CacheDev {
   unsigned long long imask;
   float* ring;               // [rcap x ldn]
   long long rcap;
-  long long* state;          // device [4]: head, size, limit, occupied index slots
+  long long* state;          // device [8]: head, size, limit, occupied index slots, head at SB start
 };
 
 // One recursion level l >= 1 of a superbatch.
@@ -83,6 +83,7 @@ struct LevelDev {
   int* n_u;                  // [S]
   int32_t* inv;
   long long* slot;
+  long long* p0;             // index position of each U entry at superbatch start (-1: absent)
   // compute list C_l, compacted over the superbatch (q = 0..n_c_total-1)
   int32_t* c_b;              // batch of q
   int32_t* c_u;              // unique-list index of q inside its batch
@@ -92,6 +93,7 @@ struct LevelDev {
   int* n_c;                  // [S]
   int* n_c_total;            // [1]
   int c_cap;                 // S * cap
+  unsigned char* sup;        // [S*cap] miss q superseded by a later re-miss of its key in the SB
   // sampled neighbours of each q (compute-centric [q*k + m])
   int32_t* nb_node;
   uint32_t* nb_ts;
