@@ -143,63 +143,62 @@ void launch_layernorm(const float* y, float* r, int Dp, int dn, int dnp, int de,
 }
 
 // -------------------------------------------------------------------- score
-// p_e = sigmoid(W_a2 ReLU(W_a1 [h_src || h_dst] + b_a1) + b_a2) (R10); the
-// targets' rows are reached through the batch's inverse index (DedupInvert).
-__global__ void k_score(const float* __restrict__ HL, int ldh, LevelDev top, int S, EdgeSrc es,
-                        const float* __restrict__ Wa1, const float* __restrict__ ba1, const float* __restrict__ Wa2,
-                        float ba2, int dn, int dnp, float* __restrict__ scores) {
-  extern __shared__ float x[];  // [2 dnp]
-  __shared__ float red[32];
-  for (int w = blockIdx.x; w < S * es.B; w += gridDim.x) {
+// p_e = sigmoid(W_a2 ReLU(W_a1 [h_src || h_dst] + b_a1) + b_a2) (R10) as
+// (1) row resolution through each batch's inverse index (DedupInvert),
+// (2) the hidden layer as a projection GEMM over the S*B edges, (3) a warp
+// per edge for the W_a2 dot product and the sigmoid.
+__global__ void k_score_rows(const float* __restrict__ HL, int ldh, LevelDev top, int S, EdgeSrc es,
+                             const float** __restrict__ rs, const float** __restrict__ rd,
+                             long long* __restrict__ oidx, int* __restrict__ m_dev) {
+  const int tot = S * es.B;
+  if (blockIdx.x == 0 && threadIdx.x == 0) *m_dev = tot;
+  for (int w = blockIdx.x * blockDim.x + threadIdx.x; w < tot; w += gridDim.x * blockDim.x) {
     const int b = w / es.B, e = w - b * es.B;
     const int64_t lo = es.e0 + (int64_t)b * es.B;
     const int64_t rem = es.n_edges - lo;
     const int Bb = (int)(rem < es.B ? (rem < 0 ? 0 : rem) : es.B);
-    if (e >= Bb) continue;  // uniform per block
-    const size_t seg = (size_t)b * top.cap;
-    const int qs = top.c_base[b] + top.inv[seg + e];
-    const int qd = top.c_base[b] + top.inv[seg + Bb + e];
-    const float* hs = HL + (size_t)qs * ldh;
-    const float* hd = HL + (size_t)qd * ldh;
-    for (int c = threadIdx.x; c < dnp; c += blockDim.x) {
-      x[c] = hs[c];
-      x[dnp + c] = hd[c];
+    if (e < Bb) {
+      const size_t seg = (size_t)b * top.cap;
+      rs[w] = HL + (size_t)(top.c_base[b] + top.inv[seg + e]) * ldh;
+      rd[w] = HL + (size_t)(top.c_base[b] + top.inv[seg + Bb + e]) * ldh;
+      oidx[w] = lo + e;
+    } else {  // past the stream end: any valid row, result discarded
+      rs[w] = HL;
+      rd[w] = HL;
+      oidx[w] = -1;
     }
-    __syncthreads();
-    float part = 0.f;
-    for (int j = threadIdx.x; j < dn; j += blockDim.x) {
-      const float4* wr = reinterpret_cast<const float4*>(Wa1 + (size_t)j * 2 * dnp);
-      const float4* xv = reinterpret_cast<const float4*>(x);
-      float z = 0.f;
-      for (int q = 0; q < (2 * dnp) / 4; ++q) {
-        const float4 a = wr[q], bb = xv[q];
-        z = fmaf(a.x, bb.x, z);
-        z = fmaf(a.y, bb.y, z);
-        z = fmaf(a.z, bb.z, z);
-        z = fmaf(a.w, bb.w, z);
-      }
-      z = fmaxf(z + ba1[j], 0.f);
-      part = fmaf(Wa2[j], z, part);
-    }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
-    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = part;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      float s = 0.f;
-      for (int ww = 0; ww < (int)(blockDim.x >> 5); ++ww) s += red[ww];
-      scores[lo + e] = 1.f / (1.f + expf(-(s + ba2)));
-    }
-    __syncthreads();
   }
 }
 
-void launch_score(const float* HL, int ldh, LevelDev top, int S, EdgeSrc es, const float* Wa1, const float* ba1,
-                  const float* Wa2, float ba2, int dn, int dnp, float* scores, cudaStream_t st) {
-  int blocks = S * es.B;
-  if (blocks > 1184) blocks = 1184;
+void launch_score_rows(const float* HL, int ldh, LevelDev top, int S, EdgeSrc es, const float** rs,
+                       const float** rd, long long* oidx, int* m_dev, cudaStream_t st) {
+  int blocks = (S * es.B + 255) / 256;
   if (blocks < 1) blocks = 1;
-  k_score<<<blocks, 128, 2 * dnp * sizeof(float), st>>>(HL, ldh, top, S, es, Wa1, ba1, Wa2, ba2, dn, dnp, scores);
+  k_score_rows<<<blocks, 256, 0, st>>>(HL, ldh, top, S, es, rs, rd, oidx, m_dev);
+}
+
+__global__ void k_score_head(const float* __restrict__ z, int ldz, const long long* __restrict__ oidx, int M,
+                             const float* __restrict__ Wa2, float ba2, int dn, float* __restrict__ scores) {
+  const int lane = threadIdx.x & 31;
+  const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, nw = (gridDim.x * blockDim.x) >> 5;
+  for (int w = warp; w < M; w += nw) {
+    const long long o = oidx[w];
+    if (o < 0) continue;
+    const float* zr = z + (size_t)w * ldz;
+    float s = 0.f;
+    for (int j = lane; j < dn; j += 32) s = fmaf(Wa2[j], zr[j], s);
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
+    if (lane == 0) scores[o] = 1.f / (1.f + expf(-(s + ba2)));
+  }
+}
+
+void launch_score_head(const float* z, int ldz, const long long* oidx, int M, const float* Wa2, float ba2, int dn,
+                       float* scores, cudaStream_t st) {
+  int blocks = (M * 32 + 255) / 256;
+  if (blocks < 1) blocks = 1;
+  if (blocks > 1184) blocks = 1184;
+  k_score_head<<<blocks, 256, 0, st>>>(z, ldz, oidx, M, Wa2, ba2, dn, scores);
 }
 
 __global__ void k_invert(const float* __restrict__ HL, int ldh, LevelDev top, int n, int dn,

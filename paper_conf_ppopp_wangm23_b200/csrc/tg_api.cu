@@ -42,6 +42,13 @@ struct tg_ctx {
   float *omega = nullptr, *phi = nullptr, *table = nullptr;
   float *Wa1 = nullptr, *ba1 = nullptr, *Wa2 = nullptr;
   float ba2 = 0.f;
+  TcWeights tcWa1;
+  // score workspace (S * B edges)
+  const float** sc_rs = nullptr;
+  const float** sc_rd = nullptr;
+  long long* sc_oidx = nullptr;
+  float* sc_z = nullptr;
+  int* sc_m = nullptr;
   // recursion levels (index l = 1..L), caches for l = 1..L-1
   LevelDev lv[TG_MAX_LAYERS + 1]{};
   int cap[TG_MAX_LAYERS + 1]{};
@@ -367,10 +374,26 @@ tg_status stream_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, cons
     TRY(run_superbatch(ctx, S, true, es, 2 * batch, st));
     {
       Prof pf(ctx, TG_ST_SCORE, st);
-      launch_score(ctx->HL, ctx->dnp, ctx->lv[ctx->L], S, es, ctx->Wa1, ctx->ba1, ctx->Wa2, ctx->ba2, ctx->d_n,
-                   ctx->dnp, scores, st);
+      launch_score_rows(ctx->HL, ctx->dnp, ctx->lv[ctx->L], S, es, ctx->sc_rs, ctx->sc_rd, ctx->sc_oidx, ctx->sc_m,
+                        st);
+      GemmArgs g{};  // hidden layer of the affinity MLP: ReLU(W_a1 [h_src || h_dst] + b_a1)
+      g.a_rows0 = ctx->sc_rs;
+      g.K0 = ctx->dnp;
+      g.a_rows1 = ctx->sc_rd;
+      g.K = 2 * ctx->dnp;
+      g.B = ctx->Wa1;
+      g.N = ctx->dnp;
+      g.bias = ctx->ba1;
+      g.relu = 1;
+      g.C = ctx->sc_z;
+      g.ldc = ctx->dnp;
+      g.m_dev = ctx->sc_m;
+      g.m_max = S * batch;
+      if (ctx->cfg.precision != TG_PREC_FP32) launch_gemm_tc(g, ctx->tcWa1, ctx->cfg.precision, st);
+      else launch_gemm_simt(g, st);
+      launch_score_head(ctx->sc_z, ctx->dnp, ctx->sc_oidx, S * batch, ctx->Wa2, ctx->ba2, ctx->d_n, scores, st);
     }
-    TRY(launched(ctx));
+    TRY(launched(ctx, 3));
     TRY(finish(ctx, S, log, b0, st));
   }
   return TG_OK;
@@ -503,7 +526,7 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
   const int L = cfg->n_layers, H = cfg->n_heads, k = cfg->n_neighbors, d_t = cfg->d_t;
   const int d_n = ctx->g.d_n, d_e = ctx->g.d_e;
   const int D = d_n + d_e + d_t;
-  if (L < 1 || L > TG_MAX_LAYERS || H < 1 || k < 1 || k > kMaxK || d_t < 1 || D % H) return TG_EINVAL;
+  if (L < 1 || L > TG_MAX_LAYERS || H < 1 || H > 8 || k < 1 || k > kMaxK || d_t < 1 || D % H) return TG_EINVAL;
   if (cfg->max_batch_targets < 1 || cfg->cache_limit < 0 || cfg->time_window < 0) return TG_EINVAL;
   if (cfg->precision < TG_PREC_FP32 || cfg->precision > TG_PREC_BF16) return TG_EINVAL;
   if (cfg->superbatch < 0 || cfg->superbatch > kMaxS) return TG_EINVAL;
@@ -656,6 +679,14 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     CK(cudaMemcpy(ctx->ba1, b.data(), b.size() * 4, cudaMemcpyHostToDevice));
     CK(cudaMemcpy(ctx->Wa2, w2.data(), w2.size() * 4, cudaMemcpyHostToDevice));
     ctx->ba2 = ba2[0];
+    if (cfg->precision != TG_PREC_FP32)
+      TRY(tc_prepare_weights(ctx->Wa1, dnp, 2 * dnp, cfg->precision, &ctx->tcWa1, ctx->owned));
+    const size_t ne = (size_t)S * ((cfg->max_batch_targets + 1) / 2);
+    TRY(dalloc(ctx, &ctx->sc_rs, ne));
+    TRY(dalloc(ctx, &ctx->sc_rd, ne));
+    TRY(dalloc(ctx, &ctx->sc_oidx, ne));
+    TRY(dalloc(ctx, &ctx->sc_z, ne * dnp));
+    TRY(dalloc(ctx, &ctx->sc_m, 1));
   }
   // ---- recursion levels: batch-segmented lists + superbatch compute lists
   int maxC = 0;

@@ -203,9 +203,12 @@ void launch_gemm_simt(const GemmArgs& g, cudaStream_t st);
 void launch_layernorm(const float* y, float* r, int Dp, int dn, int dnp, int de, int dep, int dt,
                       const float* gamma, const float* beta, const int* m_dev, int m_max, cudaStream_t st);
 
-// Scores p_e = sigmoid(MLP(h_src, h_dst)) (R10) for every edge of the superbatch.
-void launch_score(const float* HL, int ldh, LevelDev top, int S, EdgeSrc es, const float* Wa1, const float* ba1,
-                  const float* Wa2, float ba2, int dn, int dnp, float* scores, cudaStream_t st);
+// Scores p_e = sigmoid(MLP(h_src, h_dst)) (R10) for every edge of the superbatch:
+// row resolution, hidden layer as a projection GEMM, then the W_a2 head.
+void launch_score_rows(const float* HL, int ldh, LevelDev top, int S, EdgeSrc es, const float** rs,
+                       const float** rd, long long* oidx, int* m_dev, cudaStream_t st);
+void launch_score_head(const float* z, int ldz, const long long* oidx, int M, const float* Wa2, float ba2, int dn,
+                       float* scores, cudaStream_t st);
 // out[i] = H_L[q(i)] for a single-batch embed call (DedupInvert, Alg. 1 l.20).
 void launch_invert(const float* HL, int ldh, LevelDev top, int n, int dn, float* out, cudaStream_t st);
 void launch_prep_nodes(const int32_t* nodes, const uint32_t* ts, int n, LevelDev top, cudaStream_t st);
