@@ -1,13 +1,18 @@
 // tcgen05 tensor-core GEMM for the dense per-target projections (sm_100a):
 //   C[M x N] = epilogue(A[M x K] . B[N x K]^T)
-// A rows are gathered through row pointers (or dense), converted on the fly
-// and written into shared memory in the canonical K-major 128B-swizzled UMMA
-// layout; B (the weights) is pre-tiled at model load into the same layout, one
-// contiguous image per (N tile, K block), and fetched with TMA bulk copies
-// (cp.async.bulk, mbarrier complete_tx). One elected thread issues
-// tcgen05.mma (M = 128, N = BN <= 256) with the accumulator in TMEM; the
-// epilogue reads it back with tcgen05.ld (32x32b) and fuses bias, the
-// attention residual q, ReLU and the (gathered) store.
+//
+// Persistent, warp-specialized, mbarrier-pipelined:
+//   warps 0-3  A producers: thread t owns row m0+t of the tile; gathers the
+//              row through its row pointer(s) (or dense), converts it (tf32
+//              hi/lo split or bf16) and writes it into shared memory in the
+//              canonical K-major 128B-swizzled UMMA layout;
+//   warp 4     B producer: one lane issues TMA bulk copies (cp.async.bulk,
+//              mbarrier complete_tx) of the pre-tiled weight images;
+//   warp 5     MMA issuer: one lane issues tcgen05.mma (M = 128, N = BN) into a
+//              double-buffered TMEM accumulator and commits to mbarriers;
+//   warps 6-9  epilogue: tcgen05.ld (32x32b) -> bias / attention residual q /
+//              ReLU -> row store (dense or gathered destinations).
+// STAGES shared-memory stages (3-4) decouple the producers from the tensor core.
 //
 // TG_PREC_TF32X3: kind::tf32 with the 3-term split a.b ~ ah.bh + ah.bl + al.bh
 // (ah = rna_tf32(a), al = rna_tf32(a - ah)): fp32-level accuracy on tensor
@@ -22,8 +27,10 @@
 namespace tg {
 
 constexpr int TC_BM = 128;
-constexpr int TC_THREADS = 128;
-constexpr int TC_STAGES = 2;
+constexpr int TC_WARPS = 10;
+constexpr int TC_THREADS = TC_WARPS * 32;
+constexpr int TC_MAXSTAGES = 4;
+constexpr int TC_ACC_COLS = 256;  // per accumulator buffer (x2 = all 512 TMEM columns)
 
 __host__ __device__ inline int tc_epc(int prec) { return prec == TG_PREC_BF16 ? 64 : 32; }  // elems / 128B
 __host__ __device__ inline int tc_planes(int prec) { return prec == TG_PREC_TF32X3 ? 2 : 1; }
@@ -31,6 +38,13 @@ __host__ __device__ inline int tc_planes(int prec) { return prec == TG_PREC_TF32
 // offset of 16-byte chunk c of row r inside a 128B-swizzled K-major tile
 __host__ __device__ inline unsigned sw128(int r, int c) {
   return (unsigned)((r >> 3) * 1024 + (r & 7) * 128 + ((c ^ (r & 7)) << 4));
+}
+
+static inline int tc_stages(int prec, int BN) {
+  const size_t st = (size_t)tc_planes(prec) * ((size_t)TC_BM * 128 + (size_t)BN * 128);
+  int s = (int)((200 * 1024) / st);
+  if (s > TC_MAXSTAGES) s = TC_MAXSTAGES;
+  return s < 2 ? 2 : s;
 }
 
 // ------------------------------------------------------------ host: weights
@@ -58,7 +72,8 @@ static inline uint16_t bf16_rn(float x) {
 
 tg_status tc_prepare_weights(const float* W, int N, int K, int precision, TcWeights* out,
                              std::vector<void*>& owned) {
-  const int ntn = (N + 255) / 256;
+  // N tiles of <= 128 columns (more CTAs at the small M of a superbatch)
+  const int ntn = (N + 127) / 128;
   int BN = (N + ntn - 1) / ntn;
   BN = (BN + 15) & ~15;
   const int epc = tc_epc(precision);
@@ -130,18 +145,18 @@ __device__ __forceinline__ uint64_t umma_desc(uint32_t saddr) {
 
 __device__ __forceinline__ uint32_t umma_idesc(int prec, int N) {
   uint32_t d = 0;
-  d |= 1u << 4;                                   // D = f32
+  d |= 1u << 4;                                         // D = f32
   const uint32_t fmt = prec == TG_PREC_BF16 ? 1u : 2u;  // bf16 : tf32
-  d |= fmt << 7;                                  // A format
-  d |= fmt << 10;                                 // B format
-  d |= (uint32_t)(N >> 3) << 17;                  // N / 8
-  d |= (uint32_t)(TC_BM >> 4) << 24;              // M / 16
+  d |= fmt << 7;                                        // A format
+  d |= fmt << 10;                                       // B format
+  d |= (uint32_t)(N >> 3) << 17;                        // N / 8
+  d |= (uint32_t)(TC_BM >> 4) << 24;                    // M / 16
   return d;
 }
 
-__device__ __forceinline__ void mma_issue(int prec, uint32_t tmem, uint64_t da, uint64_t db, uint32_t idesc,
-                                          uint32_t acc) {
-  if (prec == TG_PREC_BF16) {
+template <int PREC>
+__device__ __forceinline__ void mma_issue(uint32_t tmem, uint64_t da, uint64_t db, uint32_t idesc, uint32_t acc) {
+  if (PREC == TG_PREC_BF16) {
     asm volatile(
         "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
         "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}\n" ::"r"(tmem),
@@ -160,6 +175,9 @@ __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
 __device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(smem_u32(bar)), "r"(bytes)
                : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(smem_u32(bar)) : "memory");
 }
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   const uint32_t a = smem_u32(bar);
@@ -186,21 +204,14 @@ __device__ __forceinline__ float rna_tf32(float x) {
   return __uint_as_float(r);
 }
 
-// A chunk c (16 B of smem) of row `row`, k-block kb: 4 floats (tf32) or 8 floats (bf16).
-__device__ __forceinline__ float4 tc_load4(const GemmArgs& g, int row, int M, int col) {
-  if (row >= M || col >= g.K) return make_float4(0.f, 0.f, 0.f, 0.f);
-  const float* p;
-  if (col < g.K0) {
-    p = g.a_rows0 ? g.a_rows0[row] + col : g.a_base0 + (size_t)row * g.lda0 + col;
-  } else {
-    const int cc = col - g.K0;
-    p = g.a_rows1 ? g.a_rows1[row] + cc : g.a_base1 + (size_t)row * g.lda1 + cc;
-  }
+__device__ __forceinline__ float4 tc_load4(const GemmArgs& g, const float* r0, const float* r1, int col) {
+  if (col >= g.K) return make_float4(0.f, 0.f, 0.f, 0.f);
+  const float* p = col < g.K0 ? r0 + col : r1 + (col - g.K0);
   return *reinterpret_cast<const float4*>(p);
 }
 
 template <int PREC>
-__global__ void __launch_bounds__(TC_THREADS, 1) k_gemm_tc(GemmArgs g, TcWeights w) {
+__global__ void __launch_bounds__(TC_THREADS, 1) k_gemm_tc(GemmArgs g, TcWeights w, int stages) {
   constexpr int EPC = PREC == TG_PREC_BF16 ? 64 : 32;
   constexpr int PLANES = PREC == TG_PREC_TF32X3 ? 2 : 1;
   constexpr int NV = EPC / 4;  // float4 loads per row per k-block
@@ -210,163 +221,219 @@ __global__ void __launch_bounds__(TC_THREADS, 1) k_gemm_tc(GemmArgs g, TcWeights
   const uint32_t a_plane = TC_BM * 128;
   const uint32_t b_plane = (uint32_t)BN * 128;
   const uint32_t stage_bytes = PLANES * (a_plane + b_plane);
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + TC_STAGES * stage_bytes);
-  uint64_t* done = full + TC_STAGES;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(done + TC_STAGES);
-  const int tid = threadIdx.x, warp = tid >> 5;
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + stages * stage_bytes);
+  uint64_t* empty = full + TC_MAXSTAGES;
+  uint64_t* tfull = empty + TC_MAXSTAGES;   // [2]
+  uint64_t* tempty = tfull + 2;             // [2]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int M = *g.m_dev;
   const int tiles_m = (M + TC_BM - 1) / TC_BM;
   const int ntiles = tiles_m * w.ntn;
   if ((int)blockIdx.x >= ntiles) return;
+  const int nkb = w.nkb;
   if (tid == 0) {
-    for (int s = 0; s < TC_STAGES; ++s) {
-      mbar_init(&full[s], 1);
-      mbar_init(&done[s], 1);
+    for (int s = 0; s < stages; ++s) {
+      mbar_init(&full[s], TC_BM + 1);  // 128 A rows + the B producer's expect_tx
+      mbar_init(&empty[s], 1);         // MMA commit
+    }
+    for (int a = 0; a < 2; ++a) {
+      mbar_init(&tfull[a], 1);     // MMA commit after the tile's last k-block
+      mbar_init(&tempty[a], 128);  // epilogue threads drained the accumulator
     }
     asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
   }
   if (warp == 0) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;\n" ::"r"(smem_u32(tmem_slot)),
-                 "r"(256));
+                 "r"(2 * TC_ACC_COLS));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;\n");
   }
   asm volatile("tcgen05.fence::before_thread_sync;\n");
   __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;\n");
   const uint32_t tmem = *tmem_slot;
-  const uint32_t idesc = umma_idesc(PREC, BN);
-  const int nkb = w.nkb;
-  uint32_t gk = 0;  // k-blocks issued by this CTA (stage / phase bookkeeping)
-  for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
-    const int tm = t / w.ntn, tn = t - tm * w.ntn;
-    const int m0 = tm * TC_BM, n0 = tn * BN;
-    const int row = m0 + tid;  // this thread loads A row `row`
-    float4 regs[NV];
-#pragma unroll
-    for (int v = 0; v < NV; ++v) regs[v] = tc_load4(g, row, M, v * 4);
-    for (int kb = 0; kb < nkb; ++kb, ++gk) {
-      const int s = gk & 1;
-      unsigned char* sA = smem + s * stage_bytes;
-      unsigned char* sB = sA + PLANES * a_plane;
-      if (gk >= TC_STAGES) mbar_wait(&done[s], ((gk - TC_STAGES) >> 1) & 1);  // MMAs of gk-2 retired
-      if (tid == 0) {
-        const unsigned char* src = reinterpret_cast<const unsigned char*>(w.hi) +
-                                   ((size_t)tn * nkb + kb) * PLANES * b_plane;
-        mbar_expect_tx(&full[s], PLANES * b_plane);
-        bulk_g2s(sB, src, PLANES * b_plane, &full[s]);  // TMA: weight tile image(s)
+
+  if (warp < 4) {
+    // ===================== A producers
+    uint32_t gk = 0;
+    for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+      const int tm = t / w.ntn;
+      const int row = tm * TC_BM + tid;
+      const bool rv = row < M;
+      const float* r0 = nullptr;
+      const float* r1 = nullptr;
+      if (rv) {
+        r0 = g.a_rows0 ? g.a_rows0[row] : g.a_base0 + (size_t)row * g.lda0;
+        if (g.K0 < g.K) r1 = g.a_rows1 ? g.a_rows1[row] : g.a_base1 + (size_t)row * g.lda1;
       }
-      // A: registers (this k-block) -> swizzled smem, split into planes
-      const int r = tid;
-      if (PREC == TG_PREC_BF16) {
+      float4 regs[NV];
 #pragma unroll
-        for (int c = 0; c < 8; ++c) {
-          const float4 x0 = regs[2 * c], x1 = regs[2 * c + 1];
-          __nv_bfloat162 p0 = __floats2bfloat162_rn(x0.x, x0.y), p1 = __floats2bfloat162_rn(x0.z, x0.w);
-          __nv_bfloat162 p2 = __floats2bfloat162_rn(x1.x, x1.y), p3 = __floats2bfloat162_rn(x1.z, x1.w);
-          uint4 u;
-          u.x = *reinterpret_cast<uint32_t*>(&p0);
-          u.y = *reinterpret_cast<uint32_t*>(&p1);
-          u.z = *reinterpret_cast<uint32_t*>(&p2);
-          u.w = *reinterpret_cast<uint32_t*>(&p3);
-          *reinterpret_cast<uint4*>(sA + sw128(r, c)) = u;
-        }
-      } else {
+      for (int v = 0; v < NV; ++v) regs[v] = rv ? tc_load4(g, r0, r1, v * 4) : make_float4(0.f, 0.f, 0.f, 0.f);
+      for (int kb = 0; kb < nkb; ++kb, ++gk) {
+        const int s = gk % stages;
+        mbar_wait(&empty[s], ((gk / stages) & 1) ^ 1);
+        unsigned char* sA = smem + s * stage_bytes;
+        if (PREC == TG_PREC_BF16) {
 #pragma unroll
-        for (int c = 0; c < 8; ++c) {
-          const float4 x = regs[c];
-          float4 hi, lo;
-          hi.x = rna_tf32(x.x);
-          hi.y = rna_tf32(x.y);
-          hi.z = rna_tf32(x.z);
-          hi.w = rna_tf32(x.w);
-          *reinterpret_cast<float4*>(sA + sw128(r, c)) = hi;
-          if (PLANES == 2) {
-            lo.x = rna_tf32(x.x - hi.x);
-            lo.y = rna_tf32(x.y - hi.y);
-            lo.z = rna_tf32(x.z - hi.z);
-            lo.w = rna_tf32(x.w - hi.w);
-            *reinterpret_cast<float4*>(sA + a_plane + sw128(r, c)) = lo;
+          for (int c = 0; c < 8; ++c) {
+            const float4 x0 = regs[2 * c], x1 = regs[2 * c + 1];
+            __nv_bfloat162 p0 = __floats2bfloat162_rn(x0.x, x0.y), p1 = __floats2bfloat162_rn(x0.z, x0.w);
+            __nv_bfloat162 p2 = __floats2bfloat162_rn(x1.x, x1.y), p3 = __floats2bfloat162_rn(x1.z, x1.w);
+            uint4 u;
+            u.x = *reinterpret_cast<uint32_t*>(&p0);
+            u.y = *reinterpret_cast<uint32_t*>(&p1);
+            u.z = *reinterpret_cast<uint32_t*>(&p2);
+            u.w = *reinterpret_cast<uint32_t*>(&p3);
+            *reinterpret_cast<uint4*>(sA + sw128(tid, c)) = u;
+          }
+        } else {
+#pragma unroll
+          for (int c = 0; c < 8; ++c) {
+            const float4 x = regs[c];
+            float4 hi, lo;
+            hi.x = rna_tf32(x.x);
+            hi.y = rna_tf32(x.y);
+            hi.z = rna_tf32(x.z);
+            hi.w = rna_tf32(x.w);
+            *reinterpret_cast<float4*>(sA + sw128(tid, c)) = hi;
+            if (PLANES == 2) {
+              lo.x = rna_tf32(x.x - hi.x);
+              lo.y = rna_tf32(x.y - hi.y);
+              lo.z = rna_tf32(x.z - hi.z);
+              lo.w = rna_tf32(x.w - hi.w);
+              *reinterpret_cast<float4*>(sA + a_plane + sw128(tid, c)) = lo;
+            }
           }
         }
-      }
-      // prefetch the next k-block's A rows while the tensor core runs
-      if (kb + 1 < nkb) {
+        asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");  // generic -> async proxy
+        mbar_arrive(&full[s]);
+        if (kb + 1 < nkb && rv) {  // prefetch the next k-block while this one is consumed
 #pragma unroll
-        for (int v = 0; v < NV; ++v) regs[v] = tc_load4(g, row, M, (kb + 1) * EPC + v * 4);
+          for (int v = 0; v < NV; ++v) regs[v] = tc_load4(g, r0, r1, (kb + 1) * EPC + v * 4);
+        }
       }
-      asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
-      __syncthreads();
-      if (tid == 0) {
-        mbar_wait(&full[s], (gk >> 1) & 1);
+    }
+  } else if (warp == 4) {
+    // ===================== B producer (TMA bulk copies of weight tile images)
+    if (lane == 0) {
+      uint32_t gk = 0;
+      for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        const int tn = t % w.ntn;
+        for (int kb = 0; kb < nkb; ++kb, ++gk) {
+          const int s = gk % stages;
+          mbar_wait(&empty[s], ((gk / stages) & 1) ^ 1);
+          unsigned char* sB = smem + s * stage_bytes + PLANES * a_plane;
+          const unsigned char* src =
+              reinterpret_cast<const unsigned char*>(w.hi) + ((size_t)tn * nkb + kb) * PLANES * b_plane;
+          mbar_expect_tx(&full[s], PLANES * b_plane);
+          bulk_g2s(sB, src, PLANES * b_plane, &full[s]);
+        }
+      }
+    }
+  } else if (warp == 5) {
+    // ===================== MMA issuer
+    if (lane == 0) {
+      const uint32_t idesc = umma_idesc(PREC, BN);
+      uint32_t gk = 0, tc = 0;
+      for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++tc) {
+        const uint32_t acc = tc & 1;
+        mbar_wait(&tempty[acc], ((tc >> 1) & 1) ^ 1);  // epilogue drained this accumulator
         asm volatile("tcgen05.fence::after_thread_sync;\n");
-        const uint32_t aH = smem_u32(sA), bH = smem_u32(sB);
+        const uint32_t dtm = tmem + acc * TC_ACC_COLS;
+        for (int kb = 0; kb < nkb; ++kb, ++gk) {
+          const int s = gk % stages;
+          mbar_wait(&full[s], (gk / stages) & 1);
+          asm volatile("tcgen05.fence::after_thread_sync;\n");
+          const uint32_t aH = smem_u32(smem + s * stage_bytes);
+          const uint32_t bH = aH + PLANES * a_plane;
 #pragma unroll
-        for (int kk = 0; kk < 4; ++kk) {  // 4 MMAs of 32 bytes of K per 128B k-block
-          const uint32_t acc0 = (kb > 0 || kk > 0) ? 1u : 0u;
-          mma_issue(PREC, tmem, umma_desc(aH + kk * 32), umma_desc(bH + kk * 32), idesc, acc0);
-          if (PLANES == 2) {
-            mma_issue(PREC, tmem, umma_desc(aH + kk * 32), umma_desc(bH + b_plane + kk * 32), idesc, 1u);
-            mma_issue(PREC, tmem, umma_desc(aH + a_plane + kk * 32), umma_desc(bH + kk * 32), idesc, 1u);
+          for (int kk = 0; kk < 4; ++kk) {  // 4 MMAs of 32 bytes of K per 128B k-block
+            const uint32_t acc0 = (kb > 0 || kk > 0) ? 1u : 0u;
+            mma_issue<PREC>(dtm, umma_desc(aH + kk * 32), umma_desc(bH + kk * 32), idesc, acc0);
+            if (PLANES == 2) {
+              mma_issue<PREC>(dtm, umma_desc(aH + kk * 32), umma_desc(bH + b_plane + kk * 32), idesc, 1u);
+              mma_issue<PREC>(dtm, umma_desc(aH + a_plane + kk * 32), umma_desc(bH + kk * 32), idesc, 1u);
+            }
           }
+          asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n" ::"r"(
+                           smem_u32(&empty[s]))
+                       : "memory");
         }
         asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n" ::"r"(
-                         smem_u32(&done[s]))
+                         smem_u32(&tfull[acc]))
                      : "memory");
       }
     }
-    // ---- epilogue: TMEM -> registers -> bias / residual / ReLU -> global
-    const uint32_t last = gk - 1;
-    mbar_wait(&done[last & 1], (last >> 1) & 1);
-    asm volatile("tcgen05.fence::after_thread_sync;\n");
-    const int er = m0 + warp * 32 + (tid & 31);  // TMEM lane = row of the tile
-    for (int c0 = 0; c0 < BN; c0 += 16) {
-      uint32_t v[16];
-      const uint32_t taddr = tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)c0;
-      asm volatile(
-          "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];\n"
-          : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
-            "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
-          : "r"(taddr));
-      asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
+  } else {
+    // ===================== epilogue (warps 6-9 cover TMEM lane quadrants 2,3,0,1)
+    const int quad = warp & 3;
+    const int et = tid - 6 * 32;  // 0..127
+    (void)et;
+    uint32_t tc = 0;
+    for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++tc) {
+      const int tm = t / w.ntn, tn = t - tm * w.ntn;
+      const int m0 = tm * TC_BM, n0 = tn * BN;
+      const uint32_t acc = tc & 1;
+      mbar_wait(&tfull[acc], (tc >> 1) & 1);
+      asm volatile("tcgen05.fence::after_thread_sync;\n");
+      const int er = m0 + quad * 32 + lane;  // TMEM lane = row of the tile
+      float* orow = nullptr;
+      const float* qrow = nullptr;
       if (er < M) {
-        float* orow = g.c_rows ? g.c_rows[er] : g.C + (size_t)er * g.ldc;
-        const float* qrow = g.q_rows ? g.q_rows[er] : nullptr;
+        orow = g.c_rows ? g.c_rows[er] : g.C + (size_t)er * g.ldc;
+        qrow = g.q_rows ? g.q_rows[er] : nullptr;
+      }
+      for (int c0 = 0; c0 < BN; c0 += 16) {
+        uint32_t v[16];
+        const uint32_t taddr = tmem + acc * TC_ACC_COLS + ((uint32_t)(quad * 32) << 16) + (uint32_t)c0;
+        asm volatile(
+            "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, "
+            "[%16];\n"
+            : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+              "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
+            : "r"(taddr));
+        asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
+        if (orow) {
 #pragma unroll
-        for (int j4 = 0; j4 < 4; ++j4) {
-          const int c = n0 + c0 + 4 * j4;
-          if (c >= g.N) break;
-          float o[4];
+          for (int j4 = 0; j4 < 4; ++j4) {
+            const int c = n0 + c0 + 4 * j4;
+            if (c < g.N) {
+              float o[4];
 #pragma unroll
-          for (int j = 0; j < 4; ++j) {
-            float x = __uint_as_float(v[4 * j4 + j]);
-            const int cc = c + j;
-            if (g.bias) x += g.bias[cc];
-            if (qrow) {
-              if (cc < g.q_dnp) x += qrow[cc];
-              else if (cc >= g.q_dnp + g.q_dep) x += g.q_phi0[cc - g.q_dnp - g.q_dep];
+              for (int j = 0; j < 4; ++j) {
+                float x = __uint_as_float(v[4 * j4 + j]);
+                const int cc = c + j;
+                if (g.bias) x += g.bias[cc];
+                if (qrow) {
+                  if (cc < g.q_dnp) x += qrow[cc];
+                  else if (cc >= g.q_dnp + g.q_dep) x += g.q_phi0[cc - g.q_dnp - g.q_dep];
+                }
+                if (g.relu) x = fmaxf(x, 0.f);
+                o[j] = x;
+              }
+              *reinterpret_cast<float4*>(orow + c) = make_float4(o[0], o[1], o[2], o[3]);
             }
-            if (g.relu) x = fmaxf(x, 0.f);
-            o[j] = x;
           }
-          *reinterpret_cast<float4*>(orow + c) = make_float4(o[0], o[1], o[2], o[3]);
         }
       }
+      asm volatile("tcgen05.fence::before_thread_sync;\n");
+      mbar_arrive(&tempty[acc]);
     }
-    asm volatile("tcgen05.fence::before_thread_sync;\n");
-    __syncthreads();  // TMEM drained before the next tile's first MMA
-    asm volatile("tcgen05.fence::after_thread_sync;\n");
   }
+  asm volatile("tcgen05.fence::before_thread_sync;\n");
   __syncthreads();
-  if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;\n" ::"r"(tmem), "r"(256));
+  asm volatile("tcgen05.fence::after_thread_sync;\n");
+  if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;\n" ::"r"(tmem), "r"(2 * TC_ACC_COLS));
 }
 
-static size_t tc_smem(int prec, int BN) {
+static size_t tc_smem(int prec, int BN, int stages) {
   const size_t planes = tc_planes(prec);
-  return 1024 + TC_STAGES * planes * ((size_t)TC_BM * 128 + (size_t)BN * 128) + 64;
+  return 1024 + (size_t)stages * planes * ((size_t)TC_BM * 128 + (size_t)BN * 128) + 256;
 }
 
 void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaStream_t st) {
-  const size_t smem = tc_smem(precision, w.BN);
+  const int stages = tc_stages(precision, w.BN);
+  const size_t smem = tc_smem(precision, w.BN, stages);
   const int tiles = ((g.m_max + TC_BM - 1) / TC_BM) * w.ntn;
   int grid = tiles < 148 ? tiles : 148;
   if (grid < 1) grid = 1;
@@ -376,14 +443,14 @@ void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaSt
       cudaFuncSetAttribute(k_gemm_tc<TG_PREC_BF16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       set = smem;
     }
-    k_gemm_tc<TG_PREC_BF16><<<grid, TC_THREADS, smem, st>>>(g, w);
+    k_gemm_tc<TG_PREC_BF16><<<grid, TC_THREADS, smem, st>>>(g, w, stages);
   } else {
     static size_t set = 0;
     if (smem > set) {
       cudaFuncSetAttribute(k_gemm_tc<TG_PREC_TF32X3>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       set = smem;
     }
-    k_gemm_tc<TG_PREC_TF32X3><<<grid, TC_THREADS, smem, st>>>(g, w);
+    k_gemm_tc<TG_PREC_TF32X3><<<grid, TC_THREADS, smem, st>>>(g, w, stages);
   }
 }
 
