@@ -4,10 +4,15 @@
                     [--precision fp32|tf32x3|bf16] [--impl ours|reference]
 
 A *step* is one full chronological pass (batches of 200 edges) over
-the rank's contiguous shard of the stream, cold cache (tg_cache_reset, as in
-the paper's runs), i.e. the whole hot path S1-S16 per batch. For N > 1 (torchrun,
-NCCL) rank r takes batches [r*nb/N, (r+1)*nb/N); NCCL only gathers the scores
-and all-reduces the counters at the end of a step (north_star).
+the rank's stream, cold cache (tg_cache_reset, as in the paper's runs), i.e.
+the whole hot path S1-S16 per batch. For N > 1 (torchrun, NCCL), one process
+per GPU:
+  --scaling weak   (default) every rank processes its own Reddit-shaped stream
+                   (independent seed): fixed work per GPU;
+  --scaling strong the single stream is sharded into contiguous batch ranges
+                   [r*nb/N, (r+1)*nb/N) (north_star's deployment).
+NCCL only gathers the scores and all-reduces the counters at the end of a
+pass; there is no per-batch collective (batches are independent).
 
 --impl reference times the oracle (oracle/, plain float64 CPU TGAT, the
 paper's baseline role) on the host cores on a bounded sample of the same
@@ -163,7 +168,9 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="reddit")
-    ap.add_argument("--precision", default="fp32", choices=["fp32", "tf32x3", "bf16"])
+    ap.add_argument("--precision", default="bf16", choices=["fp32", "tf32x3", "bf16"])
+    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"])
+    ap.add_argument("--superbatch", type=int, default=0)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-profile", action="store_true")
@@ -181,28 +188,35 @@ def main():
             run_reference(args, cfg)
         return
 
+    import dataclasses
     import torch
     import torch.distributed as dist
     from synth import make_stream, make_params
     from paper_conf_ppopp_wangm23_b200 import (Context, TG_NCOUNTERS, counters_dict, TG_PREC_FP32,
                                               TG_PREC_TF32X3, TG_PREC_BF16)
+    from paper_conf_ppopp_wangm23_b200.shard import shard_batches, gather_scores, reduce_counters
 
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     prec = {"fp32": TG_PREC_FP32, "tf32x3": TG_PREC_TF32X3, "bf16": TG_PREC_BF16}[args.precision]
 
-    s = make_stream(args.config)
+    if args.scaling == "weak" and world > 1:
+        s = make_stream(dataclasses.replace(cfg.stream, seed=cfg.stream.seed + 7919 * rank))
+    else:
+        s = make_stream(args.config)
     flat = make_params(mc.n_layers, mc.n_heads, s.d_n, s.d_e)
     B = mc.batch
-    nb = (s.n_edges + B - 1) // B
-    b0, b1 = (rank * nb) // world, ((rank + 1) * nb) // world
-    e0, e1 = b0 * B, min(b1 * B, s.n_edges)
+    if args.scaling == "strong":
+        b0, b1, e0, e1 = shard_batches(s.n_edges, B, rank, world)
+    else:
+        b0, b1, e0, e1 = 0, (s.n_edges + B - 1) // B, 0, s.n_edges
     E_rank = e1 - e0
+    E_job = s.n_edges if args.scaling == "strong" else s.n_edges * world
     ctx = Context.from_stream(s, device=local)
     ctx.load_model(flat, n_layers=mc.n_layers, n_heads=mc.n_heads, n_neighbors=mc.n_neighbors,
                    max_batch_targets=2 * B, cache_limit=mc.cache_limit, time_window=mc.time_window,
-                   precision=prec)
+                   precision=prec, superbatch=args.superbatch)
     dev = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
     src, dst, ts = dev(s.src[e0:e1]), dev(s.dst[e0:e1]), dev(s.ts[e0:e1].view(np.int32))
     scores = torch.zeros(E_rank, dtype=torch.float32, device="cuda")
@@ -211,17 +225,21 @@ def main():
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")  # > L2 (126 MB)
     stream = torch.cuda.current_stream()
 
+    def collect(sc):
+        """End-of-pass NCCL: gather scores, all-reduce the counter vector (north_star)."""
+        if world > 1:
+            if args.scaling == "strong":
+                gather_scores(sc, s.n_edges, B, world, dist, device="cuda")
+            else:
+                parts = [torch.empty_like(sc) for _ in range(world)]
+                dist.all_gather(parts, sc)
+            reduce_counters(ctx.counters_raw(), dist, device="cuda")
+
     def step(sc=scores, a=src, b=dst, c=ts, lg=log):
         ctx.cache_reset()                       # cold cache per pass (paper's protocol)
         ctx.score_stream(a, b, c, B, sc, lg, stream=stream)
         launches = ctx.kernel_launches()
-        if world > 1:                           # NCCL: gather scores + reduce counters (north_star)
-            pad = torch.zeros(((s.n_edges + world - 1) // world) + B, dtype=torch.float32, device="cuda")
-            pad[:E_rank] = sc
-            allsc = [torch.empty_like(pad) for _ in range(world)]
-            dist.all_gather(allsc, pad)
-            cnt = torch.from_numpy(ctx.counters_raw()).cuda()
-            dist.all_reduce(cnt)
+        collect(sc)
         return launches
 
     for _ in range(args.warmup):
@@ -249,16 +267,15 @@ def main():
         tt = torch.tensor([t_rank], dtype=torch.float64, device="cuda")
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         t_max = float(tt.item())
-    value = args.steps * s.n_edges / t_max if world > 1 else args.steps * E_rank / t_max
+    value = args.steps * E_job / t_max
 
     # ---- per-batch counters of the last pass (hit rates, dedup ratios)
     lg = log.cpu().numpy().reshape(nbr, TG_NCOUNTERS)
     per = [counters_dict(r, mc.n_layers) for r in lg]
-    tot = ctx.counters()  # cumulative since last reset = last pass
+    raw = ctx.counters_raw()  # cumulative since last reset = last pass
     if world > 1:
-        t = torch.tensor(ctx.counters_raw(), device="cuda")
-        dist.all_reduce(t)
-        tot = counters_dict(t.cpu().numpy(), mc.n_layers)
+        raw = reduce_counters(raw, dist, device="cuda")
+    tot = counters_dict(raw, mc.n_layers)
 
     def rate(a, b):
         return a / b if b else None
@@ -289,6 +306,7 @@ def main():
         t0 = time.perf_counter()
         ctx.cache_reset()
         ctx.score_stream(hs_src, hs_dst, hs_ts, B, hs_sc, None, stream=stream)  # H2D in, D2H out, synced
+        collect(hs_sc.cuda(non_blocking=False)) if world > 1 else None
         t1 = time.perf_counter() - t0
         if i:
             e2e_t.append(t1)
@@ -297,7 +315,7 @@ def main():
         tt = torch.tensor([e2e_rank], dtype=torch.float64, device="cuda")
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         e2e_rank = float(tt.item())
-    e2e_val = args.steps * (s.n_edges if world > 1 else E_rank) / e2e_rank
+    e2e_val = args.steps * E_job / e2e_rank
     assert np.array_equal(hs_sc.numpy(), scores.cpu().numpy()), "host-buffer path disagrees with device path"
 
     # ---- per-stage device timing (separate profiled pass of the same workload)
@@ -315,9 +333,9 @@ def main():
         D = s.d_n + s.d_e + s.d_n
         k = mc.n_neighbors
         n_targets = sum(c[f"l{l}_misses"] for l in range(1, mc.n_layers + 1))
-        # algorithmic bytes of the attention kernel per computed target (DESIGN.md):
-        # gathered neighbour rows h_j + e_ij (HBM), Phi rows (L2 table / computed),
-        # u in and c out (2 x H x D), per-slot metadata (row ptr 8 + eid 4 + node 4 + t 4 B)
+        # algorithmic bytes of the attention kernel per computed target (DESIGN.md "Roofline"):
+        # neighbour rows h_j + e_ij, Phi rows (table or computed), u in and c out (2 x H x D),
+        # per-slot metadata (row ptr 8 + eid 4 + node 4 + t 4 B)
         per_target = k * (s.d_n + s.d_e) * 4 + k * s.d_n * 4 + 2 * mc.n_heads * D * 4 + k * 20
         attn_ms, attn_n = stages["attn"]
         achieved = (n_targets * per_target) / (attn_ms / 1e3) / 1e9
@@ -338,14 +356,16 @@ def main():
     if rank == 0:
         line = {"metric": "edges_per_sec", "value": value, "unit": "edges/s", "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t_max / args.steps,
-                "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+                "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None,
                 "dtype": {"fp32": "f32", "tf32x3": "tf32x3", "bf16": "bf16"}[args.precision],
                 "data": "synthetic",
                 "config": {"workload": args.config, "n_edges": s.n_edges, "n_nodes": s.n_nodes,
-                           "batch": B, "n_layers": mc.n_layers, "heads": mc.n_heads, "k": mc.n_neighbors,
-                           "d_n": s.d_n, "d_e": s.d_e, "cache_limit": mc.cache_limit,
+                           "edges_per_rank": E_rank, "batch": B, "n_layers": mc.n_layers, "heads": mc.n_heads,
+                           "k": mc.n_neighbors, "d_n": s.d_n, "d_e": s.d_e, "cache_limit": mc.cache_limit,
                            "time_window": mc.time_window, "opts": "dedup+cache+ttable",
-                           "parallelism": f"batch-range shards x{world}",
+                           "superbatch": args.superbatch or 16,
+                           "parallelism": (f"independent streams x{world}" if args.scaling == "weak"
+                                           else f"batch-range shards x{world}"),
                            "l2": "flushed (256 MB write) before every timed step; inputs > L2",
                            "step": "one cold-cache chronological pass over the rank's batches"},
                 "e2e": {"value": e2e_val, "unit": "edges/s", "h2d_bytes_per_step": 12 * E_rank,
