@@ -168,7 +168,7 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="reddit")
-    ap.add_argument("--precision", default="bf16", choices=["fp32", "tf32x3", "bf16"])
+    ap.add_argument("--precision", default="bf16", choices=["fp32", "tf32x3", "bf16", "tf32"])
     ap.add_argument("--scaling", default="weak", choices=["weak", "strong"])
     ap.add_argument("--superbatch", type=int, default=0)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
@@ -193,13 +193,13 @@ def main():
     import torch.distributed as dist
     from synth import make_stream, make_params
     from paper_conf_ppopp_wangm23_b200 import (Context, TG_NCOUNTERS, counters_dict, TG_PREC_FP32,
-                                              TG_PREC_TF32X3, TG_PREC_BF16)
+                                              TG_PREC_TF32X3, TG_PREC_BF16, TG_PREC_TF32)
     from paper_conf_ppopp_wangm23_b200.shard import shard_batches, gather_scores, reduce_counters
 
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    prec = {"fp32": TG_PREC_FP32, "tf32x3": TG_PREC_TF32X3, "bf16": TG_PREC_BF16}[args.precision]
+    prec = {"fp32": TG_PREC_FP32, "tf32x3": TG_PREC_TF32X3, "bf16": TG_PREC_BF16, "tf32": TG_PREC_TF32}[args.precision]
 
     if args.scaling == "weak" and world > 1:
         s = make_stream(dataclasses.replace(cfg.stream, seed=cfg.stream.seed + 7919 * rank))
@@ -357,7 +357,7 @@ def main():
         line = {"metric": "edges_per_sec", "value": value, "unit": "edges/s", "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t_max / args.steps,
                 "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None,
-                "dtype": {"fp32": "f32", "tf32x3": "tf32x3", "bf16": "bf16"}[args.precision],
+                "dtype": {"fp32": "f32", "tf32x3": "tf32x3", "bf16": "bf16", "tf32": "tf32"}[args.precision],
                 "data": "synthetic",
                 "config": {"workload": args.config, "n_edges": s.n_edges, "n_nodes": s.n_nodes,
                            "edges_per_rank": E_rank, "batch": B, "n_layers": mc.n_layers, "heads": mc.n_heads,

@@ -59,6 +59,8 @@ typedef struct tg_ctx tg_ctx; /* opaque; one per device */
 #define TG_PREC_FP32  0   /* fp32 FFMA (CUDA cores): rtol 1e-4 / atol 1e-5 vs oracle */
 #define TG_PREC_TF32X3 1  /* tcgen05 kind::tf32, 3-term hi/lo split: fp32-level error */
 #define TG_PREC_BF16  2   /* tcgen05 kind::f16 bf16 operands, fp32 accumulate: rtol 2e-2 */
+#define TG_PREC_TF32  3   /* tcgen05 kind::tf32 one pass (A streamed raw fp32, B rna-tf32): rtol 2e-2 class */
+#define TG_PREC_LAST  TG_PREC_TF32
 
 /* ------------------------------------------------------------------------ */
 /* Graph: a CTDG edge stream with static node/edge features.        */

@@ -107,7 +107,7 @@ tg_status tc_prepare_weights(const float* W, int N, int K, int precision, TcWeig
               lo[e] = tf32_rna(x - hi[e]);
             }
             memcpy(dst0, hi, 16);
-            memcpy(dst0 + plane_bytes, lo, 16);
+            if (planes == 2) memcpy(dst0 + plane_bytes, lo, 16);
           }
         }
       }
@@ -253,7 +253,41 @@ __global__ void __launch_bounds__(TC_THREADS, 1) k_gemm_tc(GemmArgs g, TcWeights
   asm volatile("tcgen05.fence::after_thread_sync;\n");
   const uint32_t tmem = *tmem_slot;
 
-  if (warp < 4) {
+  if (warp < 4 && PREC == TG_PREC_TF32) {
+    // ===================== A producers, streamed: raw fp32 rows go straight into
+    // the swizzled operand with 16-byte cp.async (zero-fill past K / M); the
+    // tensor core reads them as tf32. Completion is tracked by the full barrier
+    // (cp.async.mbarrier.arrive.noinc), so `stages` k-blocks are in flight.
+    uint32_t gk = 0;
+    for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+      const int tm = t / w.ntn;
+      const int row = tm * TC_BM + tid;
+      const bool rv = row < M;
+      const float* r0 = g.a_base0;  // any valid address for zero-fill copies
+      const float* r1 = g.a_base0;
+      if (rv) {
+        r0 = g.a_rows0 ? g.a_rows0[row] : g.a_base0 + (size_t)row * g.lda0;
+        if (g.K0 < g.K) r1 = g.a_rows1 ? g.a_rows1[row] : g.a_base1 + (size_t)row * g.lda1;
+      } else if (g.a_rows0) {
+        r0 = r1 = g.a_rows0[0];
+      }
+      for (int kb = 0; kb < nkb; ++kb, ++gk) {
+        const int s = gk % stages;
+        mbar_wait(&empty[s], ((gk / stages) & 1) ^ 1);
+        const uint32_t sA = smem_u32(smem + s * stage_bytes);
+#pragma unroll
+        for (int c = 0; c < 8; ++c) {
+          const int col = kb * EPC + c * 4;
+          const bool ok = rv && col < g.K;
+          const float* src = !ok ? r0 : (col < g.K0 ? r0 + col : r1 + (col - g.K0));
+          asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(sA + sw128(tid, c)), "l"(src),
+                       "r"(ok ? 16 : 0)
+                       : "memory");
+        }
+        asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];\n" ::"r"(smem_u32(&full[s])) : "memory");
+      }
+    }
+  } else if (warp < 4) {
     // ===================== A producers
     uint32_t gk = 0;
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
@@ -343,6 +377,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1) k_gemm_tc(GemmArgs g, TcWeights
         for (int kb = 0; kb < nkb; ++kb, ++gk) {
           const int s = gk % stages;
           mbar_wait(&full[s], (gk / stages) & 1);
+          asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");  // cp.async A -> tensor core
           asm volatile("tcgen05.fence::after_thread_sync;\n");
           const uint32_t aH = smem_u32(smem + s * stage_bytes);
           const uint32_t bH = aH + PLANES * a_plane;
@@ -444,6 +479,13 @@ void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaSt
       set = smem;
     }
     k_gemm_tc<TG_PREC_BF16><<<grid, TC_THREADS, smem, st>>>(g, w, stages);
+  } else if (precision == TG_PREC_TF32) {
+    static size_t set = 0;
+    if (smem > set) {
+      cudaFuncSetAttribute(k_gemm_tc<TG_PREC_TF32>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      set = smem;
+    }
+    k_gemm_tc<TG_PREC_TF32><<<grid, TC_THREADS, smem, st>>>(g, w, stages);
   } else {
     static size_t set = 0;
     if (smem > set) {

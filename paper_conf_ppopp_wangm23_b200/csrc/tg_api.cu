@@ -528,7 +528,7 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
   const int D = d_n + d_e + d_t;
   if (L < 1 || L > TG_MAX_LAYERS || H < 1 || H > 8 || k < 1 || k > kMaxK || d_t < 1 || D % H) return TG_EINVAL;
   if (cfg->max_batch_targets < 1 || cfg->cache_limit < 0 || cfg->time_window < 0) return TG_EINVAL;
-  if (cfg->precision < TG_PREC_FP32 || cfg->precision > TG_PREC_BF16) return TG_EINVAL;
+  if (cfg->precision < TG_PREC_FP32 || cfg->precision > TG_PREC_LAST) return TG_EINVAL;
   if (cfg->superbatch < 0 || cfg->superbatch > kMaxS) return TG_EINVAL;
   const int64_t per_layer = 4LL * D * D + 3LL * D + (int64_t)d_n * (D + d_n) + d_n + (int64_t)d_n * d_n + d_n;
   const int64_t expect = L * per_layer + 2LL * d_t + 2LL * d_n * d_n + d_n + d_n + 1;
@@ -1001,7 +1001,7 @@ tg_status tg_time_encode(tg_ctx* ctx, const int64_t* delta, int64_t n, int32_t u
 tg_status tg_gemm(tg_ctx* ctx, int32_t precision, int32_t M, int32_t N, int32_t K, const float* A,
                   const float* B, const float* bias, int32_t relu, float* C, void* cuda_stream) {
   if (!ctx || M < 0 || N < 4 || K < 4 || (N & 3) || (K & 3) || !A || !B || !C) return TG_EINVAL;
-  if (precision < TG_PREC_FP32 || precision > TG_PREC_BF16) return TG_EINVAL;
+  if (precision < TG_PREC_FP32 || precision > TG_PREC_LAST) return TG_EINVAL;
   cudaStream_t st = (cudaStream_t)cuda_stream;
   CK(cudaSetDevice(ctx->device));
   int* mdev = nullptr;
