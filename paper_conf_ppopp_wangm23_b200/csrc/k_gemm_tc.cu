@@ -72,8 +72,10 @@ static inline uint16_t bf16_rn(float x) {
 
 tg_status tc_prepare_weights(const float* W, int N, int K, int precision, TcWeights* out,
                              std::vector<void*>& owned) {
-  // N tiles of <= 128 columns (more CTAs at the small M of a superbatch)
-  const int ntn = (N + 127) / 128;
+  // N tiles of <= 256 columns: each A tile is re-read once per N tile, and the
+  // kernel is bound by L2 -> SM operand traffic at these sizes
+  // (narrow GEMMs, N <= 256, keep two N tiles for parallelism instead)
+  const int ntn = N > 256 ? (N + 255) / 256 : (N + 127) / 128;
   int BN = (N + ntn - 1) / ntn;
   BN = (BN + 15) & ~15;
   const int epc = tc_epc(precision);
