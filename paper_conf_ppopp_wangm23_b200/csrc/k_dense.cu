@@ -105,31 +105,58 @@ __global__ void k_layernorm(const float* __restrict__ y, float* __restrict__ r, 
   const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, nw = (gridDim.x * blockDim.x) >> 5;
   const int D = dn + de + dt;
   const int s1 = dnp, s2 = dnp + dep;
+  const int D4 = Dp >> 2;
+  // warp per row; the row (<= 1024 floats) is read once into registers
   for (int row = warp; row < M; row += nw) {
-    const float* yr = y + (size_t)row * Dp;
-    float* rr = r + (size_t)row * Dp;
+    const float4* yr = reinterpret_cast<const float4*>(y + (size_t)row * Dp);
+    float4* rr = reinterpret_cast<float4*>(r + (size_t)row * Dp);
+    float4 v[8];
     float sum = 0.f;
-    for (int c = lane; c < Dp; c += 32) {
-      const bool valid = c < dn || (c >= s1 && c < s1 + de) || (c >= s2 && c < s2 + dt);
-      if (valid) sum += yr[c];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const int q = lane + 32 * j;
+      v[j] = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (q < D4) {
+        v[j] = yr[q];
+        // padded columns are exact zeros (zero weight rows / bias), so they do not bias the sum
+        sum += (v[j].x + v[j].y) + (v[j].z + v[j].w);
+      }
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
     const float mu = sum / (float)D;
     float var = 0.f;
-    for (int c = lane; c < Dp; c += 32) {
-      const bool valid = c < dn || (c >= s1 && c < s1 + de) || (c >= s2 && c < s2 + dt);
-      if (valid) {
-        const float d = yr[c] - mu;
-        var = fmaf(d, d, var);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const int q = lane + 32 * j;
+      if (q < D4) {
+        const float e[4] = {v[j].x, v[j].y, v[j].z, v[j].w};
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const int c = 4 * q + i;
+          const bool valid = c < dn || (c >= s1 && c < s1 + de) || (c >= s2 && c < s2 + dt);
+          const float d = e[i] - mu;
+          if (valid) var = fmaf(d, d, var);
+        }
       }
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) var += __shfl_xor_sync(0xffffffffu, var, o);
     const float rstd = rsqrtf(var / (float)D + 1e-5f);
-    for (int c = lane; c < Dp; c += 32) {
-      const bool valid = c < dn || (c >= s1 && c < s1 + de) || (c >= s2 && c < s2 + dt);
-      rr[c] = valid ? (yr[c] - mu) * rstd * gamma[c] + beta[c] : 0.f;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const int q = lane + 32 * j;
+      if (q < D4) {
+        const float e[4] = {v[j].x, v[j].y, v[j].z, v[j].w};
+        float o4[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const int c = 4 * q + i;
+          const bool valid = c < dn || (c >= s1 && c < s1 + de) || (c >= s2 && c < s2 + dt);
+          o4[i] = valid ? (e[i] - mu) * rstd * gamma[c] + beta[c] : 0.f;
+        }
+        rr[q] = make_float4(o4[0], o4[1], o4[2], o4[3]);
+      }
     }
   }
 }

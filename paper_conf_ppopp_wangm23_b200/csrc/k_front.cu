@@ -216,7 +216,8 @@ __global__ void k_dedup_off(LevelDev lv, int S, int edge_mode, EdgeSrc es, long 
 
 static int dedup_cluster_size(int n_max) {
   int cl = 1;
-  while (cl < 16 && (long long)cl * 10000 < n_max) cl <<= 1;
+  // ~2.5k items per CTA: enough threads per batch that the phases are short
+  while (cl < 16 && ((long long)cl * 2560 < n_max || (long long)cl * 10000 < n_max)) cl <<= 1;
   return cl;
 }
 
@@ -741,6 +742,52 @@ k_probe_par(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err)
   }
 }
 
+// No lookup (top layer, R9; or cache disabled): C = the unique lists of the S
+// batches concatenated in batch order, q = c_base[b] + u. With a ring (cache
+// disabled at a cached level) the rows still go to FIFO positions head + q,
+// used as per-superbatch scratch.
+__global__ void k_compact_all(LevelDev lv, int S, CacheDev c, int has_ring, long long* cnt, int layer) {
+  __shared__ int s_pre[kMaxS + 1];
+  if (threadIdx.x == 0) {
+    int a = 0;
+    for (int b = 0; b < S; ++b) {
+      s_pre[b] = a;
+      a += lv.n_u[b];
+    }
+    s_pre[S] = a;
+  }
+  __syncthreads();
+  const long long head = has_ring ? c.state[0] : 0;
+  const int tot = S * lv.cap;
+  for (int idx = blockIdx.x * blockDim.x + threadIdx.x; idx < tot; idx += gridDim.x * blockDim.x) {
+    const int b = idx / lv.cap, u = idx - b * lv.cap;
+    if (u >= s_pre[b + 1] - s_pre[b]) continue;
+    const int q = s_pre[b] + u;
+    lv.c_b[q] = b;
+    lv.c_u[q] = u;
+    lv.c_node[q] = lv.u_node[idx];
+    lv.c_ts[q] = lv.u_ts[idx];
+    if (has_ring) lv.slot[idx] = (head + q) % c.rcap;
+  }
+  if (blockIdx.x == 0) {
+    for (int b = threadIdx.x; b < S; b += blockDim.x) {
+      const int m = s_pre[b + 1] - s_pre[b];
+      lv.c_base[b] = s_pre[b];
+      lv.n_c[b] = m;
+      cnt_add(cnt, b, layer * TG_CNT_PER_LAYER + 4, m);  // misses = embeddings computed
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      *lv.n_c_total = s_pre[S];
+      // every block has read head before the grid ends; the next launch sees the update
+    }
+  }
+}
+
+// head update of the scratch ring after k_compact_all (separate launch: no
+// intra-grid ordering needed)
+__global__ void k_ring_advance(LevelDev lv, CacheDev c) { c.state[0] += *lv.n_c_total; }
+
 __global__ void k_probe_ins(LevelDev lv, CacheDev c, int* err) {
   const int n = *lv.n_c_total;
   const long long head0 = c.state[4];
@@ -773,8 +820,8 @@ __global__ void k_probe_ins(LevelDev lv, CacheDev c, int* err) {
   }
 }
 
-void launch_probe(LevelDev lv, int S, const CacheDev* cache, long long* cnt, int layer, int* err,
-                  cudaStream_t st) {
+int launch_probe(LevelDev lv, int S, const CacheDev* cache, long long* cnt, int layer, int* err,
+                 cudaStream_t st) {
   CacheDev c{};
   int has_ring = 0, use_cache = 0;
   if (cache) {
@@ -782,9 +829,16 @@ void launch_probe(LevelDev lv, int S, const CacheDev* cache, long long* cnt, int
     has_ring = 1;
     use_cache = c.ikey != nullptr;
   }
-  if (!use_cache) {  // top layer (no lookup, R9) or cache disabled: ordered compaction only
-    k_probe<<<1, 1024, 0, st>>>(lv, S, c, 0, has_ring, cnt, layer, err);
-    return;
+  if (!use_cache) {  // top layer (no lookup, R9) or cache disabled: every unique entry is computed
+    int blocks = (S * lv.cap + 255) / 256;
+    if (blocks > 148 * 4) blocks = 148 * 4;
+    if (blocks < 1) blocks = 1;
+    k_compact_all<<<blocks, 256, 0, st>>>(lv, S, c, has_ring, cnt, layer);
+    if (has_ring) {
+      k_ring_advance<<<1, 1, 0, st>>>(lv, c);
+      return 2;
+    }
+    return 1;
   }
   int blocks = (S * lv.cap + 255) / 256;
   if (blocks > 148 * 8) blocks = 148 * 8;
@@ -822,6 +876,7 @@ void launch_probe(LevelDev lv, int S, const CacheDev* cache, long long* cnt, int
   int ib = (S * lv.cap + 255) / 256;
   if (ib > 148 * 4) ib = 148 * 4;
   k_probe_ins<<<ib, 256, 0, st>>>(lv, c, err);
+  return 4;
 }
 
 // ------------------------------------------------------------------ NghLookup

@@ -310,11 +310,12 @@ tg_status run_superbatch(tg_ctx* ctx, int S, bool edge_mode, const EdgeSrc& es, 
     launch_dedup(ctx->lv[L], S, n_max_top, edge_mode, es, cnt, L, dedup, ctx->err, st);
   }
   TRY(launched(ctx));
+  int nl;
   {
     Prof pf(ctx, TG_ST_LOOKUP, st);
-    launch_probe(ctx->lv[L], S, nullptr, cnt, L, ctx->err, st);  // no lookup at l = L
+    nl = launch_probe(ctx->lv[L], S, nullptr, cnt, L, ctx->err, st);  // no lookup at l = L
   }
-  TRY(launched(ctx));
+  TRY(launched(ctx, nl));
   for (int l = L; l >= 1; --l) {
     {
       Prof pf(ctx, TG_ST_SAMPLE, st);
@@ -332,9 +333,9 @@ tg_status run_superbatch(tg_ctx* ctx, int S, bool edge_mode, const EdgeSrc& es, 
       if (!cache_on) cd.ikey = nullptr;  // ring used as scratch only
       {
         Prof pf(ctx, TG_ST_LOOKUP, st);
-        launch_probe(ctx->lv[l - 1], S, &cd, cnt, l - 1, ctx->err, st);
+        nl = launch_probe(ctx->lv[l - 1], S, &cd, cnt, l - 1, ctx->err, st);
       }
-      TRY(launched(ctx, cache_on ? 3 : 1));
+      TRY(launched(ctx, nl));
     }
   }
   // ---- row addresses for every layer
@@ -530,6 +531,7 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
   if (cfg->max_batch_targets < 1 || cfg->cache_limit < 0 || cfg->time_window < 0) return TG_EINVAL;
   if (cfg->precision < TG_PREC_FP32 || cfg->precision > TG_PREC_LAST) return TG_EINVAL;
   if (cfg->superbatch < 0 || cfg->superbatch > kMaxS) return TG_EINVAL;
+  if (round4(d_n) + round4(d_e) + round4(d_t) > 1024) return TG_EINVAL;  // LayerNorm row in registers
   const int64_t per_layer = 4LL * D * D + 3LL * D + (int64_t)d_n * (D + d_n) + d_n + (int64_t)d_n * d_n + d_n;
   const int64_t expect = L * per_layer + 2LL * d_t + 2LL * d_n * d_n + d_n + d_n + 1;
   if (n_params != expect) return TG_EINVAL;

@@ -127,8 +127,8 @@ void launch_dedup(LevelDev lv, int S, int n_max, bool edge_mode, EdgeSrc es, lon
 // CacheLookup + compaction + slot assignment + index insert, sequential over
 // the S batches (Alg. 1 l.7-10 and CacheStore, Alg. 3, in batch order).
 // cache == nullptr: no lookup (top layer, R9, or cache disabled).
-void launch_probe(LevelDev lv, int S, const CacheDev* cache, long long* cnt, int layer, int* err,
-                  cudaStream_t st);
+int launch_probe(LevelDev lv, int S, const CacheDev* cache, long long* cnt, int layer, int* err,
+                 cudaStream_t st);  // returns the number of kernels launched
 
 // NghLookup for every q of level `lv`; writes lv.nb_* and,
 // if next != nullptr, the batch-segmented input list of level l-1 (Alg. 1 l.12).
