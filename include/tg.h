@@ -188,7 +188,7 @@ tg_status tg_time_encode(tg_ctx* ctx, const int64_t* delta, int64_t n, int32_t u
 /* Dense projection GEMM unit entry point (the kernels of the M/FFN stages):
  * C[M x N] = A[M x K] . B[N x K]^T (+ bias[N] if non-null, then ReLU if relu),
  * all device float32 row-major; precision TG_PREC_* selects SIMT fp32,
- * tcgen05 tf32x3 or tcgen05 bf16. K, N multiples of 4. Synchronous. */
+ * tcgen05 tf32x3 / tf32 / bf16. K, N multiples of 4. Stream-ordered (asynchronous). */
 tg_status tg_gemm(tg_ctx* ctx, int32_t precision, int32_t M, int32_t N, int32_t K, const float* A,
                   const float* B, const float* bias, int32_t relu, float* C, void* cuda_stream);
 

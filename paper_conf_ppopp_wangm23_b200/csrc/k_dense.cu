@@ -1,6 +1,8 @@
 // Dense per-target stages of M and the merge FFN (Eqs. 6-7) on CUDA cores
 // (TG_PREC_FP32), LayerNorm (R1), the link-prediction score (R10) and the
 // DedupInvert row copy (Alg. 1 l.20).
+#include <cuda_bf16.h>
+
 #include "tg_internal.cuh"
 
 namespace tg {
@@ -99,7 +101,8 @@ void launch_gemm_simt(const GemmArgs& g, cudaStream_t st) {
 // ---------------------------------------------------------------- LayerNorm
 __global__ void k_layernorm(const float* __restrict__ y, float* __restrict__ r, int Dp, int dn, int dnp, int de,
                             int dep, int dt, const float* __restrict__ gamma, const float* __restrict__ beta,
-                            const int* __restrict__ m_dev) {
+                            const int* __restrict__ m_dev, const float* const* __restrict__ hs_rows,
+                            unsigned short* __restrict__ rh, int ldrh) {
   const int M = *m_dev;
   const int lane = threadIdx.x & 31;
   const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, nw = (gridDim.x * blockDim.x) >> 5;
@@ -109,7 +112,7 @@ __global__ void k_layernorm(const float* __restrict__ y, float* __restrict__ r, 
   // warp per row; the row (<= 1024 floats) is read once into registers
   for (int row = warp; row < M; row += nw) {
     const float4* yr = reinterpret_cast<const float4*>(y + (size_t)row * Dp);
-    float4* rr = reinterpret_cast<float4*>(r + (size_t)row * Dp);
+    float4* rr = r ? reinterpret_cast<float4*>(r + (size_t)row * Dp) : nullptr;
     float4 v[8];
     float sum = 0.f;
 #pragma unroll
@@ -155,18 +158,38 @@ __global__ void k_layernorm(const float* __restrict__ y, float* __restrict__ r, 
           const bool valid = c < dn || (c >= s1 && c < s1 + de) || (c >= s2 && c < s2 + dt);
           o4[i] = valid ? (e[i] - mu) * rstd * gamma[c] + beta[c] : 0.f;
         }
-        rr[q] = make_float4(o4[0], o4[1], o4[2], o4[3]);
+        if (rr) rr[q] = make_float4(o4[0], o4[1], o4[2], o4[3]);
+        if (rh) {
+          __nv_bfloat162 lo = __floats2bfloat162_rn(o4[0], o4[1]), hi = __floats2bfloat162_rn(o4[2], o4[3]);
+          uint2 pk;
+          pk.x = *reinterpret_cast<uint32_t*>(&lo);
+          pk.y = *reinterpret_cast<uint32_t*>(&hi);
+          *reinterpret_cast<uint2*>(rh + (size_t)row * ldrh + 4 * q) = pk;
+        }
+      }
+    }
+    if (rh) {  // [LN(y) | h^(l-1) | 0]: the merge-FFN input (Eq. 7) as one bf16 row
+      const float4* hr = reinterpret_cast<const float4*>(hs_rows[row]);
+      for (int q = lane; 4 * q < ldrh - Dp; q += 32) {
+        float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (4 * q < dnp) x = hr[q];
+        __nv_bfloat162 lo = __floats2bfloat162_rn(x.x, x.y), hi = __floats2bfloat162_rn(x.z, x.w);
+        uint2 pk;
+        pk.x = *reinterpret_cast<uint32_t*>(&lo);
+        pk.y = *reinterpret_cast<uint32_t*>(&hi);
+        *reinterpret_cast<uint2*>(rh + (size_t)row * ldrh + Dp + 4 * q) = pk;
       }
     }
   }
 }
 
 void launch_layernorm(const float* y, float* r, int Dp, int dn, int dnp, int de, int dep, int dt,
-                      const float* gamma, const float* beta, const int* m_dev, int m_max, cudaStream_t st) {
+                      const float* gamma, const float* beta, const int* m_dev, int m_max,
+                      const float* const* hs_rows, unsigned short* rh, int ldrh, cudaStream_t st) {
   int blocks = (m_max * 32 + 255) / 256;
   if (blocks < 1) blocks = 1;
   if (blocks > 1184) blocks = 1184;
-  k_layernorm<<<blocks, 256, 0, st>>>(y, r, Dp, dn, dnp, de, dep, dt, gamma, beta, m_dev);
+  k_layernorm<<<blocks, 256, 0, st>>>(y, r, Dp, dn, dnp, de, dep, dt, gamma, beta, m_dev, hs_rows, rh, ldrh);
 }
 
 // -------------------------------------------------------------------- score
@@ -245,5 +268,8 @@ void launch_invert(const float* HL, int ldh, LevelDev top, int n, int dn, float*
   if (blocks > 1184) blocks = 1184;
   k_invert<<<blocks, 256, 0, st>>>(HL, ldh, top, n, dn, out);
 }
+
+__global__ void k_set_int(int* p, int v) { *p = v; }
+void launch_set_int(int* p, int v, cudaStream_t st) { k_set_int<<<1, 1, 0, st>>>(p, v); }
 
 }  // namespace tg

@@ -30,7 +30,10 @@ constexpr int TC_BM = 128;
 constexpr int TC_WARPS = 10;
 constexpr int TC_THREADS = TC_WARPS * 32;
 constexpr int TC_MAXSTAGES = 4;
-constexpr int TC_ACC_COLS = 256;  // per accumulator buffer (x2 = all 512 TMEM columns)
+// TMEM: two accumulator buffers of 256 columns (all 512 columns; one CTA per
+// SM). Two CTAs per SM with 2 x 128 columns each was measured slower.
+__host__ __device__ constexpr int tc_acc_cols(int) { return 256; }
+__host__ __device__ constexpr int tc_ctas_per_sm(int) { return 1; }
 
 __host__ __device__ inline int tc_epc(int prec) { return prec == TG_PREC_BF16 ? 64 : 32; }  // elems / 128B
 __host__ __device__ inline int tc_planes(int prec) { return prec == TG_PREC_TF32X3 ? 2 : 1; }
@@ -42,7 +45,8 @@ __host__ __device__ inline unsigned sw128(int r, int c) {
 
 static inline int tc_stages(int prec, int BN) {
   const size_t st = (size_t)tc_planes(prec) * ((size_t)TC_BM * 128 + (size_t)BN * 128);
-  int s = (int)((200 * 1024) / st);
+  const size_t budget = tc_ctas_per_sm(prec) == 1 ? 200 * 1024 : 108 * 1024;
+  int s = (int)(budget / st);
   if (s > TC_MAXSTAGES) s = TC_MAXSTAGES;
   return s < 2 ? 2 : s;
 }
@@ -75,7 +79,7 @@ tg_status tc_prepare_weights(const float* W, int N, int K, int precision, TcWeig
   // N tiles of <= 256 columns: each A tile is re-read once per N tile, and the
   // kernel is bound by L2 -> SM operand traffic at these sizes
   // (narrow GEMMs, N <= 256, keep two N tiles for parallelism instead)
-  const int ntn = N > 256 ? (N + 255) / 256 : (N + 127) / 128;
+  const int ntn = (N > 256 && tc_acc_cols(precision) == 256) ? (N + 255) / 256 : (N + 127) / 128;
   int BN = (N + ntn - 1) / ntn;
   BN = (BN + 15) & ~15;
   const int epc = tc_epc(precision);
@@ -247,7 +251,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1) k_gemm_tc(GemmArgs g, TcWeights
   }
   if (warp == 0) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;\n" ::"r"(smem_u32(tmem_slot)),
-                 "r"(2 * TC_ACC_COLS));
+                 "r"(2 * tc_acc_cols(PREC)));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;\n");
   }
   asm volatile("tcgen05.fence::before_thread_sync;\n");
@@ -284,6 +288,32 @@ __global__ void __launch_bounds__(TC_THREADS, 1) k_gemm_tc(GemmArgs g, TcWeights
           const float* src = !ok ? r0 : (col < g.K0 ? r0 + col : r1 + (col - g.K0));
           asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(sA + sw128(tid, c)), "l"(src),
                        "r"(ok ? 16 : 0)
+                       : "memory");
+        }
+        asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];\n" ::"r"(smem_u32(&full[s])) : "memory");
+      }
+    }
+  } else if (warp < 4 && PREC == TG_PREC_BF16 && g.a_h) {
+    // ===================== A producers, streamed bf16: the activation was
+    // written in bf16 by the producing kernel (attention, LayerNorm, FFN1), so
+    // its rows go straight into the swizzled operand (64 elements = 128 B per
+    // k-block row) with cp.async; `stages` k-blocks are in flight.
+    uint32_t gk = 0;
+    for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+      const int tm = t / w.ntn;
+      const int row = tm * TC_BM + tid;
+      const bool rv = row < M;
+      const unsigned short* ar = g.a_h + (size_t)(rv ? row : 0) * g.lda_h;
+      for (int kb = 0; kb < nkb; ++kb, ++gk) {
+        const int s = gk % stages;
+        mbar_wait(&empty[s], ((gk / stages) & 1) ^ 1);
+        const uint32_t sA = smem_u32(smem + s * stage_bytes);
+#pragma unroll
+        for (int c = 0; c < 8; ++c) {
+          const int col = kb * EPC + c * 8;
+          const bool ok = rv && col < g.lda_h;  // [K, lda_h) is zero padding
+          asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(sA + sw128(tid, c)),
+                       "l"(ok ? ar + col : ar), "r"(ok ? 16 : 0)
                        : "memory");
         }
         asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];\n" ::"r"(smem_u32(&full[s])) : "memory");
@@ -375,7 +405,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1) k_gemm_tc(GemmArgs g, TcWeights
         const uint32_t acc = tc & 1;
         mbar_wait(&tempty[acc], ((tc >> 1) & 1) ^ 1);  // epilogue drained this accumulator
         asm volatile("tcgen05.fence::after_thread_sync;\n");
-        const uint32_t dtm = tmem + acc * TC_ACC_COLS;
+        const uint32_t dtm = tmem + acc * tc_acc_cols(PREC);
         for (int kb = 0; kb < nkb; ++kb, ++gk) {
           const int s = gk % stages;
           mbar_wait(&full[s], (gk / stages) & 1);
@@ -416,13 +446,16 @@ __global__ void __launch_bounds__(TC_THREADS, 1) k_gemm_tc(GemmArgs g, TcWeights
       const int er = m0 + quad * 32 + lane;  // TMEM lane = row of the tile
       float* orow = nullptr;
       const float* qrow = nullptr;
+      unsigned short* hrow = nullptr;
       if (er < M) {
-        orow = g.c_rows ? g.c_rows[er] : g.C + (size_t)er * g.ldc;
+        if (g.c_rows) orow = g.c_rows[er];
+        else if (g.C) orow = g.C + (size_t)er * g.ldc;
         qrow = g.q_rows ? g.q_rows[er] : nullptr;
+        if (g.c_h) hrow = g.c_h + (size_t)er * g.ldc_h;
       }
       for (int c0 = 0; c0 < BN; c0 += 16) {
         uint32_t v[16];
-        const uint32_t taddr = tmem + acc * TC_ACC_COLS + ((uint32_t)(quad * 32) << 16) + (uint32_t)c0;
+        const uint32_t taddr = tmem + acc * tc_acc_cols(PREC) + ((uint32_t)(quad * 32) << 16) + (uint32_t)c0;
         asm volatile(
             "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, "
             "[%16];\n"
@@ -430,7 +463,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1) k_gemm_tc(GemmArgs g, TcWeights
               "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
             : "r"(taddr));
         asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
-        if (orow) {
+        if (orow || hrow) {
 #pragma unroll
           for (int j4 = 0; j4 < 4; ++j4) {
             const int c = n0 + c0 + 4 * j4;
@@ -448,7 +481,16 @@ __global__ void __launch_bounds__(TC_THREADS, 1) k_gemm_tc(GemmArgs g, TcWeights
                 if (g.relu) x = fmaxf(x, 0.f);
                 o[j] = x;
               }
-              *reinterpret_cast<float4*>(orow + c) = make_float4(o[0], o[1], o[2], o[3]);
+              if (orow) *reinterpret_cast<float4*>(orow + c) = make_float4(o[0], o[1], o[2], o[3]);
+              if (hrow) {  // bf16 activation for the next projection (N % 4 == 0)
+                __nv_bfloat162 lo = __floats2bfloat162_rn(o[0], o[1]), hi = __floats2bfloat162_rn(o[2], o[3]);
+                uint2 pk;
+                pk.x = *reinterpret_cast<uint32_t*>(&lo);
+                pk.y = *reinterpret_cast<uint32_t*>(&hi);
+                *reinterpret_cast<uint2*>(hrow + c) = pk;
+              }
+            } else if (hrow && c < g.ldc_h) {  // zero padding [N, ldc_h)
+              *reinterpret_cast<uint2*>(hrow + c) = make_uint2(0u, 0u);
             }
           }
         }
@@ -460,19 +502,25 @@ __global__ void __launch_bounds__(TC_THREADS, 1) k_gemm_tc(GemmArgs g, TcWeights
   asm volatile("tcgen05.fence::before_thread_sync;\n");
   __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;\n");
-  if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;\n" ::"r"(tmem), "r"(2 * TC_ACC_COLS));
+  if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;\n" ::"r"(tmem), "r"(2 * tc_acc_cols(PREC)));
 }
 
 static size_t tc_smem(int prec, int BN, int stages) {
   const size_t planes = tc_planes(prec);
-  return 1024 + (size_t)stages * planes * ((size_t)TC_BM * 128 + (size_t)BN * 128) + 256;
+  size_t s = 1024 + (size_t)stages * planes * ((size_t)TC_BM * 128 + (size_t)BN * 128) + 256;
+  // tf32x3: one CTA per SM (it allocates all 512 TMEM columns; a second
+  // co-resident CTA would block in tcgen05.alloc until the first one exits).
+  const size_t one_per_sm = 120 * 1024;
+  if (tc_ctas_per_sm(prec) == 1 && s < one_per_sm) return one_per_sm;
+  return s;
 }
 
 void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaStream_t st) {
   const int stages = tc_stages(precision, w.BN);
   const size_t smem = tc_smem(precision, w.BN, stages);
   const int tiles = ((g.m_max + TC_BM - 1) / TC_BM) * w.ntn;
-  int grid = tiles < 148 ? tiles : 148;
+  const int slots = 148 * tc_ctas_per_sm(precision);
+  int grid = tiles < slots ? tiles : slots;
   if (grid < 1) grid = 1;
   if (precision == TG_PREC_BF16) {
     static size_t set = 0;

@@ -58,6 +58,9 @@ struct tg_ctx {
   // compute workspace
   int maxC = 0;
   float *u = nullptr, *c = nullptr, *y = nullptr, *r = nullptr, *z = nullptr, *HL = nullptr;
+  // bf16 activations (TG_PREC_BF16): c, [LN(y) | h], z with row strides padded to 8
+  unsigned short *c_h = nullptr, *rh_h = nullptr, *z_h = nullptr;
+  int ld_ch = 0, ld_rh = 0, ld_z = 0;
   // counters / flags
   long long* cnt_total = nullptr;
   long long* cnt_sb = nullptr;  // [kMaxS x TG_NCOUNTERS]
@@ -68,6 +71,14 @@ struct tg_ctx {
   std::vector<cudaEvent_t> ev_pool;
   std::vector<int> ev_stage;
   size_t ev_used = 0;
+  // tg_gemm unit entry: device M and prepared-weight cache
+  int* gemm_m = nullptr;
+  struct GemmCacheEntry {
+    const float* B;
+    int N, K, prec;
+    TcWeights w;
+  };
+  std::vector<GemmCacheEntry> gemm_cache;
   // staging for host buffers
   void* stage = nullptr;
   size_t stage_bytes = 0;
@@ -221,6 +232,12 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   a.k = ctx->k;
   a.nc_dev = m_dev;
   a.nc_max = mmax;
+  const bool bfa = ctx->cfg.precision == TG_PREC_BF16;  // bf16 activations between the GEMMs
+  if (bfa) {
+    a.c = nullptr;
+    a.c_h = ctx->c_h;
+    a.ldc_h = ctx->ld_ch;
+  }
   {
     Prof pf(ctx, TG_ST_ATTN, st);
     launch_attn(a, st);
@@ -242,6 +259,10 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   g2.ldc = ctx->Dp;
   g2.m_dev = m_dev;
   g2.m_max = mmax;
+  if (bfa) {
+    g2.a_h = ctx->c_h;
+    g2.lda_h = ctx->ld_ch;
+  }
   {
     Prof pf(ctx, TG_ST_PROJ_V, st);
     if (tc) launch_gemm_tc(g2, w.tcF, ctx->cfg.precision, st);
@@ -250,8 +271,8 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   TRY(launched(ctx));
   {
     Prof pf(ctx, TG_ST_LNORM, st);
-    launch_layernorm(ctx->y, ctx->r, ctx->Dp, ctx->d_n, ctx->dnp, ctx->d_e, ctx->dep, ctx->d_t, w.lng, w.lnb, m_dev,
-                     mmax, st);
+    launch_layernorm(ctx->y, bfa ? nullptr : ctx->r, ctx->Dp, ctx->d_n, ctx->dnp, ctx->d_e, ctx->dep, ctx->d_t,
+                     w.lng, w.lnb, m_dev, mmax, lv.hs_row, bfa ? ctx->rh_h : nullptr, ctx->ld_rh, st);
   }
   TRY(launched(ctx));
   // G3: z = ReLU(W1 [r || h^(l-1)] + b1)  (Eq. 7)
@@ -269,6 +290,13 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   g3.ldc = ctx->dnp;
   g3.m_dev = m_dev;
   g3.m_max = mmax;
+  if (bfa) {
+    g3.a_h = ctx->rh_h;
+    g3.lda_h = ctx->ld_rh;
+    g3.C = nullptr;
+    g3.c_h = ctx->z_h;
+    g3.ldc_h = ctx->ld_z;
+  }
   {
     Prof pf(ctx, TG_ST_FFN1, st);
     if (tc) launch_gemm_tc(g3, w.tcW1, ctx->cfg.precision, st);
@@ -286,6 +314,10 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   g4.c_rows = lv.dst_row;
   g4.m_dev = m_dev;
   g4.m_max = mmax;
+  if (bfa) {
+    g4.a_h = ctx->z_h;
+    g4.lda_h = ctx->ld_z;
+  }
   {
     Prof pf(ctx, TG_ST_FFN2, st);
     if (tc) launch_gemm_tc(g4, w.tcW2, ctx->cfg.precision, st);
@@ -750,6 +782,14 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
   TRY(dalloc(ctx, &ctx->r, (size_t)maxC * Dp));
   TRY(dalloc(ctx, &ctx->z, (size_t)maxC * dnp));
   TRY(dalloc(ctx, &ctx->HL, (size_t)S * cap[L] * dnp));
+  if (cfg->precision == TG_PREC_BF16) {
+    ctx->ld_ch = (HDp + 7) & ~7;
+    ctx->ld_rh = (Dp + dnp + 7) & ~7;
+    ctx->ld_z = (dnp + 7) & ~7;
+    TRY(dalloc(ctx, &ctx->c_h, (size_t)maxC * ctx->ld_ch));
+    TRY(dalloc(ctx, &ctx->rh_h, (size_t)maxC * ctx->ld_rh));
+    TRY(dalloc(ctx, &ctx->z_h, (size_t)maxC * ctx->ld_z));
+  }
   TRY(dalloc(ctx, &ctx->cnt_total, TG_NCOUNTERS));
   TRY(dalloc(ctx, &ctx->cnt_sb, (size_t)kMaxS * TG_NCOUNTERS));
   CK(cudaMemset(ctx->cnt_sb, 0, (size_t)kMaxS * TG_NCOUNTERS * sizeof(long long)));
@@ -1006,9 +1046,8 @@ tg_status tg_gemm(tg_ctx* ctx, int32_t precision, int32_t M, int32_t N, int32_t 
   if (precision < TG_PREC_FP32 || precision > TG_PREC_LAST) return TG_EINVAL;
   cudaStream_t st = (cudaStream_t)cuda_stream;
   CK(cudaSetDevice(ctx->device));
-  int* mdev = nullptr;
-  CK(cudaMalloc(&mdev, sizeof(int)));
-  CK(cudaMemcpy(mdev, &M, sizeof(int), cudaMemcpyHostToDevice));
+  if (!ctx->gemm_m) TRY(dalloc(ctx, &ctx->gemm_m, 1));
+  launch_set_int(ctx->gemm_m, M, st);  // stream-ordered (device count as on the hot path)
   GemmArgs g{};
   g.a_base0 = A;
   g.lda0 = K;
@@ -1019,27 +1058,29 @@ tg_status tg_gemm(tg_ctx* ctx, int32_t precision, int32_t M, int32_t N, int32_t 
   g.relu = relu;
   g.C = C;
   g.ldc = N;
-  g.m_dev = mdev;
+  g.m_dev = ctx->gemm_m;
   g.m_max = std::max(M, 1);
-  tg_status s = TG_OK;
   if (precision == TG_PREC_FP32) {
     launch_gemm_simt(g, st);
   } else {
-    std::vector<void*> owned;
-    TcWeights w;
-    s = tc_prepare_weights(B, N, K, precision, &w, owned);
-    if (s == TG_OK) launch_gemm_tc(g, w, precision, st);
-    cudaStreamSynchronize(st);
-    for (void* p : owned) cudaFree(p);
+    // weights re-tiled once per (B, N, K, precision) and cached in the context
+    const TcWeights* w = nullptr;
+    for (auto& e : ctx->gemm_cache)
+      if (e.B == B && e.N == N && e.K == K && e.prec == precision) w = &e.w;
+    if (!w) {
+      tg_ctx::GemmCacheEntry e{B, N, K, precision, {}};
+      TRY(tc_prepare_weights(B, N, K, precision, &e.w, ctx->owned));
+      ctx->gemm_cache.push_back(e);
+      w = &ctx->gemm_cache.back().w;
+    }
+    launch_gemm_tc(g, *w, precision, st);
   }
   cudaError_t e = cudaGetLastError();
-  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
-  cudaFree(mdev);
   if (e != cudaSuccess) {
     fprintf(stderr, "libtg: tg_gemm %s\n", cudaGetErrorString(e));
     return TG_ECUDA;
   }
-  return s;
+  return TG_OK;  // stream-ordered; the caller synchronises
 }
 
 void tg_free(tg_ctx* ctx) {

@@ -169,6 +169,8 @@ struct AttnArgs {
   int dnp, dep, dtp, d_t, Dp, H, k;
   const int* nc_dev;
   int nc_max;
+  unsigned short* c_h;     // if non-null: c written as bf16 [nc x ldc_h] (zero padded) instead of fp32
+  int ldc_h;
 };
 void launch_attn(const AttnArgs& a, cudaStream_t st);
 
@@ -190,18 +192,29 @@ struct GemmArgs {
   const float* const* q_rows;
   int q_dnp, q_dep;
   const float* q_phi0;          // [dtp]
-  // output: dense C (ldc) or per-row destinations
+  // output: dense C (ldc) or per-row destinations (either may be null)
   float* C;
   int ldc;
   float* const* c_rows;
   const int* m_dev;
   int m_max;
+  // bf16 activation path (TG_PREC_BF16, tensor-core kernel only):
+  //   a_h  : dense bf16 A [M x lda_h] covering all K columns (zero padded to lda_h);
+  //          streamed into shared memory with cp.async instead of the row segments
+  //   c_h  : bf16 copy of the output [M x ldc_h], columns [N, ldc_h) written as 0
+  const unsigned short* a_h;
+  int lda_h;
+  unsigned short* c_h;
+  int ldc_h;
 };
 void launch_gemm_simt(const GemmArgs& g, cudaStream_t st);
 
 // LayerNorm over the true (unpadded) columns of each row (R1: eps 1e-5, biased var).
+// r (fp32 [M x Dp]) and/or rh (bf16 [M x ldrh] = [LN(y) | h^(l-1) | 0-pad], the
+// A operand of the merge FFN) are written when non-null.
 void launch_layernorm(const float* y, float* r, int Dp, int dn, int dnp, int de, int dep, int dt,
-                      const float* gamma, const float* beta, const int* m_dev, int m_max, cudaStream_t st);
+                      const float* gamma, const float* beta, const int* m_dev, int m_max,
+                      const float* const* hs_rows, unsigned short* rh, int ldrh, cudaStream_t st);
 
 // Scores p_e = sigmoid(MLP(h_src, h_dst)) (R10) for every edge of the superbatch:
 // row resolution, hidden layer as a projection GEMM, then the W_a2 head.
@@ -212,6 +225,8 @@ void launch_score_head(const float* z, int ldz, const long long* oidx, int M, co
 // out[i] = H_L[q(i)] for a single-batch embed call (DedupInvert, Alg. 1 l.20).
 void launch_invert(const float* HL, int ldh, LevelDev top, int n, int dn, float* out, cudaStream_t st);
 void launch_prep_nodes(const int32_t* nodes, const uint32_t* ts, int n, LevelDev top, cudaStream_t st);
+
+void launch_set_int(int* p, int v, cudaStream_t st);
 
 // fold the superbatch counter rows into the totals and the per-batch log
 void launch_finish(long long* cnt_sb, int S, long long* total, long long* log, int64_t log_row0,
