@@ -29,7 +29,7 @@ namespace tg {
 constexpr int TC_BM = 128;
 constexpr int TC_WARPS = 10;
 constexpr int TC_THREADS = TC_WARPS * 32;
-constexpr int TC_MAXSTAGES = 4;
+constexpr int TC_MAXSTAGES = 8;
 // TMEM: two accumulator buffers of 256 columns (all 512 columns; one CTA per
 // SM). Two CTAs per SM with 2 x 128 columns each was measured slower.
 __host__ __device__ constexpr int tc_acc_cols(int) { return 256; }
@@ -45,7 +45,7 @@ __host__ __device__ inline unsigned sw128(int r, int c) {
 
 static inline int tc_stages(int prec, int BN) {
   const size_t st = (size_t)tc_planes(prec) * ((size_t)TC_BM * 128 + (size_t)BN * 128);
-  const size_t budget = tc_ctas_per_sm(prec) == 1 ? 200 * 1024 : 108 * 1024;
+  const size_t budget = tc_ctas_per_sm(prec) == 1 ? 210 * 1024 : 108 * 1024;
   int s = (int)(budget / st);
   if (s > TC_MAXSTAGES) s = TC_MAXSTAGES;
   return s < 2 ? 2 : s;
@@ -217,7 +217,8 @@ __device__ __forceinline__ float4 tc_load4(const GemmArgs& g, const float* r0, c
 }
 
 template <int PREC>
-__global__ void __launch_bounds__(TC_THREADS, 1) k_gemm_tc(GemmArgs g, TcWeights w, int stages) {
+__global__ void __launch_bounds__(TC_THREADS, 1)
+    k_gemm_tc(GemmArgs g, TcWeights w, int stages, const __grid_constant__ CUtensorMap tmA, int a_tma) {
   constexpr int EPC = PREC == TG_PREC_BF16 ? 64 : 32;
   constexpr int PLANES = PREC == TG_PREC_TF32X3 ? 2 : 1;
   constexpr int NV = EPC / 4;  // float4 loads per row per k-block
@@ -240,7 +241,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1) k_gemm_tc(GemmArgs g, TcWeights
   const int nkb = w.nkb;
   if (tid == 0) {
     for (int s = 0; s < stages; ++s) {
-      mbar_init(&full[s], TC_BM + 1);  // 128 A rows + the B producer's expect_tx
+      mbar_init(&full[s], a_tma ? 1 : TC_BM + 1);  // (128 A rows +) the TMA producer's expect_tx
       mbar_init(&empty[s], 1);         // MMA commit
     }
     for (int a = 0; a < 2; ++a) {
@@ -259,7 +260,9 @@ __global__ void __launch_bounds__(TC_THREADS, 1) k_gemm_tc(GemmArgs g, TcWeights
   asm volatile("tcgen05.fence::after_thread_sync;\n");
   const uint32_t tmem = *tmem_slot;
 
-  if (warp < 4 && PREC == TG_PREC_TF32) {
+  if (warp < 4 && a_tma) {
+    // A arrives by TMA (issued by warp 4 with B): nothing to produce here
+  } else if (warp < 4 && PREC == TG_PREC_TF32) {
     // ===================== A producers, streamed: raw fp32 rows go straight into
     // the swizzled operand with 16-byte cp.async (zero-fill past K / M); the
     // tensor core reads them as tf32. Completion is tracked by the full barrier
@@ -391,7 +394,15 @@ __global__ void __launch_bounds__(TC_THREADS, 1) k_gemm_tc(GemmArgs g, TcWeights
           unsigned char* sB = smem + s * stage_bytes + PLANES * a_plane;
           const unsigned char* src =
               reinterpret_cast<const unsigned char*>(w.hi) + ((size_t)tn * nkb + kb) * PLANES * b_plane;
-          mbar_expect_tx(&full[s], PLANES * b_plane);
+          mbar_expect_tx(&full[s], PLANES * b_plane + (a_tma ? a_plane : 0u));
+          if (a_tma) {  // A tile [128 rows x 128 B] of the dense activation, 128B-swizzled by TMA
+            const int x = kb * EPC, y = (t / w.ntn) * TC_BM;
+            asm volatile(
+                "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], "
+                "[%4];\n" ::"r"(smem_u32(smem + s * stage_bytes)),
+                "l"(reinterpret_cast<uint64_t>(&tmA)), "r"(x), "r"(y), "r"(smem_u32(&full[s]))
+                : "memory");
+          }
           bulk_g2s(sB, src, PLANES * b_plane, &full[s]);
         }
       }
@@ -515,7 +526,26 @@ static size_t tc_smem(int prec, int BN, int stages) {
   return s;
 }
 
-void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaStream_t st) {
+tg_status tc_make_tensor_a(const void* base, int elem_bytes, int ld, int rows, TcTensorA* out) {
+  out->valid = 0;
+  if (!base || ld < 1 || rows < 1 || ((size_t)ld * elem_bytes) % 16) return TG_EINVAL;
+  cuuint64_t dims[2] = {(cuuint64_t)ld, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)ld * elem_bytes};
+  cuuint32_t box[2] = {(cuuint32_t)(128 / elem_bytes), (cuuint32_t)TC_BM};
+  cuuint32_t estr[2] = {1, 1};
+  const CUtensorMapDataType dt = elem_bytes == 2 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32;
+  CUresult r = cuTensorMapEncodeTiled(&out->map, dt, 2, const_cast<void*>(base), dims, strides, box, estr,
+                                      CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                                      CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return TG_ECUDA;
+  out->valid = 1;
+  return TG_OK;
+}
+
+void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaStream_t st, const TcTensorA* ta) {
+  static const CUtensorMap zero_map{};
+  const CUtensorMap& tm = (ta && ta->valid) ? ta->map : zero_map;
+  const int a_tma = (ta && ta->valid) ? 1 : 0;
   const int stages = tc_stages(precision, w.BN);
   const size_t smem = tc_smem(precision, w.BN, stages);
   const int tiles = ((g.m_max + TC_BM - 1) / TC_BM) * w.ntn;
@@ -528,21 +558,21 @@ void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaSt
       cudaFuncSetAttribute(k_gemm_tc<TG_PREC_BF16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       set = smem;
     }
-    k_gemm_tc<TG_PREC_BF16><<<grid, TC_THREADS, smem, st>>>(g, w, stages);
+    k_gemm_tc<TG_PREC_BF16><<<grid, TC_THREADS, smem, st>>>(g, w, stages, tm, a_tma);
   } else if (precision == TG_PREC_TF32) {
     static size_t set = 0;
     if (smem > set) {
       cudaFuncSetAttribute(k_gemm_tc<TG_PREC_TF32>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       set = smem;
     }
-    k_gemm_tc<TG_PREC_TF32><<<grid, TC_THREADS, smem, st>>>(g, w, stages);
+    k_gemm_tc<TG_PREC_TF32><<<grid, TC_THREADS, smem, st>>>(g, w, stages, tm, a_tma);
   } else {
     static size_t set = 0;
     if (smem > set) {
       cudaFuncSetAttribute(k_gemm_tc<TG_PREC_TF32X3>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       set = smem;
     }
-    k_gemm_tc<TG_PREC_TF32X3><<<grid, TC_THREADS, smem, st>>>(g, w, stages);
+    k_gemm_tc<TG_PREC_TF32X3><<<grid, TC_THREADS, smem, st>>>(g, w, stages, tm, 0);
   }
 }
 

@@ -61,6 +61,7 @@ struct tg_ctx {
   // bf16 activations (TG_PREC_BF16): c, [LN(y) | h], z with row strides padded to 8
   unsigned short *c_h = nullptr, *rh_h = nullptr, *z_h = nullptr;
   int ld_ch = 0, ld_rh = 0, ld_z = 0;
+  TcTensorA ta_c, ta_rh, ta_z;  // TMA tensor maps of the bf16 activations (dense GEMM A operands)
   // counters / flags
   long long* cnt_total = nullptr;
   long long* cnt_sb = nullptr;  // [kMaxS x TG_NCOUNTERS]
@@ -265,7 +266,7 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   }
   {
     Prof pf(ctx, TG_ST_PROJ_V, st);
-    if (tc) launch_gemm_tc(g2, w.tcF, ctx->cfg.precision, st);
+    if (tc) launch_gemm_tc(g2, w.tcF, ctx->cfg.precision, st, bfa ? &ctx->ta_c : nullptr);
     else launch_gemm_simt(g2, st);
   }
   TRY(launched(ctx));
@@ -299,7 +300,7 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   }
   {
     Prof pf(ctx, TG_ST_FFN1, st);
-    if (tc) launch_gemm_tc(g3, w.tcW1, ctx->cfg.precision, st);
+    if (tc) launch_gemm_tc(g3, w.tcW1, ctx->cfg.precision, st, bfa ? &ctx->ta_rh : nullptr);
     else launch_gemm_simt(g3, st);
   }
   TRY(launched(ctx));
@@ -320,7 +321,7 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   }
   {
     Prof pf(ctx, TG_ST_FFN2, st);
-    if (tc) launch_gemm_tc(g4, w.tcW2, ctx->cfg.precision, st);
+    if (tc) launch_gemm_tc(g4, w.tcW2, ctx->cfg.precision, st, bfa ? &ctx->ta_z : nullptr);
     else launch_gemm_simt(g4, st);
   }
   return launched(ctx);
@@ -789,6 +790,9 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     TRY(dalloc(ctx, &ctx->c_h, (size_t)maxC * ctx->ld_ch));
     TRY(dalloc(ctx, &ctx->rh_h, (size_t)maxC * ctx->ld_rh));
     TRY(dalloc(ctx, &ctx->z_h, (size_t)maxC * ctx->ld_z));
+    TRY(tc_make_tensor_a(ctx->c_h, 2, ctx->ld_ch, maxC, &ctx->ta_c));
+    TRY(tc_make_tensor_a(ctx->rh_h, 2, ctx->ld_rh, maxC, &ctx->ta_rh));
+    TRY(tc_make_tensor_a(ctx->z_h, 2, ctx->ld_z, maxC, &ctx->ta_z));
   }
   TRY(dalloc(ctx, &ctx->cnt_total, TG_NCOUNTERS));
   TRY(dalloc(ctx, &ctx->cnt_sb, (size_t)kMaxS * TG_NCOUNTERS));
@@ -1073,7 +1077,9 @@ tg_status tg_gemm(tg_ctx* ctx, int32_t precision, int32_t M, int32_t N, int32_t 
       ctx->gemm_cache.push_back(e);
       w = &ctx->gemm_cache.back().w;
     }
-    launch_gemm_tc(g, *w, precision, st);
+    TcTensorA ta;  // dense fp32 A via TMA in the one-pass tf32 mode
+    if (precision == TG_PREC_TF32 && M > 0) TRY(tc_make_tensor_a(A, 4, K, M, &ta));
+    launch_gemm_tc(g, *w, precision, st, ta.valid ? &ta : nullptr);
   }
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) {

@@ -1,5 +1,7 @@
 // tcgen05 tensor-core GEMM for the dense per-target projections (sm_100a).
 #pragma once
+#include <cuda.h>
+
 #include <vector>
 
 #include "tg_internal.cuh"
@@ -17,8 +19,20 @@ struct TcWeights {
   int nkb = 0;             // K blocks of 128 bytes
 };
 
+// Dense A operand loaded by TMA tensor copies (cp.async.bulk.tensor.2d, 128B
+// swizzle, box = 128 rows x 128 bytes) instead of per-thread loads.
+struct TcTensorA {
+  CUtensorMap map;
+  int valid = 0;
+};
+// base: dense row-major [rows x ld] of 2-byte (bf16) or 4-byte (fp32) elements; ld*elem % 16 == 0.
+tg_status tc_make_tensor_a(const void* base, int elem_bytes, int ld, int rows, TcTensorA* out);
+
 tg_status tc_prepare_weights(const float* W, int N, int K, int precision, TcWeights* out,
                              std::vector<void*>& owned);
-void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaStream_t st);
+// ta (optional): the A operand as a tensor map (must match the element type of
+// the precision: bf16 for TG_PREC_BF16, fp32 for TG_PREC_TF32).
+void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaStream_t st,
+                    const TcTensorA* ta = nullptr);
 
 }  // namespace tg

@@ -1,0 +1,31 @@
+"""GEMM time vs M (tiles in flight) for the G2 shape: latency- vs bandwidth-bound probe."""
+import os
+import sys
+
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+from synth import make_stream, make_params  # noqa: E402
+from paper_conf_ppopp_wangm23_b200 import Context  # noqa: E402
+
+s = make_stream("tiny")
+ctx = Context.from_stream(s).load_model(make_params(2, 2, s.d_n, s.d_e), n_neighbors=3, max_batch_targets=16,
+                                        cache_limit=100, time_window=10)
+N, K = 516, 1032
+B = torch.randn(N, K, device="cuda") / K ** 0.5
+for prec in (3, 2):
+    for M in (128, 1280, 2560, 5120, 6400, 12800, 25600):
+        A = torch.randn(M, K, device="cuda")
+        C = torch.zeros(M, N, device="cuda")
+        ctx.gemm(A, B, C, precision=prec)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        reps = 10
+        e0.record()
+        for _ in range(reps):
+            ctx.gemm(A, B, C, precision=prec)
+        e1.record()
+        torch.cuda.synchronize()
+        us = 1e3 * e0.elapsed_time(e1) / reps
+        tiles = ((M + 127) // 128) * 3
+        print(f"prec {prec} M {M:6d} tiles {tiles:4d}  {us:8.1f} us  {2 * M * N * K / us / 1e6:7.1f} TFLOP/s", flush=True)
