@@ -1,6 +1,9 @@
 """Build libtg.so in-tree with nvcc for sm_100a (no JIT cache, no torch extension).
 
     python -m paper_conf_ppopp_wangm23_b200.build [--force]
+
+TG_TRACE=1 builds the debug variant libtg_trace.so (GEMM clock64 trace, see
+k_gemm_tc.cu; loaded only when TG_LIB points at it, e.g. by tools/gemm_trace.py).
 """
 import concurrent.futures as cf
 import os
@@ -10,11 +13,15 @@ import sys
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
-LIB = os.path.join(PKG, "libtg.so")
+TRACE = os.environ.get("TG_TRACE") == "1"
+LIB = os.path.join(PKG, "libtg_trace.so" if TRACE else "libtg.so")
+BUILD = os.path.join(CSRC, "build_trace" if TRACE else "build")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xptxas", "-v",
          "--expt-relaxed-constexpr", "-I", os.path.join(ROOT, "include")]
+if TRACE:
+    FLAGS.append("-DTG_TC_TRACE")
 # NOTE: no --use_fast_math: Eq. 8 needs the accurate cosf and uncontracted mul/add (R5).
 
 
@@ -31,7 +38,7 @@ def _stale():
 
 
 def _compile(src, log):
-    obj = os.path.join(CSRC, "build", os.path.basename(src)[:-3] + ".o")
+    obj = os.path.join(BUILD, os.path.basename(src)[:-3] + ".o")
     cmd = [NVCC, *ARCH, *FLAGS, "-c", src, "-o", obj]
     r = subprocess.run(cmd, capture_output=True, text=True)
     with open(log, "a") as f:
@@ -44,8 +51,8 @@ def _compile(src, log):
 def build(force=False, verbose=False):
     if not force and not _stale():
         return LIB
-    os.makedirs(os.path.join(CSRC, "build"), exist_ok=True)
-    log = os.path.join(CSRC, "build", "ptxas.log")
+    os.makedirs(BUILD, exist_ok=True)
+    log = os.path.join(BUILD, "ptxas.log")
     open(log, "w").close()
     with cf.ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 1)) as ex:
         objs = list(ex.map(lambda s: _compile(s, log), sources()))

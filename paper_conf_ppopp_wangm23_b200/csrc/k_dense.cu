@@ -77,11 +77,6 @@ __global__ void __launch_bounds__(256) k_gemm_simt(GemmArgs g) {
       for (int j = 0; j < 4; ++j) {
         float x = acc[i][j];
         if (g.bias) x += g.bias[c + j];
-        if (g.q_rows) {
-          const int cc = c + j;
-          if (cc < g.q_dnp) x += g.q_rows[r][cc];
-          else if (cc >= g.q_dnp + g.q_dep) x += g.q_phi0[cc - g.q_dnp - g.q_dep];
-        }
         if (g.relu) x = fmaxf(x, 0.f);
         v[j] = x;
       }
@@ -102,7 +97,7 @@ void launch_gemm_simt(const GemmArgs& g, cudaStream_t st) {
 __global__ void k_layernorm(const float* __restrict__ y, float* __restrict__ r, int Dp, int dn, int dnp, int de,
                             int dep, int dt, const float* __restrict__ gamma, const float* __restrict__ beta,
                             const int* __restrict__ m_dev, const float* const* __restrict__ hs_rows,
-                            unsigned short* __restrict__ rh, int ldrh) {
+                            const float* __restrict__ phi0, unsigned short* __restrict__ rh, int ldrh) {
   const int M = *m_dev;
   const int lane = threadIdx.x & 31;
   const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, nw = (gridDim.x * blockDim.x) >> 5;
@@ -112,6 +107,8 @@ __global__ void k_layernorm(const float* __restrict__ y, float* __restrict__ r, 
   // warp per row; the row (<= 1024 floats) is read once into registers
   for (int row = warp; row < M; row += nw) {
     const float4* yr = reinterpret_cast<const float4*>(y + (size_t)row * Dp);
+    const float4* hr = reinterpret_cast<const float4*>(hs_rows[row]);
+    const float4* p0 = reinterpret_cast<const float4*>(phi0);
     float4* rr = r ? reinterpret_cast<float4*>(r + (size_t)row * Dp) : nullptr;
     float4 v[8];
     float sum = 0.f;
@@ -121,6 +118,14 @@ __global__ void k_layernorm(const float* __restrict__ y, float* __restrict__ r, 
       v[j] = make_float4(0.f, 0.f, 0.f, 0.f);
       if (q < D4) {
         v[j] = yr[q];
+        // + q = [h^(l-1) || 0 || Phi(0)] (padded columns of each part are zero)
+        float4 a = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (4 * q < dnp) a = hr[q];
+        else if (4 * q >= s2) a = p0[q - (s2 >> 2)];
+        v[j].x += a.x;
+        v[j].y += a.y;
+        v[j].z += a.z;
+        v[j].w += a.w;
         // padded columns are exact zeros (zero weight rows / bias), so they do not bias the sum
         sum += (v[j].x + v[j].y) + (v[j].z + v[j].w);
       }
@@ -169,7 +174,6 @@ __global__ void k_layernorm(const float* __restrict__ y, float* __restrict__ r, 
       }
     }
     if (rh) {  // [LN(y) | h^(l-1) | 0]: the merge-FFN input (Eq. 7) as one bf16 row
-      const float4* hr = reinterpret_cast<const float4*>(hs_rows[row]);
       for (int q = lane; 4 * q < ldrh - Dp; q += 32) {
         float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
         if (4 * q < dnp) x = hr[q];
@@ -185,11 +189,13 @@ __global__ void k_layernorm(const float* __restrict__ y, float* __restrict__ r, 
 
 void launch_layernorm(const float* y, float* r, int Dp, int dn, int dnp, int de, int dep, int dt,
                       const float* gamma, const float* beta, const int* m_dev, int m_max,
-                      const float* const* hs_rows, unsigned short* rh, int ldrh, cudaStream_t st) {
+                      const float* const* hs_rows, const float* phi0, unsigned short* rh, int ldrh,
+                      cudaStream_t st) {
   int blocks = (m_max * 32 + 255) / 256;
   if (blocks < 1) blocks = 1;
   if (blocks > 1184) blocks = 1184;
-  k_layernorm<<<blocks, 256, 0, st>>>(y, r, Dp, dn, dnp, de, dep, dt, gamma, beta, m_dev, hs_rows, rh, ldrh);
+  k_layernorm<<<blocks, 256, 0, st>>>(y, r, Dp, dn, dnp, de, dep, dt, gamma, beta, m_dev, hs_rows, phi0, rh,
+                                      ldrh);
 }
 
 // -------------------------------------------------------------------- score

@@ -10,9 +10,11 @@
 //              mbarrier complete_tx) of the pre-tiled weight images;
 //   warp 5     MMA issuer: one lane issues tcgen05.mma (M = 128, N = BN) into a
 //              double-buffered TMEM accumulator and commits to mbarriers;
-//   warps 6-9  epilogue: tcgen05.ld (32x32b) -> bias / attention residual q /
-//              ReLU -> row store (dense or gathered destinations).
-// STAGES shared-memory stages (3-4) decouple the producers from the tensor core.
+//   warps 6-13 epilogue, two warps per TMEM lane quadrant splitting the
+//              columns: tcgen05.ld (32x32b) -> per-warp shared transpose ->
+//              bias / ReLU on float4 -> coalesced row stores (dense or
+//              gathered destinations, fp32 and/or bf16).
+// `stages` shared-memory stages decouple the producers from the tensor core.
 //
 // TG_PREC_TF32X3: kind::tf32 with the 3-term split a.b ~ ah.bh + ah.bl + al.bh
 // (ah = rna_tf32(a), al = rna_tf32(a - ah)): fp32-level accuracy on tensor
@@ -27,7 +29,8 @@
 namespace tg {
 
 constexpr int TC_BM = 128;
-constexpr int TC_WARPS = 10;
+constexpr int TC_WARPS = 14;
+constexpr int TC_EPI_WARPS = 8;
 constexpr int TC_THREADS = TC_WARPS * 32;
 constexpr int TC_MAXSTAGES = 8;
 // TMEM: two accumulator buffers of 256 columns (all 512 columns; one CTA per
@@ -43,9 +46,15 @@ __host__ __device__ inline unsigned sw128(int r, int c) {
   return (unsigned)((r >> 3) * 1024 + (r & 7) * 128 + ((c ^ (r & 7)) << 4));
 }
 
+// shared memory after the stages: barriers, then a 32 x 16 fp32 transpose
+// buffer per epilogue warp
+constexpr int TC_BAR_BYTES = 256;
+constexpr int TC_STG_LD = 20;  // floats per staged row (16 columns + pad)
+constexpr int TC_EPI_BYTES = TC_EPI_WARPS * 32 * TC_STG_LD * 4;
+
 static inline int tc_stages(int prec, int BN) {
   const size_t st = (size_t)tc_planes(prec) * ((size_t)TC_BM * 128 + (size_t)BN * 128);
-  const size_t budget = tc_ctas_per_sm(prec) == 1 ? 210 * 1024 : 108 * 1024;
+  const size_t budget = tc_ctas_per_sm(prec) == 1 ? 205 * 1024 : 100 * 1024;
   int s = (int)(budget / st);
   if (s > TC_MAXSTAGES) s = TC_MAXSTAGES;
   return s < 2 ? 2 : s;
@@ -216,6 +225,30 @@ __device__ __forceinline__ float4 tc_load4(const GemmArgs& g, const float* r0, c
   return *reinterpret_cast<const float4*>(p);
 }
 
+#ifdef TG_TC_TRACE
+// Debug build only (build.py TG_TRACE=1 -> libtg_trace.so): clock64 stamps of the
+// first tile of each CTA for launches whose (N, K) matches the armed shape.
+constexpr int TCT_N = 64;
+__device__ long long tg_tct[148][TCT_N];
+__device__ int tg_tct_nk[3];  // N, K, (unused)
+#define TCT(i, v)                                                                              \
+  do {                                                                                         \
+    if (tct_on && blockIdx.x < 148 && (i) < TCT_N) tg_tct[blockIdx.x][(i)] = (long long)(v); \
+  } while (0)
+#else
+#define TCT(i, v) \
+  do {            \
+  } while (0)
+#endif
+
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t* v) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];\n"
+      : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]), "=r"(v[8]),
+        "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
+      : "r"(taddr));
+}
+
 template <int PREC>
 __global__ void __launch_bounds__(TC_THREADS, 1)
     k_gemm_tc(GemmArgs g, TcWeights w, int stages, const __grid_constant__ CUtensorMap tmA, int a_tma) {
@@ -223,7 +256,9 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   constexpr int PLANES = PREC == TG_PREC_TF32X3 ? 2 : 1;
   constexpr int NV = EPC / 4;  // float4 loads per row per k-block
   extern __shared__ __align__(1024) unsigned char smem_raw[];
-  unsigned char* smem = (unsigned char*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  // 1024-byte alignment (128B swizzle atoms) by an integer offset from smem_raw, so
+  // the compiler keeps the shared address space (LDS/STS, not generic LD/ST)
+  unsigned char* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   const int BN = w.BN;
   const uint32_t a_plane = TC_BM * 128;
   const uint32_t b_plane = (uint32_t)BN * 128;
@@ -234,10 +269,24 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   uint64_t* tempty = tfull + 2;             // [2]
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+#ifdef TG_TC_TRACE
+  const long long t_entry = clock64();
+#endif
   const int M = *g.m_dev;
   const int tiles_m = (M + TC_BM - 1) / TC_BM;
   const int ntiles = tiles_m * w.ntn;
   if ((int)blockIdx.x >= ntiles) return;
+#ifdef TG_TC_TRACE
+  // only full-grid launches are traced (a later partial launch would leave stale stamps)
+  const bool tct_on = tg_tct_nk[0] == g.N && tg_tct_nk[1] == g.K && ntiles >= (int)gridDim.x;
+  if (tid == 0) {
+    long long gt;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt));
+    TCT(0, t_entry);
+    TCT(1, gt);
+    TCT(63, M);
+  }
+#endif
   const int nkb = w.nkb;
   if (tid == 0) {
     for (int s = 0; s < stages; ++s) {
@@ -246,7 +295,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     }
     for (int a = 0; a < 2; ++a) {
       mbar_init(&tfull[a], 1);     // MMA commit after the tile's last k-block
-      mbar_init(&tempty[a], 128);  // epilogue threads drained the accumulator
+      mbar_init(&tempty[a], TC_EPI_WARPS * 32);  // epilogue threads drained the accumulator
     }
     asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
   }
@@ -259,6 +308,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;\n");
   const uint32_t tmem = *tmem_slot;
+  if (tid == 0) TCT(2, clock64());
 
   if (warp < 4 && a_tma) {
     // A arrives by TMA (issued by warp 4 with B): nothing to produce here
@@ -394,6 +444,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           unsigned char* sB = smem + s * stage_bytes + PLANES * a_plane;
           const unsigned char* src =
               reinterpret_cast<const unsigned char*>(w.hi) + ((size_t)tn * nkb + kb) * PLANES * b_plane;
+          if (gk == 0) TCT(4, clock64());
           mbar_expect_tx(&full[s], PLANES * b_plane + (a_tma ? a_plane : 0u));
           if (a_tma) {  // A tile [128 rows x 128 B] of the dense activation, 128B-swizzled by TMA
             const int x = kb * EPC, y = (t / w.ntn) * TC_BM;
@@ -420,6 +471,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         for (int kb = 0; kb < nkb; ++kb, ++gk) {
           const int s = gk % stages;
           mbar_wait(&full[s], (gk / stages) & 1);
+          if (tc == 0) TCT(8 + kb, clock64());
           asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");  // cp.async A -> tensor core
           asm volatile("tcgen05.fence::after_thread_sync;\n");
           const uint32_t aH = smem_u32(smem + s * stage_bytes);
@@ -440,85 +492,109 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n" ::"r"(
                          smem_u32(&tfull[acc]))
                      : "memory");
+        if (tc == 0) TCT(3, clock64());
       }
     }
   } else {
-    // ===================== epilogue (warps 6-9 cover TMEM lane quadrants 2,3,0,1)
+    // ===================== epilogue: warps 6-13; warp w reads TMEM lane quadrant
+    // w % 4 (rows 32*(w%4) ..), the two warps of a quadrant take alternate
+    // 16-column chunks. tcgen05.ld leaves one row per thread, so each chunk is
+    // transposed through a per-warp shared buffer (row stride 20 floats: 16B
+    // aligned, conflict-free STS.128) and written back with lanes = 4 columns x
+    // 8 rows: float4 bias/ReLU and 64-byte coalesced row segments.
     const int quad = warp & 3;
-    const int et = tid - 6 * 32;  // 0..127
-    (void)et;
+    const int ew = warp - 6;               // 0..7
+    const int half = ew >> 2;              // which alternate chunk
+    float* stg = reinterpret_cast<float*>(smem + stages * stage_bytes + TC_BAR_BYTES) + ew * (32 * TC_STG_LD);
+    const int rq = lane >> 2, cq = lane & 3;  // read-back: row rq + 8i, float4 column cq
     uint32_t tc = 0;
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++tc) {
       const int tm = t / w.ntn, tn = t - tm * w.ntn;
       const int m0 = tm * TC_BM, n0 = tn * BN;
       const uint32_t acc = tc & 1;
-      mbar_wait(&tfull[acc], (tc >> 1) & 1);
-      asm volatile("tcgen05.fence::after_thread_sync;\n");
-      const int er = m0 + quad * 32 + lane;  // TMEM lane = row of the tile
+      const int er = m0 + quad * 32 + lane;
       float* orow = nullptr;
-      const float* qrow = nullptr;
       unsigned short* hrow = nullptr;
       if (er < M) {
         if (g.c_rows) orow = g.c_rows[er];
         else if (g.C) orow = g.C + (size_t)er * g.ldc;
-        qrow = g.q_rows ? g.q_rows[er] : nullptr;
         if (g.c_h) hrow = g.c_h + (size_t)er * g.ldc_h;
       }
-      for (int c0 = 0; c0 < BN; c0 += 16) {
+      mbar_wait(&tfull[acc], (tc >> 1) & 1);
+      if (tc == 0 && warp == 6 && lane == 0) TCT(5, clock64());
+      asm volatile("tcgen05.fence::after_thread_sync;\n");
+      bool released = false;
+      for (int c0 = 16 * half; c0 < BN; c0 += 32) {
         uint32_t v[16];
-        const uint32_t taddr = tmem + acc * tc_acc_cols(PREC) + ((uint32_t)(quad * 32) << 16) + (uint32_t)c0;
-        asm volatile(
-            "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, "
-            "[%16];\n"
-            : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
-              "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
-            : "r"(taddr));
+        tmem_ld16(tmem + acc * tc_acc_cols(PREC) + ((uint32_t)(quad * 32) << 16) + (uint32_t)c0, v);
         asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
-        if (orow || hrow) {
+        if (c0 + 32 >= BN) {  // this warp's last chunk: hand the accumulator back
+          asm volatile("tcgen05.fence::before_thread_sync;\n");
+          mbar_arrive(&tempty[acc]);
+          released = true;
+        }
 #pragma unroll
-          for (int j4 = 0; j4 < 4; ++j4) {
-            const int c = n0 + c0 + 4 * j4;
-            if (c < g.N) {
-              float o[4];
+        for (int j = 0; j < 4; ++j)
+          *reinterpret_cast<float4*>(stg + lane * TC_STG_LD + 4 * j) =
+              make_float4(__uint_as_float(v[4 * j]), __uint_as_float(v[4 * j + 1]), __uint_as_float(v[4 * j + 2]),
+                          __uint_as_float(v[4 * j + 3]));
+        __syncwarp();
+        const int cl = c0 + 4 * cq;  // first of this lane's 4 columns inside the tile
+        const int c = n0 + cl;
+        const bool cin = cl < BN && c < g.N;                    // N % 4 == 0: all 4 or none
+        const bool cpad = cl < BN && c >= g.N && c < g.ldc_h;  // bf16 zero padding [N, ldc_h)
+        float4 b4 = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (cin && g.bias) b4 = *reinterpret_cast<const float4*>(g.bias + c);
 #pragma unroll
-              for (int j = 0; j < 4; ++j) {
-                float x = __uint_as_float(v[4 * j4 + j]);
-                const int cc = c + j;
-                if (g.bias) x += g.bias[cc];
-                if (qrow) {
-                  if (cc < g.q_dnp) x += qrow[cc];
-                  else if (cc >= g.q_dnp + g.q_dep) x += g.q_phi0[cc - g.q_dnp - g.q_dep];
-                }
-                if (g.relu) x = fmaxf(x, 0.f);
-                o[j] = x;
-              }
-              if (orow) *reinterpret_cast<float4*>(orow + c) = make_float4(o[0], o[1], o[2], o[3]);
-              if (hrow) {  // bf16 activation for the next projection (N % 4 == 0)
-                __nv_bfloat162 lo = __floats2bfloat162_rn(o[0], o[1]), hi = __floats2bfloat162_rn(o[2], o[3]);
-                uint2 pk;
-                pk.x = *reinterpret_cast<uint32_t*>(&lo);
-                pk.y = *reinterpret_cast<uint32_t*>(&hi);
-                *reinterpret_cast<uint2*>(hrow + c) = pk;
-              }
-            } else if (hrow && c < g.ldc_h) {  // zero padding [N, ldc_h)
-              *reinterpret_cast<uint2*>(hrow + c) = make_uint2(0u, 0u);
+        for (int i = 0; i < 4; ++i) {
+          const int r = rq + 8 * i;
+          float4 x = *reinterpret_cast<const float4*>(stg + r * TC_STG_LD + 4 * cq);
+          x.x += b4.x;
+          x.y += b4.y;
+          x.z += b4.z;
+          x.w += b4.w;
+          if (g.relu) {
+            x.x = fmaxf(x.x, 0.f);
+            x.y = fmaxf(x.y, 0.f);
+            x.z = fmaxf(x.z, 0.f);
+            x.w = fmaxf(x.w, 0.f);
+          }
+          float* orr = reinterpret_cast<float*>(__shfl_sync(0xffffffffu, reinterpret_cast<long long>(orow), r));
+          if (orr && cin) *reinterpret_cast<float4*>(orr + c) = x;
+          if (g.c_h) {
+            unsigned short* hr =
+                reinterpret_cast<unsigned short*>(__shfl_sync(0xffffffffu, reinterpret_cast<long long>(hrow), r));
+            if (hr && (cin || cpad)) {
+              if (!cin) x = make_float4(0.f, 0.f, 0.f, 0.f);
+              __nv_bfloat162 lo = __floats2bfloat162_rn(x.x, x.y), hi = __floats2bfloat162_rn(x.z, x.w);
+              uint2 pk;
+              pk.x = *reinterpret_cast<uint32_t*>(&lo);
+              pk.y = *reinterpret_cast<uint32_t*>(&hi);
+              *reinterpret_cast<uint2*>(hr + c) = pk;
             }
           }
         }
+        __syncwarp();
       }
-      asm volatile("tcgen05.fence::before_thread_sync;\n");
-      mbar_arrive(&tempty[acc]);
+      if (!released) {  // no chunk for this warp (BN <= 16)
+        asm volatile("tcgen05.fence::before_thread_sync;\n");
+        mbar_arrive(&tempty[acc]);
+      }
+      if (tc == 0 && warp == 6 && lane == 0) TCT(6, clock64());
     }
   }
+  if (lane == 0 && warp >= 4 && warp <= 6) TCT(56 + warp, clock64());  // role done (before the barrier)
   asm volatile("tcgen05.fence::before_thread_sync;\n");
   __syncthreads();
+  if (tid == 0) TCT(7, clock64());
+  if (tid == 6 * 32) TCT(55, clock64());
   asm volatile("tcgen05.fence::after_thread_sync;\n");
   if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;\n" ::"r"(tmem), "r"(2 * tc_acc_cols(PREC)));
 }
 
 static size_t tc_smem(int prec, int BN, int stages) {
   const size_t planes = tc_planes(prec);
-  size_t s = 1024 + (size_t)stages * planes * ((size_t)TC_BM * 128 + (size_t)BN * 128) + 256;
+  size_t s = 1024 + (size_t)stages * planes * ((size_t)TC_BM * 128 + (size_t)BN * 128) + TC_BAR_BYTES + TC_EPI_BYTES;
   // tf32x3: one CTA per SM (it allocates all 512 TMEM columns; a second
   // co-resident CTA would block in tcgen05.alloc until the first one exits).
   const size_t one_per_sm = 120 * 1024;
@@ -575,5 +651,15 @@ void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaSt
     k_gemm_tc<TG_PREC_TF32X3><<<grid, TC_THREADS, smem, st>>>(g, w, stages, tm, 0);
   }
 }
+
+#ifdef TG_TC_TRACE
+extern "C" int tg_debug_tc_trace(int arm_n, int arm_k, int mode, long long* host) {
+  if (host) return (int)cudaMemcpyFromSymbol(host, tg_tct, sizeof(tg_tct));
+  int nk[3] = {arm_n, arm_k, mode};
+  static long long zero[148][TCT_N] = {};
+  cudaMemcpyToSymbol(tg_tct, zero, sizeof(zero));
+  return (int)cudaMemcpyToSymbol(tg_tct_nk, nk, sizeof(nk));
+}
+#endif
 
 }  // namespace tg

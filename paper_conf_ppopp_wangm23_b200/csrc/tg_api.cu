@@ -244,7 +244,7 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
     launch_attn(a, st);
   }
   TRY(launched(ctx));
-  // G2: y = F c + b_fc + q  (W_v and W_fc folded; residual q of Eq. 4)
+  // G2: y = F c + b_fc  (W_v and W_fc folded; the residual q of Eq. 4 is added by the LayerNorm)
   GemmArgs g2{};
   g2.a_base0 = ctx->c;
   g2.lda0 = HDp;
@@ -252,10 +252,6 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   g2.B = w.F;
   g2.N = ctx->Dp;
   g2.bias = w.bfc;
-  g2.q_rows = lv.hs_row;
-  g2.q_dnp = ctx->dnp;
-  g2.q_dep = ctx->dep;
-  g2.q_phi0 = ctx->table;  // Phi(0): row 0 of the table
   g2.C = ctx->y;
   g2.ldc = ctx->Dp;
   g2.m_dev = m_dev;
@@ -273,7 +269,8 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   {
     Prof pf(ctx, TG_ST_LNORM, st);
     launch_layernorm(ctx->y, bfa ? nullptr : ctx->r, ctx->Dp, ctx->d_n, ctx->dnp, ctx->d_e, ctx->dep, ctx->d_t,
-                     w.lng, w.lnb, m_dev, mmax, lv.hs_row, bfa ? ctx->rh_h : nullptr, ctx->ld_rh, st);
+                     w.lng, w.lnb, m_dev, mmax, lv.hs_row, ctx->table /* Phi(0): row 0 */,
+                     bfa ? ctx->rh_h : nullptr, ctx->ld_rh, st);
   }
   TRY(launched(ctx));
   // G3: z = ReLU(W1 [r || h^(l-1)] + b1)  (Eq. 7)

@@ -188,10 +188,6 @@ struct GemmArgs {
   int N, K;
   const float* bias;            // [N] or null
   int relu;
-  // residual q = [hs || 0 || Phi0] added in the epilogue (G2), if q_rows != null
-  const float* const* q_rows;
-  int q_dnp, q_dep;
-  const float* q_phi0;          // [dtp]
   // output: dense C (ldc) or per-row destinations (either may be null)
   float* C;
   int ldc;
@@ -209,12 +205,15 @@ struct GemmArgs {
 };
 void launch_gemm_simt(const GemmArgs& g, cudaStream_t st);
 
-// LayerNorm over the true (unpadded) columns of each row (R1: eps 1e-5, biased var).
-// r (fp32 [M x Dp]) and/or rh (bf16 [M x ldrh] = [LN(y) | h^(l-1) | 0-pad], the
-// A operand of the merge FFN) are written when non-null.
+// LayerNorm over the true (unpadded) columns of each row (R1: eps 1e-5, biased var)
+// of y + q, with the attention residual q = [h^(l-1) || 0 || Phi(0)] (Eq. 4)
+// added on load (y = F c + b_fc comes from G2). r (fp32 [M x Dp]) and/or rh
+// (bf16 [M x ldrh] = [LN(y+q) | h^(l-1) | 0-pad], the A operand of the merge
+// FFN) are written when non-null.
 void launch_layernorm(const float* y, float* r, int Dp, int dn, int dnp, int de, int dep, int dt,
                       const float* gamma, const float* beta, const int* m_dev, int m_max,
-                      const float* const* hs_rows, unsigned short* rh, int ldrh, cudaStream_t st);
+                      const float* const* hs_rows, const float* phi0, unsigned short* rh, int ldrh,
+                      cudaStream_t st);
 
 // Scores p_e = sigmoid(MLP(h_src, h_dst)) (R10) for every edge of the superbatch:
 // row resolution, hidden layer as a projection GEMM, then the W_a2 head.
