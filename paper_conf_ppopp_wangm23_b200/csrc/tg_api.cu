@@ -49,8 +49,11 @@ struct tg_ctx {
   long long* sc_oidx = nullptr;
   float* sc_z = nullptr;
   int* sc_m = nullptr;
-  // recursion levels (index l = 1..L), caches for l = 1..L-1
-  LevelDev lv[TG_MAX_LAYERS + 1]{};
+  // recursion levels (index l = 1..L), caches for l = 1..L-1. Two sets: the
+  // front half of superbatch i+1 (dedup, lookup, sampling, resolve) fills one
+  // set on the front stream while the layers of superbatch i read the other.
+  LevelDev lvs[2][TG_MAX_LAYERS + 1]{};
+  LevelDev* lv = lvs[0];
   int cap[TG_MAX_LAYERS + 1]{};
   CacheDev cache[TG_MAX_LAYERS]{};
   long long* cache_state = nullptr;
@@ -64,7 +67,11 @@ struct tg_ctx {
   TcTensorA ta_c, ta_rh, ta_z;  // TMA tensor maps of the bf16 activations (dense GEMM A operands)
   // counters / flags
   long long* cnt_total = nullptr;
-  long long* cnt_sb = nullptr;  // [kMaxS x TG_NCOUNTERS]
+  long long* cnt_sb = nullptr;  // [kMaxS x TG_NCOUNTERS] of the current set
+  long long* cnt_sbs[2] = {nullptr, nullptr};
+  // front stream + events of the two-set pipeline (stream_edges)
+  cudaStream_t fst = nullptr;
+  cudaEvent_t ev_front[2] = {nullptr, nullptr}, ev_back[2] = {nullptr, nullptr}, ev_in = nullptr, ev_fend = nullptr;
   int* err = nullptr;
   int64_t launches = 0;
   // per-stage profiling (events around launches)
@@ -328,7 +335,14 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
 // Embed(L, .) for S batches (Alg. 1): edge_mode -> batches of the stream
 // (targets src || dst), else one batch of explicit targets (prepared in lv[L]).
 // ------------------------------------------------------------------------
-tg_status run_superbatch(tg_ctx* ctx, int S, bool edge_mode, const EdgeSrc& es, int n_max_top, cudaStream_t st) {
+void select_set(tg_ctx* ctx, int s) {
+  ctx->lv = ctx->lvs[s];
+  ctx->cnt_sb = ctx->cnt_sbs[s];
+}
+
+// Top-down half (Alg. 1 l.5-12) and row resolution: reads only the inputs, the
+// graph and the cache index, writes the current level set.
+tg_status run_front(tg_ctx* ctx, int S, bool edge_mode, const EdgeSrc& es, int n_max_top, cudaStream_t st) {
   const int L = ctx->L, k = ctx->k;
   const bool dedup = ctx->cfg.opts & TG_OPT_DEDUP;
   const bool cache_on = ctx->cfg.opts & TG_OPT_CACHE;
@@ -382,10 +396,18 @@ tg_status run_superbatch(tg_ctx* ctx, int S, bool edge_mode, const EdgeSrc& es, 
     Prof pf(ctx, TG_ST_RESOLVE, st);
     launch_resolve(ra, ctx->err, st);
   }
-  TRY(launched(ctx));
-  // ---- bottom-up (Alg. 1 l.13-18): M and FFN, layer by layer over all S batches
-  for (int l = 1; l <= L; ++l) TRY(run_layer(ctx, l, st));
+  return launched(ctx);
+}
+
+// Bottom-up half (Alg. 1 l.13-18): M and FFN, layer by layer over all S batches.
+tg_status run_back(tg_ctx* ctx, cudaStream_t st) {
+  for (int l = 1; l <= ctx->L; ++l) TRY(run_layer(ctx, l, st));
   return TG_OK;
+}
+
+tg_status run_superbatch(tg_ctx* ctx, int S, bool edge_mode, const EdgeSrc& es, int n_max_top, cudaStream_t st) {
+  TRY(run_front(ctx, S, edge_mode, es, n_max_top, st));
+  return run_back(ctx, st);
 }
 
 tg_status finish(tg_ctx* ctx, int S, long long* log, int64_t row0, cudaStream_t st) {
@@ -399,10 +421,24 @@ tg_status finish(tg_ctx* ctx, int S, long long* log, int64_t row0, cudaStream_t 
 tg_status stream_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, const uint32_t* ts, int64_t n_edges,
                        int batch, float* scores, long long* log, cudaStream_t st) {
   const int64_t nb = (n_edges + batch - 1) / batch;
-  for (int64_t b0 = 0; b0 < nb; b0 += ctx->S) {
+  // Two-set pipeline: superbatch i's front half runs on ctx->fst into level set
+  // i % 2 as soon as superbatch i-2's layers released that set, overlapping the
+  // layers of superbatch i-1 on st. The cache index is only touched by front
+  // halves (in order on fst) and ring rows only by layers (in order on st), so
+  // every kernel sees the same data as in the serial order.
+  CK(cudaEventRecord(ctx->ev_in, st));
+  CK(cudaStreamWaitEvent(ctx->fst, ctx->ev_in, 0));
+  int64_t sb = 0;
+  for (int64_t b0 = 0; b0 < nb; b0 += ctx->S, ++sb) {
     const int S = (int)std::min<int64_t>(ctx->S, nb - b0);
+    const int set = (int)(sb & 1);
     EdgeSrc es{src, dst, ts, n_edges, b0 * batch, batch};
-    TRY(run_superbatch(ctx, S, true, es, 2 * batch, st));
+    select_set(ctx, set);
+    if (sb >= 2) CK(cudaStreamWaitEvent(ctx->fst, ctx->ev_back[set], 0));
+    TRY(run_front(ctx, S, true, es, 2 * batch, ctx->fst));
+    CK(cudaEventRecord(ctx->ev_front[set], ctx->fst));
+    CK(cudaStreamWaitEvent(st, ctx->ev_front[set], 0));
+    TRY(run_back(ctx, st));
     {
       Prof pf(ctx, TG_ST_SCORE, st);
       launch_score_rows(ctx->HL, ctx->dnp, ctx->lv[ctx->L], S, es, ctx->sc_rs, ctx->sc_rd, ctx->sc_oidx, ctx->sc_m,
@@ -426,7 +462,11 @@ tg_status stream_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, cons
     }
     TRY(launched(ctx, 3));
     TRY(finish(ctx, S, log, b0, st));
+    CK(cudaEventRecord(ctx->ev_back[set], st));
   }
+  CK(cudaEventRecord(ctx->ev_fend, ctx->fst));  // join the front stream into st
+  CK(cudaStreamWaitEvent(st, ctx->ev_fend, 0));
+  select_set(ctx, 0);
   return TG_OK;
 }
 
@@ -722,8 +762,9 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
   }
   // ---- recursion levels: batch-segmented lists + superbatch compute lists
   int maxC = 0;
+  for (int set = 0; set < 2; ++set)
   for (int l = 1; l <= L; ++l) {
-    LevelDev& v = ctx->lv[l];
+    LevelDev& v = ctx->lvs[set][l];
     const size_t n = (size_t)S * cap[l];
     ctx->cap[l] = cap[l];
     v.cap = cap[l];
@@ -792,8 +833,20 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     TRY(tc_make_tensor_a(ctx->z_h, 2, ctx->ld_z, maxC, &ctx->ta_z));
   }
   TRY(dalloc(ctx, &ctx->cnt_total, TG_NCOUNTERS));
-  TRY(dalloc(ctx, &ctx->cnt_sb, (size_t)kMaxS * TG_NCOUNTERS));
-  CK(cudaMemset(ctx->cnt_sb, 0, (size_t)kMaxS * TG_NCOUNTERS * sizeof(long long)));
+  for (int set = 0; set < 2; ++set) {
+    TRY(dalloc(ctx, &ctx->cnt_sbs[set], (size_t)kMaxS * TG_NCOUNTERS));
+    CK(cudaMemset(ctx->cnt_sbs[set], 0, (size_t)kMaxS * TG_NCOUNTERS * sizeof(long long)));
+  }
+  select_set(ctx, 0);
+  if (!ctx->fst) {
+    CK(cudaStreamCreateWithFlags(&ctx->fst, cudaStreamNonBlocking));
+    for (int i = 0; i < 2; ++i) {
+      CK(cudaEventCreateWithFlags(&ctx->ev_front[i], cudaEventDisableTiming));
+      CK(cudaEventCreateWithFlags(&ctx->ev_back[i], cudaEventDisableTiming));
+    }
+    CK(cudaEventCreateWithFlags(&ctx->ev_in, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&ctx->ev_fend, cudaEventDisableTiming));
+  }
   CK(cudaDeviceSynchronize());
   ctx->loaded = true;
   return tg_cache_reset(ctx, -1);
@@ -1092,6 +1145,9 @@ void tg_free(tg_ctx* ctx) {
   cudaDeviceSynchronize();
   for (void* p : ctx->owned) cudaFree(p);
   for (cudaEvent_t e : ctx->ev_pool) cudaEventDestroy(e);
+  for (cudaEvent_t e : {ctx->ev_front[0], ctx->ev_front[1], ctx->ev_back[0], ctx->ev_back[1], ctx->ev_in, ctx->ev_fend})
+    if (e) cudaEventDestroy(e);
+  if (ctx->fst) cudaStreamDestroy(ctx->fst);
   if (ctx->stage) cudaFree(ctx->stage);
   delete ctx;
 }
