@@ -610,7 +610,20 @@ tg_status tc_make_tensor_a(const void* base, int elem_bytes, int ld, int rows, T
   cuuint32_t box[2] = {(cuuint32_t)(128 / elem_bytes), (cuuint32_t)TC_BM};
   cuuint32_t estr[2] = {1, 1};
   const CUtensorMapDataType dt = elem_bytes == 2 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32;
-  CUresult r = cuTensorMapEncodeTiled(&out->map, dt, 2, const_cast<void*>(base), dims, strides, box, estr,
+  // Resolved through the runtime so libtg.so does not link libcuda (absent on GPU-less build hosts).
+  typedef CUresult (*encode_fn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+  static encode_fn encode = nullptr;
+  if (!encode) {
+    void* fp = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fp, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess || !fp)
+      return TG_ECUDA;
+    encode = (encode_fn)fp;
+  }
+  CUresult r = encode(&out->map, dt, 2, const_cast<void*>(base), dims, strides, box, estr,
                                       CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
                                       CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return TG_ECUDA;
