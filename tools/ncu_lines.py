@@ -11,6 +11,7 @@ import subprocess
 ap = argparse.ArgumentParser()
 ap.add_argument("rep")
 ap.add_argument("--top", type=int, default=30)
+ap.add_argument("--sort", default="samples")
 a = ap.parse_args()
 out = subprocess.run(["ncu", "-i", a.rep, "--page", "source", "--csv", "--print-source", "cuda,sass"],
                      capture_output=True, text=True).stdout
@@ -51,7 +52,7 @@ for r in rows[hi + 1:]:
 ti = sum(c["instr"] for c in agg.values())
 ts = sum(c["samples"] for c in agg.values())
 print(f"instructions {ti:.0f}  samples {ts:.0f}")
-for ln, c in sorted(agg.items(), key=lambda kv: -kv[1]["samples"])[:a.top]:
+for ln, c in sorted(agg.items(), key=lambda kv: -kv[1][a.sort])[:a.top]:
     top = sorted(((v, k) for k, v in c.items() if k not in ("instr", "samples")), reverse=True)[:3]
     print(f"{ln:5d} {100 * c['instr'] / ti:5.1f}%i {100 * c['samples'] / ts:5.1f}%s  {src_of.get(ln, '')[:64]:64s} "
           + " ".join(f"{k}:{int(v)}" for v, k in top))
