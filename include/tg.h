@@ -109,8 +109,9 @@ typedef struct {
  *   shared:       omega[d_t], phi[d_t], W_a1[d_n*2d_n], b_a1[d_n], W_a2[d_n], b_a2[1]
  * Uploads/prepares weights, builds Phi table and Phi(0),
  * allocates workspaces and the cache, and resets it. Synchronous.
- * Errors: TG_ESTATE (no graph), TG_EINVAL (n_params mismatch, bad cfg),
- * TG_ENOMEM, TG_ECUDA. May be called again to replace the model. */
+ * Errors: TG_ESTATE (no graph), TG_EINVAL (n_params mismatch, bad cfg, or a time
+ * encoder with |omega_c| * 2^32 + |phi_c| >= 1e15, beyond the device cosine's fp64
+ * argument reduction), TG_ENOMEM, TG_ECUDA. May be called again to replace the model. */
 tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* params, int64_t n_params);
 
 /* ------------------------------------------------------------------------ */

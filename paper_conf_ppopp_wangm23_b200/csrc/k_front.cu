@@ -1011,20 +1011,24 @@ __global__ void k_resolve(ResolveArgs a, int* err) {
                                 : a.HL + (size_t)q * a.ldn;
     } else {
       const size_t o = (size_t)q * k + m;
-      const float* r;
+      long long row;
+      const float* base;
       if (l == 1) {
         int node = lv.nb_node[o];
         if (node < 0) {
           atomicOr(err, kErrNodeRange);
           node = 0;
         }
-        r = a.X + (size_t)node * a.ldn;
+        row = node;
+        base = a.X;
       } else {
         const int nb = lv.n_c[b];
         const size_t seg = (size_t)b * pv.cap;
-        r = a.ring[l - 1] + (size_t)pv.slot[seg + pv.inv[seg + nb + (size_t)p * k + m]] * a.ldn;
+        row = pv.slot[seg + pv.inv[seg + nb + (size_t)p * k + m]];
+        base = a.ring[l - 1];
       }
-      lv.nb_row[o] = r;
+      lv.nb_row[o] = base + (size_t)row * a.ldn;
+      lv.nb_hidx[o] = (int32_t)row;
     }
   }
 }

@@ -65,6 +65,7 @@ struct tg_ctx {
   unsigned short *c_h = nullptr, *rh_h = nullptr, *z_h = nullptr;
   int ld_ch = 0, ld_rh = 0, ld_z = 0;
   TcTensorA ta_c, ta_rh, ta_z;  // TMA tensor maps of the bf16 activations (dense GEMM A operands)
+  AttnMaps am[TG_MAX_LAYERS + 1]{};  // per level l: TMA row-gather maps (h rows of level l, E, Phi table)
   // counters / flags
   long long* cnt_total = nullptr;
   long long* cnt_sb = nullptr;  // [kMaxS x TG_NCOUNTERS] of the current set
@@ -240,6 +241,7 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   a.k = ctx->k;
   a.nc_dev = m_dev;
   a.nc_max = mmax;
+  a.nb_hidx = lv.nb_hidx;
   const bool bfa = ctx->cfg.precision == TG_PREC_BF16;  // bf16 activations between the GEMMs
   if (bfa) {
     a.c = nullptr;
@@ -248,7 +250,59 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   }
   {
     Prof pf(ctx, TG_ST_ATTN, st);
-    launch_attn(a, st);
+    launch_attn(a, &ctx->am[l], st);
+  }
+  static const bool attn_sync = getenv("TG_ATTN_SYNC") != nullptr;  // debug
+  if (attn_sync) cudaStreamSynchronize(st);
+  static const bool attn_check = getenv("TG_ATTN_CHECK") != nullptr;  // debug: gather vs CTA kernel
+  if (attn_check && !bfa) {
+    int nc = 0;
+    cudaStreamSynchronize(st);
+    cudaMemcpy(&nc, m_dev, sizeof(int), cudaMemcpyDeviceToHost);
+    float* ref = nullptr;
+    cudaMalloc(&ref, (size_t)std::max(nc, 1) * HDp * sizeof(float));
+    AttnArgs b = a;
+    b.c = ref;
+    b.nb_hidx = nullptr;  // forces the CTA kernel
+    launch_attn(b, nullptr, st);
+    cudaStreamSynchronize(st);
+    std::vector<float> x((size_t)nc * HDp), y((size_t)nc * HDp);
+    cudaMemcpy(x.data(), ctx->c, x.size() * 4, cudaMemcpyDeviceToHost);
+    cudaMemcpy(y.data(), ref, y.size() * 4, cudaMemcpyDeviceToHost);
+    if (getenv("TG_ATTN_USE_REF")) cudaMemcpy(ctx->c, ref, y.size() * 4, cudaMemcpyDeviceToDevice);
+    cudaFree(ref);
+    int bad = 0;
+    float gmd = 0.f;
+    for (int p = 0; p < nc; ++p) {
+      float md = 0.f, mag = 0.f;
+      int jw = 0;
+      for (int j = 0; j < HDp; ++j) mag = std::max(mag, std::fabs(y[(size_t)p * HDp + j]));
+      for (int j = 0; j < HDp; ++j) {
+        const float d = std::fabs(x[(size_t)p * HDp + j] - y[(size_t)p * HDp + j]) / (1e-20f + mag);
+        if (d > md) {
+          md = d;
+          jw = j;
+        }
+      }
+      gmd = std::max(gmd, md);
+      if (md > 1e-5f && bad++ < 8)
+        fprintf(stderr, "attn check: level %d target %d/%d max diff/rowmax %g at col %d (got %g ref %g)\n", l, p, nc,
+                md, jw, x[(size_t)p * HDp + jw], y[(size_t)p * HDp + jw]);
+    }
+    fprintf(stderr, "attn check: level %d: %d of %d targets differ (max rel %g)\n", l, bad, nc, gmd);
+    {
+      const size_t nr = (size_t)nc * ctx->k;
+      std::vector<const float*> rp(nr);
+      std::vector<int32_t> hi(nr);
+      cudaMemcpy(rp.data(), lv.nb_row, nr * sizeof(void*), cudaMemcpyDeviceToHost);
+      cudaMemcpy(hi.data(), lv.nb_hidx, nr * 4, cudaMemcpyDeviceToHost);
+      const float* hb = l == 1 ? ctx->X : ctx->cache[l - 1].ring;
+      int nbad = 0;
+      for (size_t i = 0; i < nr; ++i)
+        if (rp[i] != hb + (size_t)hi[i] * ctx->g.ldn && nbad++ < 4)
+          fprintf(stderr, "attn check: row %zu ptr off %td vs idx %d\n", i, (rp[i] - hb), hi[i]);
+      fprintf(stderr, "attn check: level %d: %d of %zu row indices inconsistent\n", l, nbad, nr);
+    }
   }
   TRY(launched(ctx));
   // G2: y = F c + b_fc  (W_v and W_fc folded; the residual q of Eq. 4 is added by the LayerNorm)
@@ -638,6 +692,10 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
   // ---- time encoder: Phi table [max(W,1) x dtp] on device; Phi(0) = row 0
   const float* om = params + L * per_layer;
   const float* ph = om + d_t;
+  // The device cosine reduces its argument in fp64 (two-term Cody-Waite), accurate for
+  // |dt * omega + phi| < 1e15; dt < 2^32 (R4), so bound |omega| and |phi| accordingly.
+  for (int c = 0; c < d_t; ++c)
+    if (!(std::fabs((double)om[c]) * 4294967296.0 + std::fabs((double)ph[c]) < 1e15)) return TG_EINVAL;
   TRY(dalloc(ctx, &ctx->omega, d_t));
   TRY(dalloc(ctx, &ctx->phi, d_t));
   const int Wrows = std::max(ctx->W, 1);
@@ -792,6 +850,7 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     TRY(dalloc(ctx, &v.nb_eid, n * k));
     TRY(dalloc(ctx, &v.hs_row, n));
     TRY(dalloc(ctx, &v.nb_row, n * k));
+    TRY(dalloc(ctx, &v.nb_hidx, n * k));
     TRY(dalloc(ctx, &v.dst_row, n));
     CK(cudaMemset(v.n_c_total, 0, sizeof(int)));
     CK(cudaMemset(v.n_in, 0, kMaxS * sizeof(int)));
@@ -831,6 +890,17 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     TRY(tc_make_tensor_a(ctx->c_h, 2, ctx->ld_ch, maxC, &ctx->ta_c));
     TRY(tc_make_tensor_a(ctx->rh_h, 2, ctx->ld_rh, maxC, &ctx->ta_rh));
     TRY(tc_make_tensor_a(ctx->z_h, 2, ctx->ld_z, maxC, &ctx->ta_z));
+  }
+  // TMA row-gather maps for the attention (feature rows <= 256 fp32; else the CTA kernel gathers)
+  for (int l = 1; l <= L; ++l) {
+    AttnMaps& m = ctx->am[l];
+    m.valid = 0;
+    const float* hb = l == 1 ? ctx->X : ctx->cache[l - 1].ring;
+    const long long hrows = l == 1 ? ctx->g.V + 1 : ctx->cache[l - 1].rcap;
+    if (attn_make_rows_map(hb, dnp, ctx->g.ldn, hrows, &m.h) == TG_OK &&
+        attn_make_rows_map(ctx->Ef, ctx->dep, ctx->g.lde, ctx->g.E + 1, &m.e) == TG_OK &&
+        attn_make_rows_map(ctx->table, ctx->dtp, ctx->dtp, std::max(ctx->W, 1), &m.t) == TG_OK)
+      m.valid = 1;
   }
   TRY(dalloc(ctx, &ctx->cnt_total, TG_NCOUNTERS));
   for (int set = 0; set < 2; ++set) {

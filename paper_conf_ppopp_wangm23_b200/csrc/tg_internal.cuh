@@ -16,6 +16,7 @@
 // superbatch in (batch, unique-list) order, with its neighbour slots stored
 // compute-centric at [q*k + m].
 #pragma once
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -101,6 +102,7 @@ struct LevelDev {
   // row addresses resolved for the layer-l compute
   const float** hs_row;      // [c_cap]     h^(l-1) of the target
   const float** nb_row;      // [c_cap * k] h^(l-1) of each neighbour
+  int32_t* nb_hidx;          // [c_cap * k] its row in the level's h tensor (X at l = 1, else ring l-1)
   float** dst_row;           // [c_cap]     where h^(l) goes (ring slot or H_L)
 };
 
@@ -171,8 +173,15 @@ struct AttnArgs {
   int nc_max;
   unsigned short* c_h;     // if non-null: c written as bf16 [nc x ldc_h] (zero padded) instead of fp32
   int ldc_h;
+  const int32_t* nb_hidx;  // row indices of nb_row in maps.h (gather path)
 };
-void launch_attn(const AttnArgs& a, cudaStream_t st);
+// TMA row-gather maps of the attention sources: h rows of the level, E rows, Phi table rows.
+struct AttnMaps {
+  CUtensorMap h, e, t;
+  int valid;
+};
+tg_status attn_make_rows_map(const float* base, int row_elems, int ld, long long rows, CUtensorMap* out);
+void launch_attn(const AttnArgs& a, const AttnMaps* maps, cudaStream_t st);
 
 // C[M x N] = A[M x K] B^T + epilogue, fp32 CUDA cores (TG_PREC_FP32).
 // A row p = seg0[p][0:K0] || seg1[p][0:K-K0] (seg pointers from arrays or dense bases).
