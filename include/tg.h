@@ -215,7 +215,8 @@ int64_t tg_kernel_launches(tg_ctx* ctx);
 #define TG_ST_FFN2 10    /* includes the CacheStore payload write          */
 #define TG_ST_SCORE 11
 #define TG_ST_OTHER 12
-#define TG_NSTAGES 13
+#define TG_ST_PHI 13     /* TimeEncode of dt >= W rows (front stream, Eq. 8) */
+#define TG_NSTAGES 14
 tg_status tg_profile_enable(tg_ctx* ctx, int32_t on);
 tg_status tg_profile_read(tg_ctx* ctx, double* ms, int64_t* launches, int32_t n);
 

@@ -65,7 +65,12 @@ struct tg_ctx {
   unsigned short *c_h = nullptr, *rh_h = nullptr, *z_h = nullptr;
   int ld_ch = 0, ld_rh = 0, ld_z = 0;
   TcTensorA ta_c, ta_rh, ta_z;  // TMA tensor maps of the bf16 activations (dense GEMM A operands)
-  AttnMaps am[TG_MAX_LAYERS + 1]{};  // per level l: TMA row-gather maps (h rows of level l, E, Phi table)
+  AttnMaps am[2][TG_MAX_LAYERS + 1]{};  // per set and level l: TMA row-gather maps (h rows, E rows, Phi rows)
+  int cur_set = 0;
+  // Phi rows per set: [table (W rows) | direct rows of level 1 | level 2 | ...] (k_phi_rows, front stream)
+  float* phi_buf[2] = {nullptr, nullptr};
+  long long phi_row0[TG_MAX_LAYERS + 1]{};
+  bool phi_pre = false;
   // counters / flags
   long long* cnt_total = nullptr;
   long long* cnt_sb = nullptr;  // [kMaxS x TG_NCOUNTERS] of the current set
@@ -242,6 +247,7 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   a.nc_dev = m_dev;
   a.nc_max = mmax;
   a.nb_hidx = lv.nb_hidx;
+  a.phi_row0 = ctx->phi_pre ? ctx->phi_row0[l] : -1;
   const bool bfa = ctx->cfg.precision == TG_PREC_BF16;  // bf16 activations between the GEMMs
   if (bfa) {
     a.c = nullptr;
@@ -250,7 +256,7 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   }
   {
     Prof pf(ctx, TG_ST_ATTN, st);
-    launch_attn(a, &ctx->am[l], st);
+    launch_attn(a, &ctx->am[ctx->cur_set][l], st);
   }
   static const bool attn_sync = getenv("TG_ATTN_SYNC") != nullptr;  // debug
   if (attn_sync) cudaStreamSynchronize(st);
@@ -390,6 +396,7 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
 // (targets src || dst), else one batch of explicit targets (prepared in lv[L]).
 // ------------------------------------------------------------------------
 void select_set(tg_ctx* ctx, int s) {
+  ctx->cur_set = s;
   ctx->lv = ctx->lvs[s];
   ctx->cnt_sb = ctx->cnt_sbs[s];
 }
@@ -450,7 +457,29 @@ tg_status run_front(tg_ctx* ctx, int S, bool edge_mode, const EdgeSrc& es, int n
     Prof pf(ctx, TG_ST_RESOLVE, st);
     launch_resolve(ra, ctx->err, st);
   }
-  return launched(ctx);
+  TRY(launched(ctx));
+  if (ctx->phi_pre && ctx->am[ctx->cur_set][1].valid) {  // TimeEncode of the dt >= W rows (Eq. 8)
+    PhiRowsArgs pa{};
+    for (int l = 0; l <= L; ++l) {
+      pa.lv[l] = ctx->lv[l];
+      pa.row0[l] = ctx->phi_row0[l];
+    }
+    pa.out = ctx->phi_buf[ctx->cur_set];
+    pa.omega = ctx->omega;
+    pa.phi = ctx->phi;
+    pa.L = L;
+    pa.k = k;
+    pa.W = ctx->W;
+    pa.use_table = use_table;
+    pa.d_t = ctx->d_t;
+    pa.dtp = ctx->dtp;
+    {
+      Prof pf(ctx, TG_ST_PHI, st);
+      launch_phi_rows(pa, st);
+    }
+    TRY(launched(ctx));
+  }
+  return TG_OK;
 }
 
 // Bottom-up half (Alg. 1 l.13-18): M and FFN, layer by layer over all S batches.
@@ -891,16 +920,37 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     TRY(tc_make_tensor_a(ctx->rh_h, 2, ctx->ld_rh, maxC, &ctx->ta_rh));
     TRY(tc_make_tensor_a(ctx->z_h, 2, ctx->ld_z, maxC, &ctx->ta_z));
   }
-  // TMA row-gather maps for the attention (feature rows <= 256 fp32; else the CTA kernel gathers)
-  for (int l = 1; l <= L; ++l) {
-    AttnMaps& m = ctx->am[l];
-    m.valid = 0;
-    const float* hb = l == 1 ? ctx->X : ctx->cache[l - 1].ring;
-    const long long hrows = l == 1 ? ctx->g.V + 1 : ctx->cache[l - 1].rcap;
-    if (attn_make_rows_map(hb, dnp, ctx->g.ldn, hrows, &m.h) == TG_OK &&
-        attn_make_rows_map(ctx->Ef, ctx->dep, ctx->g.lde, ctx->g.E + 1, &m.e) == TG_OK &&
-        attn_make_rows_map(ctx->table, ctx->dtp, ctx->dtp, std::max(ctx->W, 1), &m.t) == TG_OK)
-      m.valid = 1;
+  // Phi rows of dt >= W computed ahead on the front stream into a per-set buffer that follows a
+  // copy of the table, so the attention gathers every Phi row from one tensor (dense row index
+  // W + q*k + m per level; skipped when the buffers would exceed 16 GB: in-kernel Phi instead)
+  {
+    long long rows = Wrows;
+    for (int l = 1; l <= L; ++l) {
+      ctx->phi_row0[l] = rows;
+      rows += (long long)ctx->lvs[0][l].c_cap * k;
+    }
+    const size_t bytes = (size_t)rows * ctx->dtp * sizeof(float);
+    ctx->phi_pre = 2 * bytes <= (16ull << 30) && rows < (1ll << 31);
+    if (ctx->phi_pre)
+      for (int set = 0; set < 2; ++set) {
+        TRY(dalloc(ctx, &ctx->phi_buf[set], (size_t)rows * ctx->dtp));
+        CK(cudaMemcpy(ctx->phi_buf[set], ctx->table, (size_t)Wrows * ctx->dtp * sizeof(float),
+                      cudaMemcpyDeviceToDevice));
+      }
+    // TMA row-gather maps for the attention (feature rows <= 256 fp32; else the CTA kernel gathers)
+    for (int set = 0; set < 2; ++set)
+      for (int l = 1; l <= L; ++l) {
+        AttnMaps& m = ctx->am[set][l];
+        m.valid = 0;
+        const float* hb = l == 1 ? ctx->X : ctx->cache[l - 1].ring;
+        const long long hrows = l == 1 ? ctx->g.V + 1 : ctx->cache[l - 1].rcap;
+        const float* tb = ctx->phi_pre ? ctx->phi_buf[set] : ctx->table;
+        const long long trows = ctx->phi_pre ? rows : Wrows;
+        if (attn_make_rows_map(hb, dnp, ctx->g.ldn, hrows, &m.h) == TG_OK &&
+            attn_make_rows_map(ctx->Ef, ctx->dep, ctx->g.lde, ctx->g.E + 1, &m.e) == TG_OK &&
+            attn_make_rows_map(tb, ctx->dtp, ctx->dtp, trows, &m.t) == TG_OK)
+          m.valid = 1;
+      }
   }
   TRY(dalloc(ctx, &ctx->cnt_total, TG_NCOUNTERS));
   for (int set = 0; set < 2; ++set) {

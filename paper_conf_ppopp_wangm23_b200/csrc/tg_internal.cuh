@@ -174,6 +174,7 @@ struct AttnArgs {
   unsigned short* c_h;     // if non-null: c written as bf16 [nc x ldc_h] (zero padded) instead of fp32
   int ldc_h;
   const int32_t* nb_hidx;  // row indices of nb_row in maps.h (gather path)
+  long long phi_row0;      // >= 0: Phi rows of dt >= W precomputed at rows phi_row0 + p*k + m of maps.t
 };
 // TMA row-gather maps of the attention sources: h rows of the level, E rows, Phi table rows.
 struct AttnMaps {
@@ -181,6 +182,18 @@ struct AttnMaps {
   int valid;
 };
 tg_status attn_make_rows_map(const float* base, int row_elems, int ld, long long rows, CUtensorMap* out);
+
+// Phi(t - t_j) rows of every (target, neighbour) pair with dt >= W (or no
+// table) of levels 1..L, written to out + (row0[l] + q*k + m) * dtp (Eq. 8).
+struct PhiRowsArgs {
+  LevelDev lv[TG_MAX_LAYERS + 1];
+  long long row0[TG_MAX_LAYERS + 1];
+  float* out;
+  const float* omega;
+  const float* phi;
+  int L, k, W, use_table, d_t, dtp;
+};
+void launch_phi_rows(const PhiRowsArgs& a, cudaStream_t st);
 void launch_attn(const AttnArgs& a, const AttnMaps* maps, cudaStream_t st);
 
 // C[M x N] = A[M x K] B^T + epilogue, fp32 CUDA cores (TG_PREC_FP32).

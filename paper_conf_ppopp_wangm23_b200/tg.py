@@ -27,7 +27,7 @@ EXPORTS = ("tg_graph_load", "tg_model_load", "tg_embed_batch", "tg_score_edges",
            "tg_kernel_launches", "tg_free", "tg_strerror", "tg_version", "tg_profile_enable",
            "tg_profile_read", "tg_gemm")
 STAGES = ("prep", "dedup", "lookup", "sample", "resolve", "proj_k", "attn", "proj_v", "lnorm", "ffn1", "ffn2",
-          "score", "other")
+          "score", "other", "phi")
 
 
 class TGError(RuntimeError):
