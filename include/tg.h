@@ -99,7 +99,10 @@ typedef struct {
   int32_t superbatch;         /* S: batches per launch sequence in tg_score_stream (0 = 16,
                                * 1 = one batch at a time). Semantics per batch are unchanged:
                                * dedup scope, cache lookups and FIFO inserts stay per batch
-                               * and in batch order, so outputs and counters do not depend on S. */
+                               * and in batch order, so outputs and counters do not depend on S.
+                               * S is lowered so that S x (per-batch capacity of each cached
+                               * level) fits the cache passes' DSMEM hash (157,286 keys):
+                               * batch 200, k = 20 keeps S <= 18; batch 2,000 runs S = 1. */
 } tg_model_cfg;
 
 /* params: host float32 [n_params] in this order (row-major, Linear = [out x in]),

@@ -24,7 +24,7 @@ __device__ __forceinline__ float4 gemm_load_a(const GemmArgs& g, int row, int M,
   return *reinterpret_cast<const float4*>(p);
 }
 
-__global__ void __launch_bounds__(256) k_gemm_simt(GemmArgs g) {
+__global__ void __launch_bounds__(256) k_gemm_simt(GemmArgs g) { pdl_enter();
   __shared__ __align__(16) float As[GBK][GBM + 4];
   __shared__ __align__(16) float Bs[GBK][GBN + 4];
   const int M = *g.m_dev;
@@ -90,14 +90,14 @@ void launch_gemm_simt(const GemmArgs& g, cudaStream_t st) {
   const int tiles = ((g.m_max + GBM - 1) / GBM) * ((g.N + GBN - 1) / GBN);
   int blocks = tiles < 148 * 4 ? tiles : 148 * 4;
   if (blocks < 1) blocks = 1;
-  k_gemm_simt<<<blocks, 256, 0, st>>>(g);
+  launch_k(k_gemm_simt, dim3(blocks), dim3(256), 0, st, g);
 }
 
 // ---------------------------------------------------------------- LayerNorm
 __global__ void k_layernorm(const float* __restrict__ y, float* __restrict__ r, int Dp, int dn, int dnp, int de,
                             int dep, int dt, const float* __restrict__ gamma, const float* __restrict__ beta,
                             const int* __restrict__ m_dev, const float* const* __restrict__ hs_rows,
-                            const float* __restrict__ phi0, unsigned short* __restrict__ rh, int ldrh) {
+                            const float* __restrict__ phi0, unsigned short* __restrict__ rh, int ldrh) { pdl_enter();
   const int M = *m_dev;
   const int lane = threadIdx.x & 31;
   const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, nw = (gridDim.x * blockDim.x) >> 5;
@@ -194,7 +194,7 @@ void launch_layernorm(const float* y, float* r, int Dp, int dn, int dnp, int de,
   int blocks = (m_max * 32 + 255) / 256;
   if (blocks < 1) blocks = 1;
   if (blocks > 1184) blocks = 1184;
-  k_layernorm<<<blocks, 256, 0, st>>>(y, r, Dp, dn, dnp, de, dep, dt, gamma, beta, m_dev, hs_rows, phi0, rh,
+  launch_k(k_layernorm, dim3(blocks), dim3(256), 0, st, y, r, Dp, dn, dnp, de, dep, dt, gamma, beta, m_dev, hs_rows, phi0, rh,
                                       ldrh);
 }
 
@@ -205,7 +205,7 @@ void launch_layernorm(const float* y, float* r, int Dp, int dn, int dnp, int de,
 // per edge for the W_a2 dot product and the sigmoid.
 __global__ void k_score_rows(const float* __restrict__ HL, int ldh, LevelDev top, int S, EdgeSrc es,
                              const float** __restrict__ rs, const float** __restrict__ rd,
-                             long long* __restrict__ oidx, int* __restrict__ m_dev) {
+                             long long* __restrict__ oidx, int* __restrict__ m_dev) { pdl_enter();
   const int tot = S * es.B;
   if (blockIdx.x == 0 && threadIdx.x == 0) *m_dev = tot;
   for (int w = blockIdx.x * blockDim.x + threadIdx.x; w < tot; w += gridDim.x * blockDim.x) {
@@ -230,11 +230,11 @@ void launch_score_rows(const float* HL, int ldh, LevelDev top, int S, EdgeSrc es
                        const float** rd, long long* oidx, int* m_dev, cudaStream_t st) {
   int blocks = (S * es.B + 255) / 256;
   if (blocks < 1) blocks = 1;
-  k_score_rows<<<blocks, 256, 0, st>>>(HL, ldh, top, S, es, rs, rd, oidx, m_dev);
+  launch_k(k_score_rows, dim3(blocks), dim3(256), 0, st, HL, ldh, top, S, es, rs, rd, oidx, m_dev);
 }
 
 __global__ void k_score_head(const float* __restrict__ z, int ldz, const long long* __restrict__ oidx, int M,
-                             const float* __restrict__ Wa2, float ba2, int dn, float* __restrict__ scores) {
+                             const float* __restrict__ Wa2, float ba2, int dn, float* __restrict__ scores) { pdl_enter();
   const int lane = threadIdx.x & 31;
   const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, nw = (gridDim.x * blockDim.x) >> 5;
   for (int w = warp; w < M; w += nw) {
@@ -254,11 +254,11 @@ void launch_score_head(const float* z, int ldz, const long long* oidx, int M, co
   int blocks = (M * 32 + 255) / 256;
   if (blocks < 1) blocks = 1;
   if (blocks > 1184) blocks = 1184;
-  k_score_head<<<blocks, 256, 0, st>>>(z, ldz, oidx, M, Wa2, ba2, dn, scores);
+  launch_k(k_score_head, dim3(blocks), dim3(256), 0, st, z, ldz, oidx, M, Wa2, ba2, dn, scores);
 }
 
 __global__ void k_invert(const float* __restrict__ HL, int ldh, LevelDev top, int n, int dn,
-                         float* __restrict__ out) {
+                         float* __restrict__ out) { pdl_enter();
   const long long tot = (long long)n * dn;
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < tot; i += (long long)gridDim.x * blockDim.x) {
     const long long r = i / dn;
@@ -272,10 +272,10 @@ void launch_invert(const float* HL, int ldh, LevelDev top, int n, int dn, float*
   long long tot = (long long)n * dn;
   int blocks = (int)((tot + 255) / 256);
   if (blocks > 1184) blocks = 1184;
-  k_invert<<<blocks, 256, 0, st>>>(HL, ldh, top, n, dn, out);
+  launch_k(k_invert, dim3(blocks), dim3(256), 0, st, HL, ldh, top, n, dn, out);
 }
 
-__global__ void k_set_int(int* p, int v) { *p = v; }
-void launch_set_int(int* p, int v, cudaStream_t st) { k_set_int<<<1, 1, 0, st>>>(p, v); }
+__global__ void k_set_int(int* p, int v) { pdl_enter(); *p = v; }
+void launch_set_int(int* p, int v, cudaStream_t st) { launch_k(k_set_int, dim3(1), dim3(1), 0, st, p, v); }
 
 }  // namespace tg

@@ -54,7 +54,7 @@ __device__ __forceinline__ int batch_edges(const EdgeSrc& es, int b, int64_t& lo
 // with an ordered scan across the cluster (first-occurrence order, R8);
 // phase D reads the inverse index.
 __global__ void __launch_bounds__(kDedupThreads, 1)
-k_dedup(LevelDev lv, int edge_mode, EdgeSrc es, long long* cnt, int layer, int* err) {
+k_dedup(LevelDev lv, int edge_mode, EdgeSrc es, long long* cnt, int layer, int* err) { pdl_enter();
   extern __shared__ __align__(16) unsigned char smem[];
   unsigned long long* skey = reinterpret_cast<unsigned long long*>(smem);
   unsigned int* spos = reinterpret_cast<unsigned int*>(skey + kDedupSlots);
@@ -179,7 +179,7 @@ k_dedup(LevelDev lv, int edge_mode, EdgeSrc es, long long* cnt, int layer, int* 
 }
 
 // dedup disabled (ablation): identity unique list and inverse index
-__global__ void k_dedup_off(LevelDev lv, int S, int edge_mode, EdgeSrc es, long long* cnt, int layer) {
+__global__ void k_dedup_off(LevelDev lv, int S, int edge_mode, EdgeSrc es, long long* cnt, int layer) { pdl_enter();
   for (int b = blockIdx.y; b < S; b += gridDim.y) {
     int64_t elo = 0;
     int Bb = 0, n;
@@ -227,7 +227,7 @@ void launch_dedup(LevelDev lv, int S, int n_max, bool edge_mode, EdgeSrc es, lon
     int bx = (n_max + 255) / 256;
     if (bx < 1) bx = 1;
     if (bx > 64) bx = 64;
-    k_dedup_off<<<dim3(bx, S), 256, 0, st>>>(lv, S, edge_mode ? 1 : 0, es, cnt, layer);
+    launch_k(k_dedup_off, dim3(dim3(bx, S)), dim3(256), 0, st, lv, S, edge_mode ? 1 : 0, es, cnt, layer);
     return;
   }
   const int cl = dedup_cluster_size(n_max);
@@ -238,19 +238,8 @@ void launch_dedup(LevelDev lv, int S, int n_max, bool edge_mode, EdgeSrc es, lon
     cudaFuncSetAttribute(k_dedup, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
     attr_done = true;
   }
-  cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3(cl * S);
-  cfg.blockDim = dim3(kDedupThreads);
-  cfg.dynamicSmemBytes = smem;
-  cfg.stream = st;
-  cudaLaunchAttribute attr[1];
-  attr[0].id = cudaLaunchAttributeClusterDimension;
-  attr[0].val.clusterDim.x = cl;
-  attr[0].val.clusterDim.y = 1;
-  attr[0].val.clusterDim.z = 1;
-  cfg.attrs = attr;
-  cfg.numAttrs = 1;
-  cudaLaunchKernelEx(&cfg, k_dedup, lv, edge_mode ? 1 : 0, es, cnt, layer, err);
+  launch_k_cluster(k_dedup, dim3(cl * S), dim3(kDedupThreads), smem, st, cl, lv, edge_mode ? 1 : 0, es, cnt, layer,
+                   err);
 }
 
 // ------------------------------------------------------- CacheLookup / Store
@@ -266,7 +255,7 @@ __device__ __forceinline__ unsigned long long ld_volatile_u64(const unsigned lon
 }
 
 __global__ void __launch_bounds__(1024, 1)
-k_probe(LevelDev lv, int S, CacheDev c, int use_cache, int has_ring, long long* cnt, int layer, int* err) {
+k_probe(LevelDev lv, int S, CacheDev c, int use_cache, int has_ring, long long* cnt, int layer, int* err) { pdl_enter();
   __shared__ int s_warp[32];
   __shared__ int s_base;
   __shared__ long long s_head, s_size;
@@ -411,7 +400,7 @@ k_probe(LevelDev lv, int S, CacheDev c, int use_cache, int has_ring, long long* 
 //      global index (key -> head0 + q), skipping keys re-missed later.
 // The newest copy of a key is always first on its probe chain (an insert
 // takes the first dead or empty slot), so lookups stop at the first match.
-__global__ void k_probe_pre(LevelDev lv, int S, CacheDev c) {
+__global__ void k_probe_pre(LevelDev lv, int S, CacheDev c) { pdl_enter();
   const int tot = S * lv.cap;
   for (int idx = blockIdx.x * blockDim.x + threadIdx.x; idx < tot; idx += gridDim.x * blockDim.x) {
     const int b = idx / lv.cap, i = idx - b * lv.cap;
@@ -432,12 +421,12 @@ __global__ void k_probe_pre(LevelDev lv, int S, CacheDev c) {
   }
 }
 
-constexpr int kSeqCL = 16;        // cluster CTAs of the ordered pass
+constexpr int kSeqCL = kSeqCLMax;
 constexpr int kSeqThreads = 1024;
-constexpr int kSeqSlots = 16384;  // DSMEM hash slots per CTA
+constexpr int kSeqSlots = kSeqSlotsPerCTA;
 
 __global__ void __launch_bounds__(kSeqThreads, 1)
-k_probe_seq(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err) {
+k_probe_seq(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err) { pdl_enter();
   extern __shared__ __align__(16) unsigned char smem[];
   unsigned long long* skey = reinterpret_cast<unsigned long long*>(smem);
   int* sq = reinterpret_cast<int*>(skey + kSeqSlots);  // key -> q of its latest miss in this SB
@@ -582,7 +571,7 @@ k_probe_seq(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err)
 // misses with an ordered scan (their FIFO positions are head0 + q) and hands
 // every later occurrence the ring slot of its first one.
 __global__ void __launch_bounds__(kSeqThreads, 1)
-k_probe_par(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err) {
+k_probe_par(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err) { pdl_enter();
   extern __shared__ __align__(16) unsigned char smem[];
   unsigned long long* skey = reinterpret_cast<unsigned long long*>(smem);
   unsigned* sval = reinterpret_cast<unsigned*>(skey + kSeqSlots);  // min j, later: ring slot
@@ -746,7 +735,7 @@ k_probe_par(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err)
 // batches concatenated in batch order, q = c_base[b] + u. With a ring (cache
 // disabled at a cached level) the rows still go to FIFO positions head + q,
 // used as per-superbatch scratch.
-__global__ void k_compact_all(LevelDev lv, int S, CacheDev c, int has_ring, long long* cnt, int layer) {
+__global__ void k_compact_all(LevelDev lv, int S, CacheDev c, int has_ring, long long* cnt, int layer) { pdl_enter();
   __shared__ int s_pre[kMaxS + 1];
   if (threadIdx.x == 0) {
     int a = 0;
@@ -786,9 +775,9 @@ __global__ void k_compact_all(LevelDev lv, int S, CacheDev c, int has_ring, long
 
 // head update of the scratch ring after k_compact_all (separate launch: no
 // intra-grid ordering needed)
-__global__ void k_ring_advance(LevelDev lv, CacheDev c) { c.state[0] += *lv.n_c_total; }
+__global__ void k_ring_advance(LevelDev lv, CacheDev c) { pdl_enter(); c.state[0] += *lv.n_c_total; }
 
-__global__ void k_probe_ins(LevelDev lv, CacheDev c, int* err) {
+__global__ void k_probe_ins(LevelDev lv, CacheDev c, int* err) { pdl_enter();
   const int n = *lv.n_c_total;
   const long long head0 = c.state[4];
   const long long live_lo = c.state[0] - c.state[1];
@@ -833,16 +822,16 @@ int launch_probe(LevelDev lv, int S, const CacheDev* cache, long long* cnt, int 
     int blocks = (S * lv.cap + 255) / 256;
     if (blocks > 148 * 4) blocks = 148 * 4;
     if (blocks < 1) blocks = 1;
-    k_compact_all<<<blocks, 256, 0, st>>>(lv, S, c, has_ring, cnt, layer);
+    launch_k(k_compact_all, dim3(blocks), dim3(256), 0, st, lv, S, c, has_ring, cnt, layer);
     if (has_ring) {
-      k_ring_advance<<<1, 1, 0, st>>>(lv, c);
+      launch_k(k_ring_advance, dim3(1), dim3(1), 0, st, lv, c);
       return 2;
     }
     return 1;
   }
   int blocks = (S * lv.cap + 255) / 256;
   if (blocks > 148 * 8) blocks = 148 * 8;
-  k_probe_pre<<<blocks, 256, 0, st>>>(lv, S, c);
+  launch_k(k_probe_pre, dim3(blocks), dim3(256), 0, st, lv, S, c);
   const size_t smem = (size_t)kSeqSlots * (sizeof(unsigned long long) + sizeof(int));
   static bool attr = false;
   if (!attr) {
@@ -853,29 +842,17 @@ int launch_probe(LevelDev lv, int S, const CacheDev* cache, long long* cnt, int 
   // cluster large enough for every key of the superbatch to be an in-SB miss (load <= 0.6)
   int cl = 1;
   while (cl < kSeqCL && (long long)cl * kSeqSlots * 6 / 10 < (long long)S * lv.cap) cl <<= 1;
-  cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3(cl);
-  cfg.blockDim = dim3(kSeqThreads);
-  cfg.dynamicSmemBytes = smem;
-  cfg.stream = st;
-  cudaLaunchAttribute at[1];
-  at[0].id = cudaLaunchAttributeClusterDimension;
-  at[0].val.clusterDim.x = cl;
-  at[0].val.clusterDim.y = 1;
-  at[0].val.clusterDim.z = 1;
-  cfg.attrs = at;
-  cfg.numAttrs = 1;
   static bool attr2 = false;
   if (!attr2) {
     cudaFuncSetAttribute(k_probe_par, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     cudaFuncSetAttribute(k_probe_par, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
     attr2 = true;
   }
-  cudaLaunchKernelEx(&cfg, k_probe_par, lv, S, c, cnt, layer, err);
-  cudaLaunchKernelEx(&cfg, k_probe_seq, lv, S, c, cnt, layer, err);
+  launch_k_cluster(k_probe_par, dim3(cl), dim3(kSeqThreads), smem, st, cl, lv, S, c, cnt, layer, err);
+  launch_k_cluster(k_probe_seq, dim3(cl), dim3(kSeqThreads), smem, st, cl, lv, S, c, cnt, layer, err);
   int ib = (S * lv.cap + 255) / 256;
   if (ib > 148 * 4) ib = 148 * 4;
-  k_probe_ins<<<ib, 256, 0, st>>>(lv, c, err);
+  launch_k(k_probe_ins, dim3(ib), dim3(256), 0, st, lv, c, err);
   return 4;
 }
 
@@ -887,7 +864,7 @@ int launch_probe(LevelDev lv, int S, const CacheDev* cache, long long* cnt, int 
 // I_{l-1} = [C_l ; N(C_l)] of each batch (Alg. 1 l.12). Also counts, per
 // batch, how many Phi(dt) the precomputed window serves (Sec. 4.3).
 __global__ void k_sample(GraphDev g, LevelDev lv, int S, int k, LevelDev nx, int has_next, int W, int use_table,
-                         long long* cnt, int layer, int* err) {
+                         long long* cnt, int layer, int* err) { pdl_enter();
   const int lane = threadIdx.x & 31;
   const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int nwarps = (gridDim.x * blockDim.x) >> 5;
@@ -974,13 +951,13 @@ void launch_sample(const GraphDev& g, LevelDev lv, int S, int k, const LevelDev*
   if (blocks > 148 * 8) blocks = 148 * 8;
   LevelDev nx{};
   if (next) nx = *next;
-  k_sample<<<blocks, 256, 0, st>>>(g, lv, S, k, nx, next ? 1 : 0, W, use_table, cnt, layer, err);
+  launch_k(k_sample, dim3(blocks), dim3(256), 0, st, g, lv, S, k, nx, next ? 1 : 0, W, use_table, cnt, layer, err);
 }
 
 // ---------------------------------------------------------------- row lookup
 // Layer l reads h^(l-1): x_i at l = 1 (Alg. 1 l.2-3), else the ring
 // slot of the target's unique entry at level l-1 (through inv, Alg. 1 l.20).
-__global__ void k_resolve(ResolveArgs a, int* err) {
+__global__ void k_resolve(ResolveArgs a, int* err) { pdl_enter();
   const int l = blockIdx.y + 1;
   const LevelDev& lv = a.lv[l];
   const LevelDev& pv = a.lv[l - 1];
@@ -1038,12 +1015,12 @@ void launch_resolve(const ResolveArgs& a, int* err, cudaStream_t st) {
   int bx = (int)((mx + 255) / 256);
   if (bx < 1) bx = 1;
   if (bx > 592) bx = 592;
-  k_resolve<<<dim3(bx, a.L), 256, 0, st>>>(a, err);
+  launch_k(k_resolve, dim3(dim3(bx, a.L)), dim3(256), 0, st, a, err);
 }
 
 // ------------------------------------------------------------------- misc
 __global__ void k_prep_nodes(const int32_t* __restrict__ nodes, const uint32_t* __restrict__ ts, int n,
-                             LevelDev top) {
+                             LevelDev top) { pdl_enter();
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
     top.in_node[i] = nodes[i];
     top.in_ts[i] = ts[i];
@@ -1054,11 +1031,11 @@ __global__ void k_prep_nodes(const int32_t* __restrict__ nodes, const uint32_t* 
 void launch_prep_nodes(const int32_t* nodes, const uint32_t* ts, int n, LevelDev top, cudaStream_t st) {
   int blocks = n > 0 ? (n + 255) / 256 : 1;
   if (blocks > 592) blocks = 592;
-  k_prep_nodes<<<blocks, 256, 0, st>>>(nodes, ts, n, top);
+  launch_k(k_prep_nodes, dim3(blocks), dim3(256), 0, st, nodes, ts, n, top);
 }
 
 __global__ void k_finish(long long* __restrict__ cnt_sb, int S, long long* __restrict__ total,
-                         long long* __restrict__ log, int64_t row0) {
+                         long long* __restrict__ log, int64_t row0) { pdl_enter();
   for (int i = threadIdx.x; i < S * TG_NCOUNTERS; i += blockDim.x) {
     const long long v = cnt_sb[i];
     if (v) atomicAdd((unsigned long long*)(total + i % TG_NCOUNTERS), (unsigned long long)v);
@@ -1069,7 +1046,7 @@ __global__ void k_finish(long long* __restrict__ cnt_sb, int S, long long* __res
 
 void launch_finish(long long* cnt_sb, int S, long long* total, long long* log, int64_t log_row0,
                    cudaStream_t st) {
-  k_finish<<<1, 1024, 0, st>>>(cnt_sb, S, total, log, log_row0);
+  launch_k(k_finish, dim3(1), dim3(1024), 0, st, cnt_sb, S, total, log, log_row0);
 }
 
 }  // namespace tg

@@ -252,6 +252,7 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t* v) {
 template <int PREC>
 __global__ void __launch_bounds__(TC_THREADS, 1)
     k_gemm_tc(GemmArgs g, TcWeights w, int stages, const __grid_constant__ CUtensorMap tmA, int a_tma) {
+  pdl_enter();
   constexpr int EPC = PREC == TG_PREC_BF16 ? 64 : 32;
   constexpr int PLANES = PREC == TG_PREC_TF32X3 ? 2 : 1;
   constexpr int NV = EPC / 4;  // float4 loads per row per k-block
@@ -647,21 +648,21 @@ void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaSt
       cudaFuncSetAttribute(k_gemm_tc<TG_PREC_BF16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       set = smem;
     }
-    k_gemm_tc<TG_PREC_BF16><<<grid, TC_THREADS, smem, st>>>(g, w, stages, tm, a_tma);
+    launch_k(k_gemm_tc<TG_PREC_BF16>, dim3(grid), dim3(TC_THREADS), smem, st, g, w, stages, tm, a_tma);
   } else if (precision == TG_PREC_TF32) {
     static size_t set = 0;
     if (smem > set) {
       cudaFuncSetAttribute(k_gemm_tc<TG_PREC_TF32>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       set = smem;
     }
-    k_gemm_tc<TG_PREC_TF32><<<grid, TC_THREADS, smem, st>>>(g, w, stages, tm, a_tma);
+    launch_k(k_gemm_tc<TG_PREC_TF32>, dim3(grid), dim3(TC_THREADS), smem, st, g, w, stages, tm, a_tma);
   } else {
     static size_t set = 0;
     if (smem > set) {
       cudaFuncSetAttribute(k_gemm_tc<TG_PREC_TF32X3>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       set = smem;
     }
-    k_gemm_tc<TG_PREC_TF32X3><<<grid, TC_THREADS, smem, st>>>(g, w, stages, tm, 0);
+    launch_k(k_gemm_tc<TG_PREC_TF32X3>, dim3(grid), dim3(TC_THREADS), smem, st, g, w, stages, tm, 0);
   }
 }
 

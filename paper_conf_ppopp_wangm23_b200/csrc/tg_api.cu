@@ -16,6 +16,14 @@
 
 using namespace tg;
 
+bool tg::pdl_enabled() {
+  static const bool on = [] {
+    const char* e = getenv("TG_PDL");
+    return !(e && e[0] == '0');
+  }();
+  return on;
+}
+
 namespace {
 
 struct LayerW {
@@ -688,20 +696,27 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
   const int64_t per_layer = 4LL * D * D + 3LL * D + (int64_t)d_n * (D + d_n) + d_n + (int64_t)d_n * d_n + d_n;
   const int64_t expect = L * per_layer + 2LL * d_t + 2LL * d_n * d_n + d_n + d_n + 1;
   if (n_params != expect) return TG_EINVAL;
-  const int S = cfg->superbatch ? cfg->superbatch : 16;
+  int S = cfg->superbatch ? cfg->superbatch : 16;
   // per-batch capacities: I_L = targets; I_{l-1} = C_l (k+1) <= I_l (k+1)
   int cap[TG_MAX_LAYERS + 1];
   int64_t cc = cfg->max_batch_targets;
   cap[L] = (int)cc;
   for (int l = L - 1; l >= 1; --l) {
     cc = cc * (k + 1);
-    if (cc * S > ((int64_t)1 << 26)) return TG_EINVAL;
+    if (cc > ((int64_t)1 << 26)) return TG_EINVAL;
     cap[l] = (int)cc;
   }
   for (int l = 1; l <= L; ++l) {
     if (cap[l] > 16 * 10000) return TG_EINVAL;                   // dedup cluster bound
-    if (cap[l] > 1024 * kProbeIPT) return TG_EINVAL;             // probe CTA bound
+    if (cap[l] > kSeqCLMax * 1024 * kProbeIPT) return TG_EINVAL; // ordered cache pass bound
   }
+  // every key of a superbatch's cached level must fit the cache passes' DSMEM hash
+  // (load <= 0.6): S shrinks for large batches (batch 2,000 at k = 20 -> S = 1)
+  for (int l = 1; l < L; ++l) {
+    const int64_t fit = (int64_t)kSeqCLMax * kSeqSlotsPerCTA * 6 / 10 / cap[l];
+    if (fit < S) S = fit < 1 ? 1 : (int)fit;
+  }
+  if ((int64_t)cap[1] * S > ((int64_t)1 << 26)) return TG_EINVAL;
   if (cudaSetDevice(ctx->device) != cudaSuccess) return TG_ECUDA;
   ctx->cfg = *cfg;
   ctx->S = S;

@@ -32,6 +32,61 @@ constexpr int kDedupThreads = 1024;
 constexpr int kDedupIPT = 16;      // items per thread per CTA (ordered scan)
 constexpr int kDedupSlots = 16384; // smem hash slots per CTA (load <= ~0.6)
 constexpr int kProbeIPT = 16;
+constexpr int kSeqCLMax = 16;        // cluster CTAs of the ordered cache passes
+constexpr int kSeqSlotsPerCTA = 16384; // their DSMEM hash slots per CTA
+
+// ---- programmatic dependent launch (PDL). Every kernel of the hot path is
+// launched with programmatic stream serialization, so its CTAs may become
+// resident while the previous kernel of the same stream drains. Each kernel
+// calls pdl_wait() before its first global-memory access (read OR write: the
+// predecessor may still read what this kernel overwrites) -- it returns once
+// the predecessor grid has completed and its writes are visible -- and then
+// pdl_trigger(), which lets the *next* kernel start its own prologue. Only
+// shared-memory / TMEM / barrier setup and kernel parameters are touched
+// before pdl_wait(). Without a programmatic predecessor both are no-ops.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;\n" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;\n" ::: "memory"); }
+__device__ __forceinline__ void pdl_enter() {
+  pdl_wait();
+  pdl_trigger();
+}
+bool pdl_enabled();  // TG_PDL=0 disables (A/B measurement)
+
+// cudaLaunchKernelEx with the PDL attribute (+ an optional cluster size)
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_k(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                            Args... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
+}
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_k_cluster(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                                    int cluster_x, Args... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[2];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
+  at[1].id = cudaLaunchAttributeClusterDimension;
+  at[1].val.clusterDim.x = cluster_x;
+  at[1].val.clusterDim.y = 1;
+  at[1].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 2;
+  return cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
+}
 
 // device error bits (sticky)
 enum : int { kErrNodeRange = 1, kErrIndexFull = 2, kErrDedupFull = 4, kErrEidRange = 8 };

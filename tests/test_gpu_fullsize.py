@@ -1,0 +1,130 @@
+"""Parity at BASELINE.json's full sizes, in the launch configuration bench.py times.
+
+Each whole stream (configs[1..4]) runs through ``tg_score_stream`` exactly as ``bench.py``
+launches it (superbatch S = 16, the bench's precision), cold cache. The plain oracle
+(oracle/tgat.py) then recomputes a stratified sample of batches one by one -- valid because every
+batch's scores are a pure function of (graph, weights, batch) -- and the
+per-batch counters of the whole stream are compared bit-exactly with the Alg. 1/3 bookkeeping
+simulator (oracle/tgopt.py, compute=False), FIFO eviction included where the stream's key
+universe exceeds the 2M-item limit (LastFM: 2E+1 = 2.59M keys).
+
+Tolerances (north_star, R17): fp32-level modes |d| <= 1e-5 + 1e-4|ref|; bf16 GEMM operands
+rtol = atol = 2e-2.
+"""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+
+from tests.gpu_helpers import close, setup, make_ctx, make_oracle
+
+pytestmark = pytest.mark.gpu
+TOL = {1: (1e-4, 1e-5), 2: (2e-2, 2e-2)}   # tf32x3 / bf16
+BENCH_S = 16                               # bench.py's superbatch
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _need_gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_ppopp_wangm23_b200 import lib
+    lib()
+
+
+def _run(ctx, s, batch, E=None):
+    from paper_conf_ppopp_wangm23_b200 import TG_NCOUNTERS
+    E = s.n_edges if E is None else E
+    nb = (E + batch - 1) // batch
+    d = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    scores = torch.full((E,), -1.0, dtype=torch.float32, device="cuda")
+    log = torch.zeros(nb * TG_NCOUNTERS, dtype=torch.int64, device="cuda")
+    ctx.score_stream(d(s.src[:E]), d(s.dst[:E]), d(s.ts[:E].view(np.int32)), batch, scores, log)
+    torch.cuda.synchronize()
+    return scores.cpu().numpy(), log.cpu().numpy().reshape(nb, TG_NCOUNTERS)
+
+
+def _picks(nb, extra=()):
+    """Stratified batch sample: first, second, evenly spaced interior, last (R13 partial)."""
+    return sorted(set([0, 1, nb // 4, nb // 2, (3 * nb) // 4, nb - 1] + list(extra)))
+
+
+def _check_scores(s, flat, mc, scores, picks, prec):
+    o = make_oracle(s, flat, mc)
+    for b in picks:
+        lo, hi = b * mc.batch, min((b + 1) * mc.batch, s.n_edges)
+        _, ref = o.infer_batch(s.src[lo:hi], s.dst[lo:hi], s.ts[lo:hi])
+        ok, err, nbad = close(scores[lo:hi], ref, *TOL[prec])
+        assert ok, (b, err, nbad)
+
+
+def _check_counters(s, flat, mc, log, limit):
+    from oracle.tgopt import TGOptSim
+    from paper_conf_ppopp_wangm23_b200 import counters_dict
+    sim = TGOptSim(make_oracle(s, flat, mc), cache_limit=limit, time_window=mc.time_window,
+                   compute=False)
+    for b, lo in enumerate(range(0, s.n_edges, mc.batch)):
+        hi = min(lo + mc.batch, s.n_edges)
+        sim.reset_counters()
+        sim.infer_batch(s.src[lo:hi], s.dst[lo:hi], s.ts[lo:hi])
+        want = sim.counters()
+        got = counters_dict(log[b], mc.n_layers)
+        assert got == want, (b, {k: (got[k], want[k]) for k in want if got[k] != want[k]})
+    return sim
+
+
+@pytest.mark.parametrize("name", ["reddit", "wiki", "mooc"])
+def test_fullsize_stream_bench_config(name):
+    """Whole stream, bench launch config (bf16, S = 16): sampled scores vs the plain oracle and
+    every batch's counters vs the Alg. 1/3 simulator, bit-exact."""
+    cfg, s, flat = setup(name)
+    mc = cfg.model
+    ctx = make_ctx(s, flat, mc, precision=2, superbatch=BENCH_S)
+    scores, log = _run(ctx, s, mc.batch)
+    assert np.isfinite(scores).all() and (scores >= 0).all() and (scores <= 1).all()
+    nb = log.shape[0]
+    _check_scores(s, flat, mc, scores, _picks(nb), 2)
+    _check_counters(s, flat, mc, log, mc.cache_limit)
+    from paper_conf_ppopp_wangm23_b200 import counters_dict
+    assert ctx.counters()["l1_misses"] == sum(counters_dict(r, mc.n_layers)["l1_misses"] for r in log)
+    ctx.close()
+
+
+def test_fullsize_reddit_fp32_level():
+    """Reddit stream in the fp32-level tensor-core mode (3xTF32): sampled scores at 1e-4/1e-5."""
+    cfg, s, flat = setup("reddit")
+    mc = cfg.model
+    ctx = make_ctx(s, flat, mc, precision=1, superbatch=BENCH_S)
+    scores, _ = _run(ctx, s, mc.batch)
+    _check_scores(s, flat, mc, scores, _picks(scores.size // mc.batch + 1), 1)
+    ctx.close()
+
+
+def test_fullsize_lastfm_fifo_eviction():
+    """LastFM-shaped stream (1.29M edges): 2E+1 > the 2M limit, so FIFO eviction happens inside
+    the pass (Alg. 3 l.1-4, R11). Counters (evictions included) bit-exact for every batch;
+    sampled scores after the first eviction vs the plain oracle."""
+    cfg, s, flat = setup("lastfm")
+    mc = cfg.model
+    ctx = make_ctx(s, flat, mc, precision=2, superbatch=BENCH_S)
+    scores, log = _run(ctx, s, mc.batch)
+    _check_counters(s, flat, mc, log, mc.cache_limit)
+    from paper_conf_ppopp_wangm23_b200 import counters_dict
+    ev = np.array([counters_dict(r, mc.n_layers)["l1_evicted"] for r in log])
+    assert ev.sum() > 0, "stream should exercise FIFO eviction"
+    first = int(np.argmax(ev > 0))
+    nb = log.shape[0]
+    _check_scores(s, flat, mc, scores, _picks(nb, [first, first + 1, (first + nb) // 2]), 2)
+    ctx.close()
+
+
+def test_fullsize_large_batch2000():
+    """configs[4] shape (1M nodes, 10M edges, batch 2,000), one rank's share of the 8-way split:
+    the first 1/8 of the stream, cold cache; sampled batches vs the plain oracle."""
+    cfg, s, flat = setup("large")
+    mc = cfg.model
+    E8 = (s.n_edges // 8 // mc.batch) * mc.batch
+    ctx = make_ctx(s, flat, mc, precision=2, superbatch=BENCH_S, max_targets=2 * mc.batch)
+    scores, log = _run(ctx, s, mc.batch, E8)       # the graph holds the whole stream (R14)
+    nb = log.shape[0]
+    _check_scores(s, flat, mc, scores, [0, nb // 2, nb - 1], 2)
+    ctx.close()

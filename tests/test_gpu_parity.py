@@ -121,6 +121,7 @@ def test_time_encode_table_equals_direct_and_oracle():
     o = make_oracle(s, flat, cfg.model)
     rng = np.random.default_rng(2)
     delta = np.concatenate([np.arange(0, 10_000), rng.integers(0, 3_000_000_000, 20_000),
+                            rng.integers(10_000, 4_000_000, 20_000),  # fp32-reduced range
                             np.array([2**24 + 1, 2**31 + 5, 0])]).astype(np.int64)
     n = delta.size
     d_t = s.d_n
