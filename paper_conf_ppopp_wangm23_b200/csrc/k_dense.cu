@@ -94,22 +94,42 @@ void launch_gemm_simt(const GemmArgs& g, cudaStream_t st) {
 }
 
 // ---------------------------------------------------------------- LayerNorm
-__global__ void k_layernorm(const float* __restrict__ y, float* __restrict__ r, int Dp, int dn, int dnp, int de,
-                            int dep, int dt, const float* __restrict__ gamma, const float* __restrict__ beta,
-                            const int* __restrict__ m_dev, const float* const* __restrict__ hs_rows,
-                            const float* __restrict__ phi0, unsigned short* __restrict__ rh, int ldrh) { pdl_enter();
+// r = LN(y + q; gamma, beta) with q = [h^(l-1) | 0 | Phi(0)] (Eq. 4/6, R1, R3),
+// mean and biased variance over the D valid columns, eps 1e-5. Warp per row;
+// per-column parameters (gamma, beta, valid weight, Phi(0) block of q) are
+// staged in shared memory once per CTA; the grid is one resident wave that
+// strides over the rows. Outputs: fp32 r [M x Dp] and/or the bf16 merge-FFN
+// input row rh = [LN(y) (Dp) | 0 | h^(l-1) at rh_off (16-byte aligned) | 0] (Eq. 7).
+constexpr int kLnMaxD4 = 256;  // Dp <= 1024 (checked at model load)
+__global__ void __launch_bounds__(256, 4)
+    k_layernorm(const float* __restrict__ y, float* __restrict__ r, int Dp, int dn, int dnp, int de, int dep, int dt,
+                const float* __restrict__ gamma, const float* __restrict__ beta, const int* __restrict__ m_dev,
+                const float* const* __restrict__ hs_rows, const float* __restrict__ phi0,
+                unsigned short* __restrict__ rh, int ldrh, int rh_off) {
+  __shared__ float4 s_g[kLnMaxD4], s_b[kLnMaxD4], s_w[kLnMaxD4], s_q[kLnMaxD4];
+  const int D4 = Dp >> 2;
+  const int s1 = dnp, s2 = dnp + dep;
+  for (int q = threadIdx.x; q < D4; q += blockDim.x) {  // parameters only: before the PDL wait
+    s_g[q] = reinterpret_cast<const float4*>(gamma)[q];
+    s_b[q] = reinterpret_cast<const float4*>(beta)[q];
+    float w[4];
+    for (int i = 0; i < 4; ++i) {
+      const int c = 4 * q + i;
+      w[i] = (c < dn || (c >= s1 && c < s1 + de) || (c >= s2 && c < s2 + dt)) ? 1.f : 0.f;
+    }
+    s_w[q] = make_float4(w[0], w[1], w[2], w[3]);
+    s_q[q] = 4 * q >= s2 ? reinterpret_cast<const float4*>(phi0)[q - (s2 >> 2)] : make_float4(0.f, 0.f, 0.f, 0.f);
+  }
+  pdl_enter();
+  __syncthreads();
   const int M = *m_dev;
   const int lane = threadIdx.x & 31;
   const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, nw = (gridDim.x * blockDim.x) >> 5;
-  const int D = dn + de + dt;
-  const int s1 = dnp, s2 = dnp + dep;
-  const int D4 = Dp >> 2;
-  // warp per row; the row (<= 1024 floats) is read once into registers
+  const float D = (float)(dn + de + dt);
+  const int nh4 = dnp >> 2;
   for (int row = warp; row < M; row += nw) {
     const float4* yr = reinterpret_cast<const float4*>(y + (size_t)row * Dp);
     const float4* hr = reinterpret_cast<const float4*>(hs_rows[row]);
-    const float4* p0 = reinterpret_cast<const float4*>(phi0);
-    float4* rr = r ? reinterpret_cast<float4*>(r + (size_t)row * Dp) : nullptr;
     float4 v[8];
     float sum = 0.f;
 #pragma unroll
@@ -117,55 +137,41 @@ __global__ void k_layernorm(const float* __restrict__ y, float* __restrict__ r, 
       const int q = lane + 32 * j;
       v[j] = make_float4(0.f, 0.f, 0.f, 0.f);
       if (q < D4) {
-        v[j] = yr[q];
-        // + q = [h^(l-1) || 0 || Phi(0)] (padded columns of each part are zero)
-        float4 a = make_float4(0.f, 0.f, 0.f, 0.f);
-        if (4 * q < dnp) a = hr[q];
-        else if (4 * q >= s2) a = p0[q - (s2 >> 2)];
-        v[j].x += a.x;
-        v[j].y += a.y;
-        v[j].z += a.z;
-        v[j].w += a.w;
-        // padded columns are exact zeros (zero weight rows / bias), so they do not bias the sum
-        sum += (v[j].x + v[j].y) + (v[j].z + v[j].w);
+        const float4 a = yr[q];
+        const float4 b = q < nh4 ? hr[q] : s_q[q];  // + q = [h || 0 || Phi(0)] (pads are zero)
+        v[j] = make_float4(a.x + b.x, a.y + b.y, a.z + b.z, a.w + b.w);
+        sum += (v[j].x + v[j].y) + (v[j].z + v[j].w);  // padded columns are exact zeros
       }
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
-    const float mu = sum / (float)D;
+    const float mu = sum / D;
     float var = 0.f;
 #pragma unroll
     for (int j = 0; j < 8; ++j) {
       const int q = lane + 32 * j;
       if (q < D4) {
-        const float e[4] = {v[j].x, v[j].y, v[j].z, v[j].w};
-#pragma unroll
-        for (int i = 0; i < 4; ++i) {
-          const int c = 4 * q + i;
-          const bool valid = c < dn || (c >= s1 && c < s1 + de) || (c >= s2 && c < s2 + dt);
-          const float d = e[i] - mu;
-          if (valid) var = fmaf(d, d, var);
-        }
+        const float4 w = s_w[q];
+        const float dx = v[j].x - mu, dy = v[j].y - mu, dz = v[j].z - mu, dw = v[j].w - mu;
+        var = fmaf(w.x * dx, dx, var);
+        var = fmaf(w.y * dy, dy, var);
+        var = fmaf(w.z * dz, dz, var);
+        var = fmaf(w.w * dw, dw, var);
       }
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) var += __shfl_xor_sync(0xffffffffu, var, o);
-    const float rstd = rsqrtf(var / (float)D + 1e-5f);
+    const float rstd = rsqrtf(var / D + 1e-5f);
 #pragma unroll
     for (int j = 0; j < 8; ++j) {
       const int q = lane + 32 * j;
       if (q < D4) {
-        const float e[4] = {v[j].x, v[j].y, v[j].z, v[j].w};
-        float o4[4];
-#pragma unroll
-        for (int i = 0; i < 4; ++i) {
-          const int c = 4 * q + i;
-          const bool valid = c < dn || (c >= s1 && c < s1 + de) || (c >= s2 && c < s2 + dt);
-          o4[i] = valid ? (e[i] - mu) * rstd * gamma[c] + beta[c] : 0.f;
-        }
-        if (rr) rr[q] = make_float4(o4[0], o4[1], o4[2], o4[3]);
+        const float4 g = s_g[q], b = s_b[q];  // zero on padded columns -> output 0 there
+        const float4 o4 = make_float4(fmaf((v[j].x - mu) * rstd, g.x, b.x), fmaf((v[j].y - mu) * rstd, g.y, b.y),
+                                      fmaf((v[j].z - mu) * rstd, g.z, b.z), fmaf((v[j].w - mu) * rstd, g.w, b.w));
+        if (r) reinterpret_cast<float4*>(r + (size_t)row * Dp)[q] = o4;
         if (rh) {
-          __nv_bfloat162 lo = __floats2bfloat162_rn(o4[0], o4[1]), hi = __floats2bfloat162_rn(o4[2], o4[3]);
+          __nv_bfloat162 lo = __floats2bfloat162_rn(o4.x, o4.y), hi = __floats2bfloat162_rn(o4.z, o4.w);
           uint2 pk;
           pk.x = *reinterpret_cast<uint32_t*>(&lo);
           pk.y = *reinterpret_cast<uint32_t*>(&hi);
@@ -173,10 +179,11 @@ __global__ void k_layernorm(const float* __restrict__ y, float* __restrict__ r, 
         }
       }
     }
-    if (rh) {  // [LN(y) | h^(l-1) | 0]: the merge-FFN input (Eq. 7) as one bf16 row
+    if (rh) {  // [Dp, ldrh): zeros, h^(l-1) at rh_off, zeros
+      const int q0 = (rh_off - Dp) >> 2;
       for (int q = lane; 4 * q < ldrh - Dp; q += 32) {
         float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
-        if (4 * q < dnp) x = hr[q];
+        if (q >= q0 && q - q0 < nh4) x = hr[q - q0];
         __nv_bfloat162 lo = __floats2bfloat162_rn(x.x, x.y), hi = __floats2bfloat162_rn(x.z, x.w);
         uint2 pk;
         pk.x = *reinterpret_cast<uint32_t*>(&lo);
@@ -189,13 +196,13 @@ __global__ void k_layernorm(const float* __restrict__ y, float* __restrict__ r, 
 
 void launch_layernorm(const float* y, float* r, int Dp, int dn, int dnp, int de, int dep, int dt,
                       const float* gamma, const float* beta, const int* m_dev, int m_max,
-                      const float* const* hs_rows, const float* phi0, unsigned short* rh, int ldrh,
+                      const float* const* hs_rows, const float* phi0, unsigned short* rh, int ldrh, int rh_off,
                       cudaStream_t st) {
-  int blocks = (m_max * 32 + 255) / 256;
+  int blocks = (m_max + 7) / 8;  // 8 warps (rows) per CTA
+  if (blocks > 148 * 4) blocks = 148 * 4;  // one resident wave (4 CTAs / SM at <= 64 registers)
   if (blocks < 1) blocks = 1;
-  if (blocks > 1184) blocks = 1184;
-  launch_k(k_layernorm, dim3(blocks), dim3(256), 0, st, y, r, Dp, dn, dnp, de, dep, dt, gamma, beta, m_dev, hs_rows, phi0, rh,
-                                      ldrh);
+  launch_k(k_layernorm, dim3(blocks), dim3(256), 0, st, y, r, Dp, dn, dnp, de, dep, dt, gamma, beta, m_dev, hs_rows,
+           phi0, rh, ldrh, rh_off);
 }
 
 // -------------------------------------------------------------------- score

@@ -21,6 +21,8 @@
 // cores. TG_PREC_BF16: kind::f16 with bf16 operands, fp32 accumulation.
 #include <cuda_bf16.h>
 
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <vector>
 
@@ -52,9 +54,14 @@ constexpr int TC_BAR_BYTES = 256;
 constexpr int TC_STG_LD = 20;  // floats per staged row (16 columns + pad)
 constexpr int TC_EPI_BYTES = TC_EPI_WARPS * 32 * TC_STG_LD * 4;
 
-static inline int tc_stages(int prec, int BN) {
+// fused-LayerNorm epilogue (g.ln): per-row partial statistics of the two
+// column halves [2][128] and the cluster exchange buffers [2 parities][4 N tiles][128]
+constexpr int TC_LN_MAXTN = 4;
+constexpr int TC_LN_BYTES = (2 * 128 + 2 * TC_LN_MAXTN * 128) * 16 + 4 * 256 * 4;  // + bias, gamma, beta, valid
+
+static inline int tc_stages(int prec, int BN, int ln = 0) {
   const size_t st = (size_t)tc_planes(prec) * ((size_t)TC_BM * 128 + (size_t)BN * 128);
-  const size_t budget = tc_ctas_per_sm(prec) == 1 ? 205 * 1024 : 100 * 1024;
+  const size_t budget = (tc_ctas_per_sm(prec) == 1 ? 205 * 1024 : 100 * 1024) - (ln ? TC_LN_BYTES : 0);
   int s = (int)(budget / st);
   if (s > TC_MAXSTAGES) s = TC_MAXSTAGES;
   return s < 2 ? 2 : s;
@@ -207,6 +214,57 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
         : "memory");
   }
 }
+// cluster-scope variants for the LayerNorm statistics exchange (DSMEM)
+__device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity) {
+  const uint32_t a = smem_u32(bar);
+  uint32_t done = 0;
+  while (!done) {
+    asm volatile(
+        "{\n\t.reg .pred P1;\n\t"
+        "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 P1, [%1], %2;\n\t"
+        "selp.b32 %0, 1, 0, P1;\n\t}\n"
+        : "=r"(done)
+        : "r"(a), "r"(parity)
+        : "memory");
+  }
+}
+__device__ __forceinline__ uint32_t mapa_u32(uint32_t local, uint32_t rank) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;\n" : "=r"(r) : "r"(local), "r"(rank));
+  return r;
+}
+__device__ __forceinline__ void st_cluster_v4(uint32_t addr, float4 v) {
+  asm volatile("st.shared::cluster.v4.f32 [%0], {%1, %2, %3, %4};\n" ::"r"(addr), "f"(v.x), "f"(v.y), "f"(v.z),
+               "f"(v.w)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_remote(uint32_t addr) {
+  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];\n" ::"r"(addr) : "memory");
+}
+// Chan et al. pairwise merge of (count, mean, M2) running statistics; fixed
+// merge order keeps every row's result independent of the batch (row-invariant)
+__device__ __forceinline__ void chan_merge(float& n, float& m, float& M2, float nb, float mb, float Mb) {
+  if (nb == 0.f) return;
+  if (n == 0.f) {
+    n = nb;
+    m = mb;
+    M2 = Mb;
+    return;
+  }
+  const float nn = n + nb, d = mb - m;
+  m = m + d * (nb / nn);
+  M2 = M2 + Mb + d * d * (n * nb / nn);
+  n = nn;
+}
+__device__ __forceinline__ bool ln_valid(const GemmArgs& g, int c) {
+  return c < g.N && (c < g.ln_dn || (c >= g.ln_s1 && c < g.ln_s1 + g.ln_de) || (c >= g.ln_s2 && c < g.ln_s2 + g.ln_dt));
+}
+// accumulator chunk (16 columns from local column cl) + bias (staged in shared memory)
+__device__ __forceinline__ void ln_chunk(const uint32_t (&v)[16], const float* s_bias, int cl, float (&x)[16]) {
+#pragma unroll
+  for (int j = 0; j < 16; ++j) x[j] = __uint_as_float(v[j]) + s_bias[cl + j];
+}
+
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
   asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n" ::"r"(
                    smem_u32(dst)),
@@ -251,7 +309,8 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t* v) {
 
 template <int PREC>
 __global__ void __launch_bounds__(TC_THREADS, 1)
-    k_gemm_tc(GemmArgs g, TcWeights w, int stages, const __grid_constant__ CUtensorMap tmA, int a_tma) {
+    k_gemm_tc(GemmArgs g, TcWeights w, int stages, const __grid_constant__ CUtensorMap tmA, int a_tma,
+              const __grid_constant__ CUtensorMap tmA2, int a2_kb0, int a2_x0) {
   pdl_enter();
   constexpr int EPC = PREC == TG_PREC_BF16 ? 64 : 32;
   constexpr int PLANES = PREC == TG_PREC_TF32X3 ? 2 : 1;
@@ -269,6 +328,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   uint64_t* tfull = empty + TC_MAXSTAGES;   // [2]
   uint64_t* tempty = tfull + 2;             // [2]
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+  uint64_t* lnbar = tempty + 3;             // [2] LayerNorm statistics exchange (g.ln)
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
 #ifdef TG_TC_TRACE
   const long long t_entry = clock64();
@@ -297,6 +357,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     for (int a = 0; a < 2; ++a) {
       mbar_init(&tfull[a], 1);     // MMA commit after the tile's last k-block
       mbar_init(&tempty[a], TC_EPI_WARPS * 32);  // epilogue threads drained the accumulator
+      if (g.ln) mbar_init(&lnbar[a], w.ntn * TC_BM);  // one arrival per row from each CTA of the cluster
     }
     asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
   }
@@ -308,6 +369,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   asm volatile("tcgen05.fence::before_thread_sync;\n");
   __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;\n");
+  if (g.ln) {  // peers arrive on this CTA's lnbar: initialised cluster-wide first
+    asm volatile("barrier.cluster.arrive.release.aligned;\n" ::: "memory");
+    asm volatile("barrier.cluster.wait.acquire.aligned;\n" ::: "memory");
+  }
   const uint32_t tmem = *tmem_slot;
   if (tid == 0) TCT(2, clock64());
 
@@ -448,11 +513,13 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           if (gk == 0) TCT(4, clock64());
           mbar_expect_tx(&full[s], PLANES * b_plane + (a_tma ? a_plane : 0u));
           if (a_tma) {  // A tile [128 rows x 128 B] of the dense activation, 128B-swizzled by TMA
-            const int x = kb * EPC, y = (t / w.ntn) * TC_BM;
+            // k-blocks >= a2_kb0 come from a second activation (columns a2_x0 + ...)
+            const bool second = kb >= a2_kb0;
+            const int x = second ? a2_x0 + (kb - a2_kb0) * EPC : kb * EPC, y = (t / w.ntn) * TC_BM;
             asm volatile(
                 "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], "
                 "[%4];\n" ::"r"(smem_u32(smem + s * stage_bytes)),
-                "l"(reinterpret_cast<uint64_t>(&tmA)), "r"(x), "r"(y), "r"(smem_u32(&full[s]))
+                "l"(reinterpret_cast<uint64_t>(second ? &tmA2 : &tmA)), "r"(x), "r"(y), "r"(smem_u32(&full[s]))
                 : "memory");
           }
           bulk_g2s(sB, src, PLANES * b_plane, &full[s]);
@@ -494,6 +561,137 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
                          smem_u32(&tfull[acc]))
                      : "memory");
         if (tc == 0) TCT(3, clock64());
+      }
+    }
+  } else if (g.ln) {
+    // ===================== epilogue with the fused LayerNorm (G2, Eq. 6: r = LN(W_fc o +
+    // b_fc + q), R1; the residual q = [h | 0 | Phi(0)] is already in the accumulator: h
+    // through the identity block of the augmented K, Phi(0) folded into the bias). The ntn
+    // CTAs of a cluster hold the ntn column tiles of the same 128 rows. Pass 1 reads the
+    // accumulator and reduces each row's (count, mean, M2) over its valid columns; the
+    // CTA's row statistics go to every CTA of the cluster through DSMEM (remote mbarrier
+    // arrive); pass 2 re-reads the accumulator, normalises with the merged statistics
+    // (fixed tile order) and stores the bf16 LN(y) block of the merge-FFN input (Eq. 7).
+    const int quad = warp & 3;
+    const int ew = warp - 6;
+    const int half = ew >> 2;
+    float* stg = reinterpret_cast<float*>(smem + stages * stage_bytes + TC_BAR_BYTES) + ew * (32 * TC_STG_LD);
+    float4* lnh = reinterpret_cast<float4*>(smem + stages * stage_bytes + TC_BAR_BYTES + TC_EPI_BYTES);  // [2][128]
+    float4* lnx = lnh + 2 * TC_BM;  // [2][TC_LN_MAXTN][128]
+    float* s_bias = reinterpret_cast<float*>(lnx + 2 * TC_LN_MAXTN * TC_BM);  // [BN] x 3
+    float* s_g = s_bias + 256;
+    float* s_b = s_g + 256;
+    float* s_w = s_b + 256;  // 1 for the valid LayerNorm columns of the tile, else 0 (gamma = beta = 0 there)
+    const int rq = lane >> 2, cq = lane & 3;
+    const int rloc = quad * 32 + lane;
+    const int ntn = w.ntn;
+    {  // this CTA's column tile is fixed (grid is a multiple of ntn)
+      const int nb0 = (int)(blockIdx.x % ntn) * BN;
+      for (int i = tid - 6 * 32; i < BN; i += TC_EPI_WARPS * 32) {
+        const int c = nb0 + i;
+        const bool in = c < g.N;
+        s_bias[i] = in ? g.bias[c] : 0.f;
+        s_g[i] = in ? g.ln_g[c] : 0.f;
+        s_b[i] = in ? g.ln_b[c] : 0.f;
+        s_w[i] = ln_valid(g, c) ? 1.f : 0.f;
+      }
+      asm volatile("bar.sync 1, %0;\n" ::"n"(TC_EPI_WARPS * 32) : "memory");
+    }
+    uint32_t tc = 0;
+    for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++tc) {
+      const int tm = t / ntn, tn = t - tm * ntn;
+      const int m0 = tm * TC_BM, n0 = tn * BN;
+      const uint32_t acc = tc & 1, par = tc & 1;
+      const int er = m0 + rloc;
+      unsigned short* hrow = er < M ? g.c_h + (size_t)er * g.ldc_h : nullptr;
+      mbar_wait(&tfull[acc], (tc >> 1) & 1);
+      asm volatile("tcgen05.fence::after_thread_sync;\n");
+      const uint32_t tacc = tmem + acc * tc_acc_cols(PREC) + ((uint32_t)(quad * 32) << 16);
+      // ---- pass 1: row statistics of this thread's column chunks
+      float sn = 0.f, sm = 0.f, sM = 0.f;
+      for (int c0 = 16 * half; c0 < BN; c0 += 32) {
+        uint32_t v[16];
+        tmem_ld16(tacc + (uint32_t)c0, v);
+        asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
+        float x[16];
+        ln_chunk(v, s_bias, c0, x);
+        float cs = 0.f, cn = 0.f;  // branch-free: weights s_w select the valid columns
+#pragma unroll
+        for (int j = 0; j < 16; ++j) {
+          cs = fmaf(s_w[c0 + j], x[j], cs);
+          cn += s_w[c0 + j];
+        }
+        if (cn > 0.f) {
+          const float cm = cs / cn;
+          float cM = 0.f;
+#pragma unroll
+          for (int j = 0; j < 16; ++j) {
+            const float d = x[j] - cm;
+            cM = fmaf(s_w[c0 + j] * d, d, cM);
+          }
+          chan_merge(sn, sm, sM, cn, cm, cM);
+        }
+      }
+      lnh[half * TC_BM + rloc] = make_float4(sn, sm, sM, 0.f);
+      asm volatile("bar.sync 1, %0;\n" ::"n"(TC_EPI_WARPS * 32) : "memory");
+      if (half == 0) {
+        const float4 o = lnh[TC_BM + rloc];
+        chan_merge(sn, sm, sM, o.x, o.y, o.z);
+        const float4 st4 = make_float4(sn, sm, sM, 0.f);
+        const uint32_t slot = smem_u32(lnx + (par * TC_LN_MAXTN + tn) * TC_BM + rloc);
+        for (int r = 0; r < ntn; ++r) st_cluster_v4(mapa_u32(slot, (uint32_t)r), st4);
+        const uint32_t bar = smem_u32(&lnbar[par]);
+        for (int r = 0; r < ntn; ++r) mbar_arrive_remote(mapa_u32(bar, (uint32_t)r));
+      }
+      mbar_wait_cluster(&lnbar[par], (tc >> 1) & 1);
+      float n = 0.f, mu = 0.f, M2 = 0.f;
+      for (int r = 0; r < ntn; ++r) {
+        const float4 o = lnx[(par * TC_LN_MAXTN + r) * TC_BM + rloc];
+        chan_merge(n, mu, M2, o.x, o.y, o.z);
+      }
+      const float rstd = rsqrtf(M2 / fmaxf(n, 1.f) + 1e-5f);
+      // ---- pass 2: normalise, transpose through shared memory, coalesced bf16 stores
+      bool released = false;
+      for (int c0 = 16 * half; c0 < BN; c0 += 32) {
+        uint32_t v[16];
+        tmem_ld16(tacc + (uint32_t)c0, v);
+        asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
+        if (c0 + 32 >= BN) {  // this warp's last chunk: hand the accumulator back
+          asm volatile("tcgen05.fence::before_thread_sync;\n");
+          mbar_arrive(&tempty[acc]);
+          released = true;
+        }
+        float x[16];
+        ln_chunk(v, s_bias, c0, x);
+#pragma unroll
+        for (int j = 0; j < 16; ++j)
+          x[j] = fmaf((x[j] - mu) * rstd, s_g[c0 + j], s_b[c0 + j]);  // 0 where gamma = beta = 0
+#pragma unroll
+        for (int j = 0; j < 4; ++j)
+          *reinterpret_cast<float4*>(stg + lane * TC_STG_LD + 4 * j) =
+              make_float4(x[4 * j], x[4 * j + 1], x[4 * j + 2], x[4 * j + 3]);
+        __syncwarp();
+        const int c = n0 + c0 + 4 * cq;
+        const bool cin = c0 + 4 * cq < BN && c < g.N;  // N % 4 == 0: all 4 or none
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const int r = rq + 8 * i;
+          const float4 y = *reinterpret_cast<const float4*>(stg + r * TC_STG_LD + 4 * cq);
+          unsigned short* hr =
+              reinterpret_cast<unsigned short*>(__shfl_sync(0xffffffffu, reinterpret_cast<long long>(hrow), r));
+          if (hr && cin) {
+            __nv_bfloat162 lo = __floats2bfloat162_rn(y.x, y.y), hi = __floats2bfloat162_rn(y.z, y.w);
+            uint2 pk;
+            pk.x = *reinterpret_cast<uint32_t*>(&lo);
+            pk.y = *reinterpret_cast<uint32_t*>(&hi);
+            *reinterpret_cast<uint2*>(hr + c) = pk;
+          }
+        }
+        __syncwarp();
+      }
+      if (!released) {
+        asm volatile("tcgen05.fence::before_thread_sync;\n");
+        mbar_arrive(&tempty[acc]);
       }
     }
   } else {
@@ -590,12 +788,17 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   if (tid == 0) TCT(7, clock64());
   if (tid == 6 * 32) TCT(55, clock64());
   asm volatile("tcgen05.fence::after_thread_sync;\n");
+  if (g.ln) {  // no CTA leaves while a peer may still address its shared memory
+    asm volatile("barrier.cluster.arrive.release.aligned;\n" ::: "memory");
+    asm volatile("barrier.cluster.wait.acquire.aligned;\n" ::: "memory");
+  }
   if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;\n" ::"r"(tmem), "r"(2 * tc_acc_cols(PREC)));
 }
 
-static size_t tc_smem(int prec, int BN, int stages) {
+static size_t tc_smem(int prec, int BN, int stages, int ln = 0) {
   const size_t planes = tc_planes(prec);
-  size_t s = 1024 + (size_t)stages * planes * ((size_t)TC_BM * 128 + (size_t)BN * 128) + TC_BAR_BYTES + TC_EPI_BYTES;
+  size_t s = 1024 + (size_t)stages * planes * ((size_t)TC_BM * 128 + (size_t)BN * 128) + TC_BAR_BYTES + TC_EPI_BYTES +
+             (ln ? TC_LN_BYTES : 0);
   // tf32x3: one CTA per SM (it allocates all 512 TMEM columns; a second
   // co-resident CTA would block in tcgen05.alloc until the first one exits).
   const size_t one_per_sm = 120 * 1024;
@@ -632,14 +835,20 @@ tg_status tc_make_tensor_a(const void* base, int elem_bytes, int ld, int rows, T
   return TG_OK;
 }
 
-void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaStream_t st, const TcTensorA* ta) {
+void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaStream_t st, const TcTensorA* ta,
+                    const TcTensorA* ta2, int a2_kb0, int a2_x0) {
   static const CUtensorMap zero_map{};
   const CUtensorMap& tm = (ta && ta->valid) ? ta->map : zero_map;
   const int a_tma = (ta && ta->valid) ? 1 : 0;
-  const int stages = tc_stages(precision, w.BN);
-  const size_t smem = tc_smem(precision, w.BN, stages);
+  const bool two = a_tma && ta2 && ta2->valid;
+  const CUtensorMap& tm2 = two ? ta2->map : zero_map;
+  if (!two) a2_kb0 = 1 << 30;
+  const int ln = g.ln ? 1 : 0;
+  const int stages = tc_stages(precision, w.BN, ln);
+  const size_t smem = tc_smem(precision, w.BN, stages, ln);
   const int tiles = ((g.m_max + TC_BM - 1) / TC_BM) * w.ntn;
-  const int slots = 148 * tc_ctas_per_sm(precision);
+  int slots = 148 * tc_ctas_per_sm(precision);
+  if (ln) slots = slots / w.ntn * w.ntn;  // whole clusters; a cluster walks the M tiles in lockstep
   int grid = tiles < slots ? tiles : slots;
   if (grid < 1) grid = 1;
   if (precision == TG_PREC_BF16) {
@@ -648,21 +857,52 @@ void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaSt
       cudaFuncSetAttribute(k_gemm_tc<TG_PREC_BF16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       set = smem;
     }
-    launch_k(k_gemm_tc<TG_PREC_BF16>, dim3(grid), dim3(TC_THREADS), smem, st, g, w, stages, tm, a_tma);
+    if (ln) {  // as many clusters as can be co-resident (GPC sizes), each walks M tiles
+      static int max_cl = -1;
+      static int max_cl_smem = -1;
+      if (max_cl_smem != (int)smem) {
+        cudaLaunchConfig_t oc = {};
+        oc.gridDim = dim3(grid);
+        oc.blockDim = dim3(TC_THREADS);
+        oc.dynamicSmemBytes = smem;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeClusterDimension;
+        at[0].val.clusterDim.x = w.ntn;
+        at[0].val.clusterDim.y = 1;
+        at[0].val.clusterDim.z = 1;
+        oc.attrs = at;
+        oc.numAttrs = 1;
+        int n = 0;
+        if (cudaOccupancyMaxActiveClusters(&n, k_gemm_tc<TG_PREC_BF16>, &oc) != cudaSuccess) n = 0;
+        cudaGetLastError();
+        max_cl = n;
+        max_cl_smem = (int)smem;
+        if (getenv("TG_VERBOSE")) fprintf(stderr, "libtg: LN GEMM max active clusters of %d: %d (smem %zu)\n", w.ntn, n, smem);
+      }
+      if (max_cl > 0 && grid > max_cl * w.ntn) grid = max_cl * w.ntn;
+    }
+    if (ln)
+      launch_k_cluster(k_gemm_tc<TG_PREC_BF16>, dim3(grid), dim3(TC_THREADS), smem, st, w.ntn, g, w, stages, tm,
+                       a_tma, tm2, a2_kb0, a2_x0);
+    else
+      launch_k(k_gemm_tc<TG_PREC_BF16>, dim3(grid), dim3(TC_THREADS), smem, st, g, w, stages, tm, a_tma, tm2,
+               a2_kb0, a2_x0);
   } else if (precision == TG_PREC_TF32) {
     static size_t set = 0;
     if (smem > set) {
       cudaFuncSetAttribute(k_gemm_tc<TG_PREC_TF32>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       set = smem;
     }
-    launch_k(k_gemm_tc<TG_PREC_TF32>, dim3(grid), dim3(TC_THREADS), smem, st, g, w, stages, tm, a_tma);
+    launch_k(k_gemm_tc<TG_PREC_TF32>, dim3(grid), dim3(TC_THREADS), smem, st, g, w, stages, tm, a_tma, tm2,
+             a2_kb0, a2_x0);
   } else {
     static size_t set = 0;
     if (smem > set) {
       cudaFuncSetAttribute(k_gemm_tc<TG_PREC_TF32X3>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       set = smem;
     }
-    launch_k(k_gemm_tc<TG_PREC_TF32X3>, dim3(grid), dim3(TC_THREADS), smem, st, g, w, stages, tm, 0);
+    launch_k(k_gemm_tc<TG_PREC_TF32X3>, dim3(grid), dim3(TC_THREADS), smem, st, g, w, stages, tm, 0, tm2,
+             1 << 30, 0);
   }
 }
 

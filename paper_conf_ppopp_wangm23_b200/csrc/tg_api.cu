@@ -28,8 +28,11 @@ namespace {
 
 struct LayerW {
   float *P = nullptr, *bu = nullptr, *F = nullptr, *bfc = nullptr, *lng = nullptr, *lnb = nullptr;
+  float* bfcq = nullptr;  // b_fc + [0 | 0 | Phi(0)]: the constant part of the residual q (fused LN epilogue)
   float *W1 = nullptr, *b1 = nullptr, *W2 = nullptr, *b2 = nullptr;
   TcWeights tcP, tcF, tcW1, tcW2;  // tensor-core operand copies (TG_PREC_TF32X3 / BF16)
+  TcWeights tcFa;  // BF16: [F | I_h] -- G2 with the residual h^(l-1) as extra K (identity block)
+  int fa_kb0 = 0;  // first k-block of the identity block
 };
 
 }  // namespace
@@ -51,6 +54,7 @@ struct tg_ctx {
   float *Wa1 = nullptr, *ba1 = nullptr, *Wa2 = nullptr;
   float ba2 = 0.f;
   TcWeights tcWa1;
+  TcWeights tcWa1g;  // BF16 config: W_a1 as a 1-pass tf32 image (gathered fp32 H_L rows)
   // score workspace (S * B edges)
   const float** sc_rs = nullptr;
   const float** sc_rd = nullptr;
@@ -72,6 +76,7 @@ struct tg_ctx {
   // bf16 activations (TG_PREC_BF16): c, [LN(y) | h], z with row strides padded to 8
   unsigned short *c_h = nullptr, *rh_h = nullptr, *z_h = nullptr;
   int ld_ch = 0, ld_rh = 0, ld_z = 0;
+  int dpa = 0;  // BF16 merge-FFN input row [LN(y) (Dp) | 0 | h at dpa = round8(Dp) (16-byte aligned) | 0]
   TcTensorA ta_c, ta_rh, ta_z;  // TMA tensor maps of the bf16 activations (dense GEMM A operands)
   AttnMaps am[2][TG_MAX_LAYERS + 1]{};  // per set and level l: TMA row-gather maps (h rows, E rows, Phi rows)
   int cur_set = 0;
@@ -257,10 +262,23 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   a.nb_hidx = lv.nb_hidx;
   a.phi_row0 = ctx->phi_pre ? ctx->phi_row0[l] : -1;
   const bool bfa = ctx->cfg.precision == TG_PREC_BF16;  // bf16 activations between the GEMMs
+  // TG_LN_FUSE=1: LayerNorm in G2's epilogue (thread-block clusters, DSMEM statistics);
+  // measured slower end to end than G2 + k_layernorm, so off by default
+  static const bool ln_fuse_env = [] {
+    const char* e = getenv("TG_LN_FUSE");
+    return e && e[0] == '1';
+  }();
+  const bool fuse = bfa && ln_fuse_env;
   if (bfa) {
     a.c = nullptr;
     a.c_h = ctx->c_h;
     a.ldc_h = ctx->ld_ch;
+  }
+  if (fuse) {
+    a.hs_row = lv.hs_row;  // h block of the merge-FFN input, also G2's identity-block operand
+    a.rh_h = ctx->rh_h;
+    a.ld_rh = ctx->ld_rh;
+    a.rh_off = ctx->dpa;
   }
   {
     Prof pf(ctx, TG_ST_ATTN, st);
@@ -335,19 +353,36 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
     g2.a_h = ctx->c_h;
     g2.lda_h = ctx->ld_ch;
   }
+  if (fuse) {
+    // residual q (h through the identity block of tcFa, Phi(0) in bfcq) + LayerNorm fused
+    // into the epilogue, which writes the bf16 LN(y) block of the merge-FFN input
+    g2.ln = 1;
+    g2.bias = w.bfcq;
+    g2.ln_g = w.lng;
+    g2.ln_b = w.lnb;
+    g2.ln_dn = ctx->d_n;
+    g2.ln_de = ctx->d_e;
+    g2.ln_dt = ctx->d_t;
+    g2.ln_s1 = ctx->dnp;
+    g2.ln_s2 = ctx->dnp + ctx->dep;
+    g2.C = nullptr;
+    g2.c_h = ctx->rh_h;
+    g2.ldc_h = ctx->ld_rh;
+  }
   {
     Prof pf(ctx, TG_ST_PROJ_V, st);
-    if (tc) launch_gemm_tc(g2, w.tcF, ctx->cfg.precision, st, bfa ? &ctx->ta_c : nullptr);
+    if (fuse) launch_gemm_tc(g2, w.tcFa, ctx->cfg.precision, st, &ctx->ta_c, &ctx->ta_rh, w.fa_kb0, ctx->dpa);
+    else if (tc) launch_gemm_tc(g2, w.tcF, ctx->cfg.precision, st, bfa ? &ctx->ta_c : nullptr);
     else launch_gemm_simt(g2, st);
   }
   TRY(launched(ctx));
-  {
+  if (!fuse) {
     Prof pf(ctx, TG_ST_LNORM, st);
     launch_layernorm(ctx->y, bfa ? nullptr : ctx->r, ctx->Dp, ctx->d_n, ctx->dnp, ctx->d_e, ctx->dep, ctx->d_t,
                      w.lng, w.lnb, m_dev, mmax, lv.hs_row, ctx->table /* Phi(0): row 0 */,
-                     bfa ? ctx->rh_h : nullptr, ctx->ld_rh, st);
+                     bfa ? ctx->rh_h : nullptr, ctx->ld_rh, ctx->dpa, st);
+    TRY(launched(ctx));
   }
-  TRY(launched(ctx));
   // G3: z = ReLU(W1 [r || h^(l-1)] + b1)  (Eq. 7)
   GemmArgs g3{};
   g3.a_base0 = ctx->r;
@@ -547,7 +582,8 @@ tg_status stream_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, cons
       g.ldc = ctx->dnp;
       g.m_dev = ctx->sc_m;
       g.m_max = S * batch;
-      if (ctx->cfg.precision != TG_PREC_FP32) launch_gemm_tc(g, ctx->tcWa1, ctx->cfg.precision, st);
+      if (ctx->cfg.precision == TG_PREC_BF16) launch_gemm_tc(g, ctx->tcWa1g, TG_PREC_TF32, st);
+      else if (ctx->cfg.precision != TG_PREC_FP32) launch_gemm_tc(g, ctx->tcWa1, ctx->cfg.precision, st);
       else launch_gemm_simt(g, st);
       launch_score_head(ctx->sc_z, ctx->dnp, ctx->sc_oidx, S * batch, ctx->Wa2, ctx->ba2, ctx->d_n, scores, st);
     }
@@ -818,6 +854,11 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     TRY(up(&w.bu, buf));
     TRY(up(&w.F, Ff));
     TRY(up(&w.bfc, bfcp));
+    {
+      std::vector<float> bq(bfcp);
+      for (int c = 0; c < d_t; ++c) bq[dnp + ctx->dep + c] += phi0[c];
+      TRY(up(&w.bfcq, bq));
+    }
     TRY(up(&w.lng, lngp));
     TRY(up(&w.lnb, lnbp));
     TRY(up(&w.W1, W1p));
@@ -827,8 +868,35 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     if (cfg->precision != TG_PREC_FP32) {
       TRY(tc_prepare_weights(w.P, HDp, dnp, cfg->precision, &w.tcP, ctx->owned));
       TRY(tc_prepare_weights(w.F, Dp, HDp, cfg->precision, &w.tcF, ctx->owned));
-      TRY(tc_prepare_weights(w.W1, dnp, K3, cfg->precision, &w.tcW1, ctx->owned));
+      if (cfg->precision == TG_PREC_BF16) {  // h block at column dpa (see tg_ctx::dpa)
+        const int dpa = (Dp + 7) & ~7, K3b = dpa + dnp;
+        std::vector<float> W1b((size_t)dnp * K3b, 0.f);
+        for (int j = 0; j < dnp; ++j) {
+          for (int a = 0; a < Dp; ++a) W1b[(size_t)j * K3b + a] = W1p[(size_t)j * K3 + a];
+          for (int b = 0; b < dnp; ++b) W1b[(size_t)j * K3b + dpa + b] = W1p[(size_t)j * K3 + Dp + b];
+        }
+        float* dW1b = nullptr;
+        TRY(up(&dW1b, W1b));
+        TRY(tc_prepare_weights(dW1b, dnp, K3b, cfg->precision, &w.tcW1, ctx->owned));
+      } else {
+        TRY(tc_prepare_weights(w.W1, dnp, K3, cfg->precision, &w.tcW1, ctx->owned));
+      }
       TRY(tc_prepare_weights(w.W2, dnp, dnp, cfg->precision, &w.tcW2, ctx->owned));
+    }
+    if (cfg->precision == TG_PREC_BF16) {
+      // y + q_h = [F | I] [c ; h]: k-blocks [0, kb0) read c (attention output), the last
+      // ceil(dnp / 64) read h^(l-1) (bf16, the h block of the merge-FFN input row)
+      const int kb0 = (HDp + 63) / 64;
+      const int Ka = kb0 * 64 + dnp;
+      std::vector<float> Fa((size_t)Dp * Ka, 0.f);
+      for (int n = 0; n < Dp; ++n) {
+        for (int j = 0; j < HDp; ++j) Fa[(size_t)n * Ka + j] = Ff[(size_t)n * HDp + j];
+        if (n < dnp) Fa[(size_t)n * Ka + kb0 * 64 + n] = 1.f;
+      }
+      float* dFa = nullptr;
+      TRY(up(&dFa, Fa));
+      TRY(tc_prepare_weights(dFa, Dp, Ka, cfg->precision, &w.tcFa, ctx->owned));
+      w.fa_kb0 = kb0;
     }
   }
   // ---- affinity score MLP (R10), padded
@@ -855,6 +923,8 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     ctx->ba2 = ba2[0];
     if (cfg->precision != TG_PREC_FP32)
       TRY(tc_prepare_weights(ctx->Wa1, dnp, 2 * dnp, cfg->precision, &ctx->tcWa1, ctx->owned));
+      if (cfg->precision == TG_PREC_BF16)
+        TRY(tc_prepare_weights(ctx->Wa1, dnp, 2 * dnp, TG_PREC_TF32, &ctx->tcWa1g, ctx->owned));
     const size_t ne = (size_t)S * ((cfg->max_batch_targets + 1) / 2);
     TRY(dalloc(ctx, &ctx->sc_rs, ne));
     TRY(dalloc(ctx, &ctx->sc_rd, ne));
@@ -926,7 +996,8 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
   TRY(dalloc(ctx, &ctx->HL, (size_t)S * cap[L] * dnp));
   if (cfg->precision == TG_PREC_BF16) {
     ctx->ld_ch = (HDp + 7) & ~7;
-    ctx->ld_rh = (Dp + dnp + 7) & ~7;
+    ctx->dpa = (Dp + 7) & ~7;
+    ctx->ld_rh = (ctx->dpa + dnp + 7) & ~7;
     ctx->ld_z = (dnp + 7) & ~7;
     TRY(dalloc(ctx, &ctx->c_h, (size_t)maxC * ctx->ld_ch));
     TRY(dalloc(ctx, &ctx->rh_h, (size_t)maxC * ctx->ld_rh));

@@ -230,6 +230,13 @@ struct AttnArgs {
   int ldc_h;
   const int32_t* nb_hidx;  // row indices of nb_row in maps.h (gather path)
   long long phi_row0;      // >= 0: Phi rows of dt >= W precomputed at rows phi_row0 + p*k + m of maps.t
+  // if rh_h: the target's own h^(l-1) row (hs_row[p], dnp floats) is also written as bf16 to
+  // rh_h[p][rh_off : rh_off+dnp] (rh_off 16-byte aligned, >= Dp) and zeros to the rest of
+  // [Dp, ld_rh): the h block of the merge-FFN input [LN(y) | h] (Eq. 7), read by G2 (residual
+  // q, Eq. 4/6, TMA at column rh_off) and G3
+  const float* const* hs_row;
+  unsigned short* rh_h;
+  int ld_rh, rh_off;
 };
 // TMA row-gather maps of the attention sources: h rows of the level, E rows, Phi table rows.
 struct AttnMaps {
@@ -279,6 +286,15 @@ struct GemmArgs {
   int lda_h;
   unsigned short* c_h;
   int ldc_h;
+  // fused LayerNorm epilogue (G2 in TG_PREC_BF16, tensor-core kernel only):
+  //   x = acc + bias;  r = LN(x; ln_g, ln_b) over the valid columns
+  //   c < ln_dn | ln_s1 <= c < ln_s1 + ln_de | ln_s2 <= c < ln_s2 + ln_dt (Eq. 6, R1),
+  //   written as bf16 to c_h[:, 0:N] only. Row statistics are exchanged between the ntn
+  //   CTAs of a thread-block cluster (DSMEM).
+  int ln;
+  const float* ln_g;
+  const float* ln_b;
+  int ln_dn, ln_de, ln_dt, ln_s1, ln_s2;
 };
 void launch_gemm_simt(const GemmArgs& g, cudaStream_t st);
 
@@ -289,7 +305,7 @@ void launch_gemm_simt(const GemmArgs& g, cudaStream_t st);
 // FFN) are written when non-null.
 void launch_layernorm(const float* y, float* r, int Dp, int dn, int dnp, int de, int dep, int dt,
                       const float* gamma, const float* beta, const int* m_dev, int m_max,
-                      const float* const* hs_rows, const float* phi0, unsigned short* rh, int ldrh,
+                      const float* const* hs_rows, const float* phi0, unsigned short* rh, int ldrh, int rh_off,
                       cudaStream_t st);
 
 // Scores p_e = sigmoid(MLP(h_src, h_dst)) (R10) for every edge of the superbatch:

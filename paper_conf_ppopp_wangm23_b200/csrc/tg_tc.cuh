@@ -32,7 +32,8 @@ tg_status tc_prepare_weights(const float* W, int N, int K, int precision, TcWeig
                              std::vector<void*>& owned);
 // ta (optional): the A operand as a tensor map (must match the element type of
 // the precision: bf16 for TG_PREC_BF16, fp32 for TG_PREC_TF32).
+// ta2 (optional): k-blocks >= a2_kb0 of A come from this second map at columns a2_x0 + 64 (kb - a2_kb0)
 void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaStream_t st,
-                    const TcTensorA* ta = nullptr);
+                    const TcTensorA* ta = nullptr, const TcTensorA* ta2 = nullptr, int a2_kb0 = 0, int a2_x0 = 0);
 
 }  // namespace tg
