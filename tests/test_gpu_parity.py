@@ -305,3 +305,32 @@ def test_gemm_kernels_vs_torch_float64(prec, rtol, atol, M, N, K):
     err = (C.double() - ref).abs()
     bound = atol + rtol * ref.abs()
     assert bool((err <= bound).all()), (prec, float(err.max()))
+
+
+def test_ln_fused_epilogue_parity_subprocess():
+    """TG_LN_FUSE=1 (LayerNorm in G2's epilogue, 3-CTA clusters, DSMEM statistics; not the
+    default) meets the bf16 tolerance too. The toggle is read once per process, hence the
+    subprocess."""
+    import os
+    import subprocess
+    import sys
+    code = r'''
+import numpy as np, torch
+from tests.gpu_helpers import close, setup, make_ctx, make_oracle
+from tests.test_gpu_parity import _stream_gpu
+cfg, s, flat = setup("config1", n_edges=2000)
+mc = cfg.model
+ctx = make_ctx(s, flat, mc, precision=2, superbatch=16)
+sc, _ = _stream_gpu(ctx, s, mc.batch)
+o = make_oracle(s, flat, mc)
+for b in (0, 4, 9):
+    lo, hi = b * mc.batch, (b + 1) * mc.batch
+    _, ref = o.infer_batch(s.src[lo:hi], s.dst[lo:hi], s.ts[lo:hi])
+    ok, err, nbad = close(sc[lo:hi], ref, 2e-2, 2e-2)
+    assert ok, (b, err, nbad)
+print("ok")
+'''
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-c", code], cwd=root, capture_output=True, text=True,
+                       env={**os.environ, "TG_LN_FUSE": "1"}, timeout=600)
+    assert r.returncode == 0 and "ok" in r.stdout, r.stderr[-2000:]
