@@ -401,6 +401,15 @@ k_probe(LevelDev lv, int S, CacheDev c, int use_cache, int has_ring, long long* 
 // The newest copy of a key is always first on its probe chain (an insert
 // takes the first dead or empty slot), so lookups stop at the first match.
 __global__ void k_probe_pre(LevelDev lv, int S, CacheDev c) { pdl_enter();
+  // an index rebuild (launch_index_maint, just before) left its filled-slot count in state[7]
+  if (blockIdx.x == 0 && threadIdx.x == 0 &&
+      c.state[3] * kIndexRebuildDen > (long long)(c.imask + 1) * kIndexRebuildNum)
+    c.state[3] = c.state[7];
+  if (blockIdx.x == 0 && threadIdx.x == 0 && c.occ_report) {  // one 64-bit store: consistent pair
+    const unsigned long long occ = (unsigned long long)c.state[3] & ((1ull << 40) - 1);
+    *(volatile unsigned long long*)c.occ_report = ((unsigned long long)(c.report_sb + 1) << 40) | occ;
+    __threadfence_system();
+  }
   const int tot = S * lv.cap;
   for (int idx = blockIdx.x * blockDim.x + threadIdx.x; idx < tot; idx += gridDim.x * blockDim.x) {
     const int b = idx / lv.cap, i = idx - b * lv.cap;
@@ -782,9 +791,10 @@ __global__ void k_probe_ins(LevelDev lv, CacheDev c, int* err) { pdl_enter();
   const long long head0 = c.state[4];
   const long long live_lo = c.state[0] - c.state[1];
   for (int q = blockIdx.x * blockDim.x + threadIdx.x; q < n; q += gridDim.x * blockDim.x) {
-    if (lv.sup[q]) continue;
     const unsigned long long key = tkey(lv.c_node[q], lv.c_ts[q]);
     const long long pos = head0 + q;
+    c.rkey[pos % c.rcap] = key;  // for index rebuilds
+    if (lv.sup[q]) continue;
     unsigned long long h = mix64(key) & c.imask;
     bool done = false;
     for (unsigned long long pr = 0; pr <= 4 * c.imask && !done; ++pr) {
@@ -807,6 +817,47 @@ __global__ void k_probe_ins(LevelDev lv, CacheDev c, int* err) { pdl_enter();
     }
     if (!done) atomicOr(err, kErrIndexFull);
   }
+}
+
+// Index rebuild, phase 1: clear (every CTA takes the same decision from state[3],
+// which nothing modifies until k_probe_pre).
+__global__ void k_index_clear(CacheDev c) { pdl_enter();
+  if (!(c.state[3] * kIndexRebuildDen > (long long)(c.imask + 1) * kIndexRebuildNum)) return;
+  const unsigned long long n = c.imask + 1;
+  for (unsigned long long i = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; i < n;
+       i += (unsigned long long)gridDim.x * blockDim.x) {
+    c.ikey[i] = kEmptyKey;
+    c.ipos[i] = -1;
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) c.state[7] = 0;
+}
+// phase 2: re-insert the live window [head - size, head); a key present several
+// times keeps its newest position (atomicMax), as the sequential inserts did.
+__global__ void k_index_reinsert(CacheDev c, int* err) { pdl_enter();
+  if (!(c.state[3] * kIndexRebuildDen > (long long)(c.imask + 1) * kIndexRebuildNum)) return;
+  const long long head = c.state[0], lo = head - c.state[1];
+  for (long long p = lo + blockIdx.x * (long long)blockDim.x + threadIdx.x; p < head;
+       p += (long long)gridDim.x * blockDim.x) {
+    const unsigned long long key = c.rkey[p % c.rcap];
+    unsigned long long h = mix64(key) & c.imask;
+    bool done = false;
+    for (unsigned long long pr = 0; pr <= c.imask && !done; ++pr) {
+      const unsigned long long k0 = atomicCAS(c.ikey + h, kEmptyKey, key);
+      if (k0 == kEmptyKey || k0 == key) {
+        atomicMax(c.ipos + h, p);
+        if (k0 == kEmptyKey) atomicAdd((unsigned long long*)(c.state + 7), 1ull);
+        done = true;
+      }
+      h = (h + 1) & c.imask;
+    }
+    if (!done) atomicOr(err, kErrIndexFull);
+  }
+}
+
+int launch_index_maint(const CacheDev& c, cudaStream_t st, int* err) {
+  launch_k(k_index_clear, dim3(148 * 4), dim3(256), 0, st, c);
+  launch_k(k_index_reinsert, dim3(148 * 4), dim3(256), 0, st, c, err);
+  return 2;
 }
 
 int launch_probe(LevelDev lv, int S, const CacheDev* cache, long long* cnt, int layer, int* err,

@@ -70,6 +70,10 @@ struct tg_ctx {
   CacheDev cache[TG_MAX_LAYERS]{};
   long long* cache_state = nullptr;
   int64_t limit0 = 0;
+  long long idx_bound[TG_MAX_LAYERS + 1]{};  // host upper bound on occupied index slots (rebuild trigger)
+  unsigned long long* occ_h = nullptr;       // host-mapped [TG_MAX_LAYERS + 1] occupancy reports
+  long long sb_count = 0;                    // superbatches issued since the last cache reset
+  long long targets_issued = 0;              // layer-L targets issued since the last cache reset
   // compute workspace
   int maxC = 0;
   float *u = nullptr, *c = nullptr, *y = nullptr, *r = nullptr, *z = nullptr, *HL = nullptr;
@@ -452,6 +456,8 @@ tg_status run_front(tg_ctx* ctx, int S, bool edge_mode, const EdgeSrc& es, int n
   const bool cache_on = ctx->cfg.opts & TG_OPT_CACHE;
   const int use_table = (ctx->cfg.opts & TG_OPT_TTABLE) ? 1 : 0;
   long long* cnt = ctx->cnt_sb;
+  ctx->targets_issued += edge_mode ? 2 * std::min<int64_t>((int64_t)S * es.B, es.n_edges - es.e0)
+                                   : (long long)S * n_max_top;
   // ---- top-down (Alg. 1 l.5-12): dedup, lookup/compaction, sampling
   {
     Prof pf(ctx, TG_ST_DEDUP, st);
@@ -479,6 +485,30 @@ tg_status run_front(tg_ctx* ctx, int S, bool edge_mode, const EdgeSrc& es, int n
       TRY(launched(ctx));
       CacheDev cd = ctx->cache[l - 1];
       if (!cache_on) cd.ikey = nullptr;  // ring used as scratch only
+      if (cache_on) {  // index rebuild when it may exceed half occupancy (host upper bound)
+        const long long slots = (long long)cd.imask + 1, per_sb = (long long)S * ctx->cap[l - 1];
+        ctx->idx_bound[l - 1] += per_sb;
+        // tighter bound from the latest device report (occupancy before superbatch sb_obs's
+        // inserts): + at most per_sb for each superbatch since (rebuilds only lower it)
+        // key universe: every cached-level key is a graph edge endpoint (node, t_e), a
+        // layer-L target, or <0, 0>; and a re-inserted (evicted) key reuses its own slot or an
+        // earlier dead one, never an empty slot -> occupied slots <= distinct keys inserted
+        const long long universe = 2 * ctx->g.E + 1 + ctx->targets_issued;
+        if (universe < ctx->idx_bound[l - 1]) ctx->idx_bound[l - 1] = universe;
+        const unsigned long long rep = ctx->occ_h ? *(volatile unsigned long long*)&ctx->occ_h[l - 1] : 0ull;
+        const long long sb_obs = (long long)(rep >> 40) - 1;
+        if (sb_obs >= 0 && sb_obs <= ctx->sb_count) {
+          const long long b = (long long)(rep & ((1ull << 40) - 1)) + (ctx->sb_count - sb_obs + 1) * per_sb;
+          if (b < ctx->idx_bound[l - 1]) ctx->idx_bound[l - 1] = b;
+        }
+        cd.occ_report = ctx->occ_h ? ctx->occ_h + (l - 1) : nullptr;
+        cd.report_sb = ctx->sb_count;
+        if (ctx->idx_bound[l - 1] * kIndexRebuildDen > slots * kIndexRebuildNum) {
+          Prof pf(ctx, TG_ST_LOOKUP, st);
+          TRY(launched(ctx, launch_index_maint(cd, st, ctx->err)));
+          ctx->idx_bound[l - 1] = slots * kIndexRebuildNum / kIndexRebuildDen;  // <= threshold afterwards
+        }
+      }
       {
         Prof pf(ctx, TG_ST_LOOKUP, st);
         nl = launch_probe(ctx->lv[l - 1], S, &cd, cnt, l - 1, ctx->err, st);
@@ -486,6 +516,7 @@ tg_status run_front(tg_ctx* ctx, int S, bool edge_mode, const EdgeSrc& es, int n
       TRY(launched(ctx, nl));
     }
   }
+  ++ctx->sb_count;
   // ---- row addresses for every layer
   ResolveArgs ra{};
   for (int l = 0; l <= L; ++l) ra.lv[l] = ctx->lv[l];
@@ -983,6 +1014,7 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     TRY(dalloc(ctx, &cd.ikey, icap));
     TRY(dalloc(ctx, &cd.ipos, icap));
     TRY(dalloc(ctx, &cd.ring, (size_t)rcap * dnp));
+    TRY(dalloc(ctx, &cd.rkey, (size_t)rcap));
     cd.imask = icap - 1;
     cd.rcap = rcap;
     cd.state = ctx->cache_state + 8 * l;
@@ -1053,6 +1085,10 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     CK(cudaEventCreateWithFlags(&ctx->ev_in, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&ctx->ev_fend, cudaEventDisableTiming));
   }
+  if (!ctx->occ_h) {
+    CK(cudaHostAlloc(&ctx->occ_h, (TG_MAX_LAYERS + 1) * sizeof(unsigned long long), cudaHostAllocMapped));
+    memset(ctx->occ_h, 0, (TG_MAX_LAYERS + 1) * sizeof(unsigned long long));
+  }
   CK(cudaDeviceSynchronize());
   ctx->loaded = true;
   return tg_cache_reset(ctx, -1);
@@ -1071,7 +1107,11 @@ tg_status tg_cache_reset(tg_ctx* ctx, int64_t new_limit) {
     CK(cudaMemset(cd.ikey, 0xFF, (cd.imask + 1) * sizeof(unsigned long long)));
     long long st[8] = {0, 0, ctx->cfg.cache_limit, 0, 0, 0, 0, 0};
     CK(cudaMemcpy(cd.state, st, sizeof(st), cudaMemcpyHostToDevice));
+    ctx->idx_bound[l] = 0;
+    if (ctx->occ_h) ctx->occ_h[l] = 0;
   }
+  ctx->sb_count = 0;
+  ctx->targets_issued = 0;
   CK(cudaMemset(ctx->cnt_total, 0, TG_NCOUNTERS * sizeof(long long)));
   CK(cudaMemset(ctx->cnt_sb, 0, (size_t)kMaxS * TG_NCOUNTERS * sizeof(long long)));
   CK(cudaMemset(ctx->err, 0, sizeof(int)));
@@ -1354,6 +1394,7 @@ void tg_free(tg_ctx* ctx) {
   for (cudaEvent_t e : {ctx->ev_front[0], ctx->ev_front[1], ctx->ev_back[0], ctx->ev_back[1], ctx->ev_in, ctx->ev_fend})
     if (e) cudaEventDestroy(e);
   if (ctx->fst) cudaStreamDestroy(ctx->fst);
+  if (ctx->occ_h) cudaFreeHost(ctx->occ_h);
   if (ctx->stage) cudaFree(ctx->stage);
   delete ctx;
 }

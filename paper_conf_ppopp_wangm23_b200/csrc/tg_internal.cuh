@@ -124,8 +124,20 @@ struct CacheDev {
   unsigned long long imask;
   float* ring;               // [rcap x ldn]
   long long rcap;
-  long long* state;          // device [8]: head, size, limit, occupied index slots, head at SB start
+  long long* state;          // device [8]: head, size, limit, occupied index slots, head at SB start,
+                             // eviction-free flag, -, slots filled by an index rebuild
+  unsigned long long* rkey;  // [rcap] key stored at each ring slot (index rebuild)
+  // host-mapped report word: ((superbatch + 1) << 40) | occupied slots, written by
+  // k_probe_pre, read by the host without synchronising (rebuild trigger bound)
+  unsigned long long* occ_report;
+  long long report_sb;       // superbatch number of this launch (set per launch)
 };
+// Index maintenance: the index never deletes, so FIFO churn (small limits) fills it with
+// dead keys and absent-key probes lengthen; when more than half of the slots are occupied
+// the index is rebuilt from the live ring window (clear, then re-insert keys of positions
+// [head - size, head), newest position per key). Returns launches issued.
+int launch_index_maint(const CacheDev& c, cudaStream_t st, int* err);
+constexpr int kIndexRebuildNum = 1, kIndexRebuildDen = 2;  // rebuild above 1/2 occupancy
 
 // One recursion level l >= 1 of a superbatch.
 struct LevelDev {

@@ -128,3 +128,18 @@ def test_fullsize_large_batch2000():
     nb = log.shape[0]
     _check_scores(s, flat, mc, scores, [0, nb // 2, nb - 1], 2)
     ctx.close()
+
+
+def test_fullsize_next4_reddit_L3_k8():
+    """NEXT-4: the deeper / narrower model, L = 3, k = 8, two cached
+    layers (R9) with one index each, on the whole Reddit-shaped stream in bf16 (S is lowered
+    to fit the cache passes): every batch's counters bit-exact against the Alg. 1/3
+    simulator, sampled scores vs the plain oracle."""
+    cfg, s, flat = setup("reddit", n_layers=3, n_neighbors=8)
+    mc = cfg.model
+    ctx = make_ctx(s, flat, mc, precision=2, superbatch=BENCH_S)
+    scores, log = _run(ctx, s, mc.batch)
+    _check_counters(s, flat, mc, log, mc.cache_limit)
+    nb = log.shape[0]
+    _check_scores(s, flat, mc, scores, [0, nb // 2, nb - 1], 2)
+    ctx.close()

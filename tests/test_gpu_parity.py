@@ -334,3 +334,23 @@ print("ok")
     r = subprocess.run([sys.executable, "-c", code], cwd=root, capture_output=True, text=True,
                        env={**os.environ, "TG_LN_FUSE": "1"}, timeout=600)
     assert r.returncode == 0 and "ok" in r.stdout, r.stderr[-2000:]
+
+
+@pytest.mark.parametrize("S", [1, 16])
+def test_index_rebuild_under_fifo_churn(S):
+    """A tiny limit (10 items) makes nearly every layer-1 lookup a miss: ~10^5 inserts into an
+    index of 2^15 (S = 1) slots, so the index crosses half occupancy and is rebuilt from the
+    live ring window several times during the pass. Counters (hits, misses, evictions) stay
+    bit-exact against the Alg. 1/3 simulator and scores equal those of a roomy cache."""
+    from paper_conf_ppopp_wangm23_b200 import counters_dict
+    cfg, s, flat = setup("config1")
+    mc = cfg.model
+    ctx = make_ctx(s, flat, mc, cache_limit=10, superbatch=S)
+    sc, log = _stream_gpu(ctx, s, mc.batch)
+    want = _sim_counters(s, flat, mc, 10)
+    for b, w in enumerate(want):
+        got = counters_dict(log[b], mc.n_layers)
+        assert got == w, (b, {k: (got[k], w[k]) for k in w if got[k] != w[k]})
+    ref = make_ctx(s, flat, mc, superbatch=S)
+    sc_ref, _ = _stream_gpu(ref, s, mc.batch)
+    assert np.array_equal(sc, sc_ref)

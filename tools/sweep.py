@@ -62,6 +62,8 @@ def run(s, flat, mc, opts, limit, passes, prec):
         "l1_hit_rate_10batch_window_max": float(np.max(win)) if c["l1_lookups"] else None,
         "computed": {f"l{l}": c[f"l{l}_misses"] for l in range(1, mc.n_layers + 1)},
         "evicted": c["l1_evicted"],
+        "hit_rate_global_per_layer": {f"l{l}": (c[f"l{l}_hits"] / c[f"l{l}_lookups"] if c[f"l{l}_lookups"] else None)
+                                      for l in range(1, mc.n_layers)},
         "time_table_hit_rate": c["t_table"] / max(1, c["t_table"] + c["t_direct"]),
         "cache_items_end": min(int(limit), c["l1_misses"]) if opts & 2 else 0,
         "cache_payload_mib_end": min(int(limit), c["l1_misses"]) * 4 * s.d_n / 2 ** 20 if opts & 2 else 0,
@@ -76,14 +78,19 @@ def main():
     ap.add_argument("--passes", type=int, default=3)
     ap.add_argument("--precision", type=int, default=2)  # TG_PREC_BF16
     ap.add_argument("--out", default=None)
+    ap.add_argument("--model", default=None, help="L,k override, e.g. 3,8 (NEXT-4: L = 3, k = 8)")
     args = ap.parse_args()
+    over = {}
+    if args.model:
+        L, k = (int(v) for v in args.model.split(","))
+        over = dict(n_layers=L, n_neighbors=k)
     from synth import get_config, make_stream, make_params
     D, C, T = 1, 2, 4  # TG_OPT_DEDUP, TG_OPT_CACHE, TG_OPT_TTABLE
     ablation = [("none", 0), ("cache", C), ("cache+dedup", C | D), ("cache+dedup+ttable", C | D | T)]
     limits = [10_000, 100_000, 1_000_000, 2_000_000, 3_000_000]
     res = []
     for name in args.configs:
-        cfg = get_config(name)
+        cfg = get_config(name, **over)
         mc = cfg.model
         s = make_stream(name)
         flat = make_params(mc.n_layers, mc.n_heads, s.d_n, s.d_e)
@@ -92,13 +99,13 @@ def main():
             row, sc = run(s, flat, mc, opts, mc.cache_limit, args.passes, args.precision)
             if ref is None:
                 ref = sc
-            row.update(config=name, sweep="ablation", opts=label, cache_limit=mc.cache_limit,
+            row.update(config=name, model=f"L{mc.n_layers}k{mc.n_neighbors}", sweep="ablation", opts=label, cache_limit=mc.cache_limit,
                        scores_equal_to_none=bool(np.array_equal(sc, ref)))
             print(json.dumps(row), flush=True)
             res.append(row)
         for lim in limits:
             row, sc = run(s, flat, mc, C | D | T, lim, args.passes, args.precision)
-            row.update(config=name, sweep="cache_limit", opts="cache+dedup+ttable", cache_limit=lim,
+            row.update(config=name, model=f"L{mc.n_layers}k{mc.n_neighbors}", sweep="cache_limit", opts="cache+dedup+ttable", cache_limit=lim,
                        scores_equal_to_none=bool(np.array_equal(sc, ref)))
             print(json.dumps(row), flush=True)
             res.append(row)
