@@ -311,7 +311,6 @@ template <int PREC>
 __global__ void __launch_bounds__(TC_THREADS, 1)
     k_gemm_tc(GemmArgs g, TcWeights w, int stages, const __grid_constant__ CUtensorMap tmA, int a_tma,
               const __grid_constant__ CUtensorMap tmA2, int a2_kb0, int a2_x0) {
-  pdl_enter();
   constexpr int EPC = PREC == TG_PREC_BF16 ? 64 : 32;
   constexpr int PLANES = PREC == TG_PREC_TF32X3 ? 2 : 1;
   constexpr int NV = EPC / 4;  // float4 loads per row per k-block
@@ -333,19 +332,16 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
 #ifdef TG_TC_TRACE
   const long long t_entry = clock64();
 #endif
-  const int M = *g.m_dev;
-  const int tiles_m = (M + TC_BM - 1) / TC_BM;
-  const int ntiles = tiles_m * w.ntn;
-  if ((int)blockIdx.x >= ntiles) return;
 #ifdef TG_TC_TRACE
   // only full-grid launches are traced (a later partial launch would leave stale stamps)
-  const bool tct_on = tg_tct_nk[0] == g.N && tg_tct_nk[1] == g.K && ntiles >= (int)gridDim.x;
+  const int Mtr = *g.m_dev;  // debug build only: read before the PDL wait
+  const bool tct_on = tg_tct_nk[0] == g.N && tg_tct_nk[1] == g.K && ((Mtr + TC_BM - 1) / TC_BM) * w.ntn >= (int)gridDim.x;
   if (tid == 0) {
     long long gt;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt));
     TCT(0, t_entry);
     TCT(1, gt);
-    TCT(63, M);
+    TCT(63, Mtr);
   }
 #endif
   const int nkb = w.nkb;
@@ -374,6 +370,12 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     asm volatile("barrier.cluster.wait.acquire.aligned;\n" ::: "memory");
   }
   const uint32_t tmem = *tmem_slot;
+  // Everything above touches only shared memory / TMEM / parameters: with programmatic
+  // dependent launch it overlaps the previous kernel's tail. The row count is its output.
+  pdl_enter();
+  const int M = *g.m_dev;
+  const int tiles_m = (M + TC_BM - 1) / TC_BM;
+  const int ntiles = tiles_m * w.ntn;  // CTAs past ntiles run no tile and fall through to the end
   if (tid == 0) TCT(2, clock64());
 
   if (warp < 4 && a_tma) {
