@@ -39,7 +39,8 @@ def _stale():
 
 def _compile(src, log):
     obj = os.path.join(BUILD, os.path.basename(src)[:-3] + ".o")
-    cmd = [NVCC, *ARCH, *FLAGS, "-c", src, "-o", obj]
+    extra = os.environ.get("TG_EXTRA_FLAGS_" + os.path.basename(src)[:-3].upper(), "").split()  # experiments
+    cmd = [NVCC, *ARCH, *FLAGS, *extra, "-c", src, "-o", obj]
     r = subprocess.run(cmd, capture_output=True, text=True)
     with open(log, "a") as f:
         f.write(" ".join(cmd) + "\n" + r.stdout + r.stderr + "\n")

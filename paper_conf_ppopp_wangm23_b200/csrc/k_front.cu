@@ -418,10 +418,10 @@ __global__ void k_probe_pre(LevelDev lv, int S, CacheDev c) { pdl_enter();
     unsigned long long h = mix64(key) & c.imask;
     long long p = -1;
     for (unsigned long long pr = 0; pr <= c.imask; ++pr) {
-      const unsigned long long k0 = c.ikey[h];
+      const unsigned long long k0 = __ldcg(c.ikey + h);
       if (k0 == kEmptyKey) break;
       if (k0 == key) {
-        p = c.ipos[h];
+        p = __ldcg(c.ipos + h);
         break;
       }
       h = (h + 1) & c.imask;
@@ -450,13 +450,13 @@ k_probe_seq(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err)
   if (c.state[5] == 1) return;  // the eviction-free parallel pass handled this superbatch
   for (int s = tid; s < kSeqSlots; s += blockDim.x) skey[s] = kEmptyKey;
   if (rank == 0 && tid == 0) {
-    s_head = c.state[0];
-    s_size = c.state[1];
+    s_head = __ldcg(c.state + 0);
+    s_size = __ldcg(c.state + 1);
     s_base = 0;
     c.state[4] = c.state[0];  // head0 for the insert pass
   }
-  const long long limit = c.state[2];
-  const long long head0 = c.state[0];
+  const long long limit = __ldcg(c.state + 2);
+  const long long head0 = __ldcg(c.state + 0);
   const unsigned long long tmask = (unsigned long long)CL * kSeqSlots - 1ull;
   cluster.sync();
   for (int b = 0; b < S; ++b) {
@@ -491,7 +491,7 @@ k_probe_seq(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err)
           }
           h = (h + 1) & tmask;
         }
-        if (sbslot[j] == 0xFFFFFFFFu) p = lv.p0[seg + i];
+        if (sbslot[j] == 0xFFFFFFFFu) p = __ldcg(lv.p0 + seg + i);
         if (p >= 0 && p >= live_lo) {
           lv.slot[seg + i] = p % c.rcap;  // hit (Alg. 1 l.8)
         } else {
@@ -591,7 +591,7 @@ k_probe_par(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err)
   const unsigned CL = cluster.num_blocks();
   const unsigned rank = cluster.block_rank();
   const int tid = threadIdx.x;
-  const long long head0 = c.state[0], size0 = c.state[1], limit = c.state[2];
+  const long long head0 = __ldcg(c.state + 0), size0 = __ldcg(c.state + 1), limit = __ldcg(c.state + 2);
   if (tid == 0) {
     int a = 0;
     for (int b = 0; b < S; ++b) {
@@ -657,7 +657,7 @@ k_probe_par(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err)
       if (*(cluster.map_shared_rank(sval, h / kSeqSlots) + (h % kSeqSlots)) == (unsigned)i) {
         firstmask |= 1u << j;
         const size_t idx = (size_t)jb[j] * lv.cap + (i - s_pre[jb[j]]);
-        const long long p = lv.p0[idx];
+        const long long p = __ldcg(lv.p0 + idx);
         if (!(p >= 0 && p >= live_lo)) {
           missmask |= 1u << j;
           ++m_local;
@@ -689,7 +689,7 @@ k_probe_par(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err)
         sl = (head0 + q) % c.rcap;
         ++q;
       } else {
-        sl = lv.p0[idx] % c.rcap;
+        sl = __ldcg(lv.p0 + idx) % c.rcap;
       }
       lv.slot[idx] = sl;
       const unsigned h = hs[j];
@@ -788,13 +788,19 @@ __global__ void k_ring_advance(LevelDev lv, CacheDev c) { pdl_enter(); c.state[0
 
 __global__ void k_probe_ins(LevelDev lv, CacheDev c, int* err) { pdl_enter();
   const int n = *lv.n_c_total;
-  const long long head0 = c.state[4];
-  const long long live_lo = c.state[0] - c.state[1];
+  const long long head0 = __ldcg(c.state + 4);
+  const long long live_lo = __ldcg(c.state + 0) - __ldcg(c.state + 1);
   for (int q = blockIdx.x * blockDim.x + threadIdx.x; q < n; q += gridDim.x * blockDim.x) {
     const unsigned long long key = tkey(lv.c_node[q], lv.c_ts[q]);
     const long long pos = head0 + q;
     c.rkey[pos % c.rcap] = key;  // for index rebuilds
-    if (lv.sup[q]) continue;
+    // Skip superseded misses and misses already evicted by the end of this superbatch
+    // (pos < live_lo: more misses than the limit, R11). Inserting a dead-on-arrival key
+    // would let its slot be locked and rewritten twice in this launch (dead -> dead ->
+    // live), an ABA under which a thread still holding the slot's first key could CAS
+    // over the live key written last. Every write below makes its slot live, and live
+    // slots are never reusable within the launch.
+    if (lv.sup[q] || pos < live_lo) continue;
     unsigned long long h = mix64(key) & c.imask;
     bool done = false;
     for (unsigned long long pr = 0; pr <= 4 * c.imask && !done; ++pr) {
@@ -852,6 +858,30 @@ __global__ void k_index_reinsert(CacheDev c, int* err) { pdl_enter();
     }
     if (!done) atomicOr(err, kErrIndexFull);
   }
+}
+
+// debug (TG_DBG_INDEX_CHECK=1): every key of the live window must be found at its newest
+// position; mismatches are counted into err[1]
+__global__ void k_index_check(CacheDev c, int* err) {
+  const long long head = c.state[0], lo = head - c.state[1];
+  for (long long p = lo + blockIdx.x * (long long)blockDim.x + threadIdx.x; p < head;
+       p += (long long)gridDim.x * blockDim.x) {
+    const unsigned long long key = c.rkey[p % c.rcap];
+    // newest position of this key within the window: scan forward is too slow; check that
+    // the index position is >= p (the newest copy is never older than any live copy)
+    unsigned long long h = mix64(key) & c.imask;
+    long long found = -2;
+    for (unsigned long long pr = 0; pr <= c.imask; ++pr) {
+      const unsigned long long k0 = __ldcg(c.ikey + h);
+      if (k0 == kEmptyKey) { found = -1; break; }
+      if (k0 == key) { found = __ldcg(c.ipos + h); break; }
+      h = (h + 1) & c.imask;
+    }
+    if (found < p) atomicAdd(err + 1, 1);
+  }
+}
+void launch_index_check(const CacheDev& c, int* err, cudaStream_t st) {
+  k_index_check<<<148, 256, 0, st>>>(c, err);
 }
 
 int launch_index_maint(const CacheDev& c, cudaStream_t st, int* err) {

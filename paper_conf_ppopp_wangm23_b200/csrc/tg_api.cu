@@ -512,6 +512,8 @@ tg_status run_front(tg_ctx* ctx, int S, bool edge_mode, const EdgeSrc& es, int n
       {
         Prof pf(ctx, TG_ST_LOOKUP, st);
         nl = launch_probe(ctx->lv[l - 1], S, &cd, cnt, l - 1, ctx->err, st);
+        static const bool dbg_check = getenv("TG_DBG_INDEX_CHECK") != nullptr;
+        if (dbg_check && cache_on) launch_index_check(cd, ctx->err, st);
       }
       TRY(launched(ctx, nl));
     }
@@ -592,7 +594,9 @@ tg_status stream_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, cons
     EdgeSrc es{src, dst, ts, n_edges, b0 * batch, batch};
     select_set(ctx, set);
     if (sb >= 2) CK(cudaStreamWaitEvent(ctx->fst, ctx->ev_back[set], 0));
-    TRY(run_front(ctx, S, true, es, 2 * batch, ctx->fst));
+    static const bool one_stream = getenv("TG_ONE_STREAM") != nullptr;  // debug: no overlap
+    TRY(run_front(ctx, S, true, es, 2 * batch, one_stream ? st : ctx->fst));
+    if (one_stream) CK(cudaEventRecord(ctx->ev_front[set], st));
     CK(cudaEventRecord(ctx->ev_front[set], ctx->fst));
     CK(cudaStreamWaitEvent(st, ctx->ev_front[set], 0));
     TRY(run_back(ctx, st));
@@ -621,6 +625,7 @@ tg_status stream_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, cons
     TRY(launched(ctx, 3));
     TRY(finish(ctx, S, log, b0, st));
     CK(cudaEventRecord(ctx->ev_back[set], st));
+
   }
   CK(cudaEventRecord(ctx->ev_fend, ctx->fst));  // join the front stream into st
   CK(cudaStreamWaitEvent(st, ctx->ev_fend, 0));
@@ -741,8 +746,8 @@ tg_status tg_graph_load(int device, const tg_graph_desc* gd, tg_ctx** out) {
   g.d_e = gd->d_e;
   g.ldn = ldn;
   g.lde = lde;
-  TRYF(dalloc(ctx, &ctx->err, 1));
-  cudaMemset(ctx->err, 0, sizeof(int));
+  TRYF(dalloc(ctx, &ctx->err, 2));  // [0] sticky error bits, [1] debug index-check mismatches
+  cudaMemset(ctx->err, 0, 2 * sizeof(int));
   *out = ctx;
   return TG_OK;
 #undef TRYF
@@ -1114,7 +1119,7 @@ tg_status tg_cache_reset(tg_ctx* ctx, int64_t new_limit) {
   ctx->targets_issued = 0;
   CK(cudaMemset(ctx->cnt_total, 0, TG_NCOUNTERS * sizeof(long long)));
   CK(cudaMemset(ctx->cnt_sb, 0, (size_t)kMaxS * TG_NCOUNTERS * sizeof(long long)));
-  CK(cudaMemset(ctx->err, 0, sizeof(int)));
+  CK(cudaMemset(ctx->err, 0, 2 * sizeof(int)));
   CK(cudaDeviceSynchronize());
   ctx->launches = 0;
   return TG_OK;
@@ -1389,6 +1394,11 @@ void tg_free(tg_ctx* ctx) {
   if (!ctx) return;
   cudaSetDevice(ctx->device);
   cudaDeviceSynchronize();
+  if (getenv("TG_DBG_INDEX_CHECK") && ctx->err) {
+    int e[2] = {0, 0};
+    cudaMemcpy(e, ctx->err, sizeof(e), cudaMemcpyDeviceToHost);
+    fprintf(stderr, "libtg: index check mismatches %d (err bits %d)\n", e[1], e[0]);
+  }
   for (void* p : ctx->owned) cudaFree(p);
   for (cudaEvent_t e : ctx->ev_pool) cudaEventDestroy(e);
   for (cudaEvent_t e : {ctx->ev_front[0], ctx->ev_front[1], ctx->ev_back[0], ctx->ev_back[1], ctx->ev_in, ctx->ev_fend})

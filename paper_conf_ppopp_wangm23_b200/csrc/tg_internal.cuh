@@ -137,6 +137,7 @@ struct CacheDev {
 // the index is rebuilt from the live ring window (clear, then re-insert keys of positions
 // [head - size, head), newest position per key). Returns launches issued.
 int launch_index_maint(const CacheDev& c, cudaStream_t st, int* err);
+void launch_index_check(const CacheDev& c, int* err, cudaStream_t st);
 constexpr int kIndexRebuildNum = 1, kIndexRebuildDen = 2;  // rebuild above 1/2 occupancy
 
 // One recursion level l >= 1 of a superbatch.
