@@ -54,10 +54,11 @@ __device__ __forceinline__ int batch_edges(const EdgeSrc& es, int b, int64_t& lo
 // with an ordered scan across the cluster (first-occurrence order, R8);
 // phase D reads the inverse index.
 __global__ void __launch_bounds__(kDedupThreads, 1)
-k_dedup(LevelDev lv, int edge_mode, EdgeSrc es, long long* cnt, int layer, int* err) { pdl_enter();
+k_dedup(LevelDev lv, int edge_mode, EdgeSrc es, long long* cnt, int layer, int* err, int nslots) {
+  // nslots: hash slots per CTA (power of two, sized to the batch: load <= 0.4)
   extern __shared__ __align__(16) unsigned char smem[];
   unsigned long long* skey = reinterpret_cast<unsigned long long*>(smem);
-  unsigned int* spos = reinterpret_cast<unsigned int*>(skey + kDedupSlots);
+  unsigned int* spos = reinterpret_cast<unsigned int*>(skey + nslots);
   __shared__ int s_warp[32];
   __shared__ int s_total;
   cg::cluster_group cluster = cg::this_cluster();
@@ -84,16 +85,17 @@ k_dedup(LevelDev lv, int edge_mode, EdgeSrc es, long long* cnt, int layer, int* 
       t = lv.in_ts[seg + i];
     }
   };
-  for (int s = tid; s < kDedupSlots; s += blockDim.x) {
+  for (int s = tid; s < nslots; s += blockDim.x) {
     skey[s] = kEmptyKey;
     spos[s] = 0xFFFFFFFFu;
   }
+  pdl_enter();  // shared-memory setup above overlaps the previous kernel's tail
   cluster.sync();
   const int chunk = (n + (int)CL - 1) / (int)CL;
   const int cbeg = min(n, (int)rank * chunk), cend = min(n, cbeg + chunk);
   const int ipt = (chunk + (int)blockDim.x - 1) / (int)blockDim.x;
   const int tbeg = cbeg + tid * ipt;
-  const unsigned long long tmask = (unsigned long long)CL * kDedupSlots - 1ull;
+  const unsigned long long tmask = (unsigned long long)CL * nslots - 1ull;
   unsigned slot[kDedupIPT];
   // ---- phase B
 #pragma unroll
@@ -107,7 +109,7 @@ k_dedup(LevelDev lv, int edge_mode, EdgeSrc es, long long* cnt, int layer, int* 
       const unsigned long long key = tkey(node, t);
       unsigned long long h = mix64(key) & tmask;
       for (unsigned long long probe = 0; probe <= tmask; ++probe) {
-        const unsigned owner = (unsigned)(h / kDedupSlots), loc = (unsigned)(h % kDedupSlots);
+        const unsigned owner = (unsigned)(h / nslots), loc = (unsigned)(h % nslots);
         unsigned long long* kp = cluster.map_shared_rank(skey, owner) + loc;
         const unsigned long long old = atomicCAS(kp, kEmptyKey, key);
         if (old == kEmptyKey || old == key) {
@@ -129,7 +131,7 @@ k_dedup(LevelDev lv, int edge_mode, EdgeSrc es, long long* cnt, int layer, int* 
     const int i = tbeg + j;
     if (j < ipt && i < cend && slot[j] != 0xFFFFFFFFu) {
       const unsigned h = slot[j];
-      const unsigned p = *(cluster.map_shared_rank(spos, h / kDedupSlots) + (h % kDedupSlots));
+      const unsigned p = *(cluster.map_shared_rank(spos, h / nslots) + (h % nslots));
       if (p == (unsigned)i) {
         firstmask |= 1u << j;
         ++c;
@@ -154,7 +156,7 @@ k_dedup(LevelDev lv, int edge_mode, EdgeSrc es, long long* cnt, int layer, int* 
       lv.u_node[seg + uid] = node;
       lv.u_ts[seg + uid] = t;
       const unsigned h = slot[j];
-      *(cluster.map_shared_rank(spos, h / kDedupSlots) + (h % kDedupSlots)) = (unsigned)uid;
+      *(cluster.map_shared_rank(spos, h / nslots) + (h % nslots)) = (unsigned)uid;
       ++uid;
     }
   }
@@ -172,7 +174,7 @@ k_dedup(LevelDev lv, int edge_mode, EdgeSrc es, long long* cnt, int layer, int* 
     const int i = tbeg + j;
     if (j < ipt && i < cend && slot[j] != 0xFFFFFFFFu) {
       const unsigned h = slot[j];
-      lv.inv[seg + i] = (int32_t) * (cluster.map_shared_rank(spos, h / kDedupSlots) + (h % kDedupSlots));
+      lv.inv[seg + i] = (int32_t) * (cluster.map_shared_rank(spos, h / nslots) + (h % nslots));
     }
   }
   cluster.sync();  // peers may still read this CTA's shared memory
@@ -231,15 +233,18 @@ void launch_dedup(LevelDev lv, int S, int n_max, bool edge_mode, EdgeSrc es, lon
     return;
   }
   const int cl = dedup_cluster_size(n_max);
-  const size_t smem = (size_t)kDedupSlots * (sizeof(unsigned long long) + sizeof(unsigned));
+  int nslots = 1024;  // per CTA: cl * nslots >= 2.5 n_max (load <= 0.4)
+  while (nslots < kDedupSlots && (long long)cl * nslots * 2 < (long long)n_max * 5) nslots <<= 1;
+  const size_t smem = (size_t)nslots * (sizeof(unsigned long long) + sizeof(unsigned));
   static bool attr_done = false;
   if (!attr_done) {
-    cudaFuncSetAttribute(k_dedup, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(k_dedup, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)((size_t)kDedupSlots * (sizeof(unsigned long long) + sizeof(unsigned))));
     cudaFuncSetAttribute(k_dedup, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
     attr_done = true;
   }
   launch_k_cluster(k_dedup, dim3(cl * S), dim3(kDedupThreads), smem, st, cl, lv, edge_mode ? 1 : 0, es, cnt, layer,
-                   err);
+                   err, nslots);
 }
 
 // ------------------------------------------------------- CacheLookup / Store
