@@ -363,7 +363,7 @@ def main():
                            "edges_per_rank": E_rank, "batch": B, "n_layers": mc.n_layers, "heads": mc.n_heads,
                            "k": mc.n_neighbors, "d_n": s.d_n, "d_e": s.d_e, "cache_limit": mc.cache_limit,
                            "time_window": mc.time_window, "opts": "dedup+cache+ttable",
-                           "superbatch": args.superbatch or 16,
+                           "superbatch": ctx.superbatch(),
                            "parallelism": (f"independent streams x{world}" if args.scaling == "weak"
                                            else f"batch-range shards x{world}"),
                            "l2": "flushed (256 MB write) before every timed step; inputs > L2",

@@ -96,13 +96,14 @@ typedef struct {
   int32_t time_window;        /* W of the precomputed Phi table (10,000)     */
   uint32_t opts;              /* TG_OPT_* bits                                        */
   int32_t precision;          /* TG_PREC_*                                            */
-  int32_t superbatch;         /* S: batches per launch sequence in tg_score_stream (0 = 16,
+  int32_t superbatch;         /* S: batches per launch sequence in tg_score_stream (0 = 32,
                                * 1 = one batch at a time). Semantics per batch are unchanged:
                                * dedup scope, cache lookups and FIFO inserts stay per batch
                                * and in batch order, so outputs and counters do not depend on S.
                                * S is lowered so that S x (per-batch capacity of each cached
-                               * level) fits the cache passes' DSMEM hash (157,286 keys):
-                               * batch 200, k = 20 keeps S <= 18; batch 2,000 runs S = 1. */
+                               * level) fits the cache passes' DSMEM hash at a worst-case load
+                               * <= 0.9 (235,929 keys): batch 200, k = 20 runs S <= 28; batch
+                               * 2,000 runs S = 1. tg_superbatch() returns the S in use. */
 } tg_model_cfg;
 
 /* params: host float32 [n_params] in this order (row-major, Linear = [out x in]),
@@ -199,6 +200,9 @@ tg_status tg_gemm(tg_ctx* ctx, int32_t precision, int32_t M, int32_t N, int32_t 
 /* Library/launch statistics for the bench: number of kernels launched by the
  * hot-path calls since the last tg_cache_reset (host-side count). */
 int64_t tg_kernel_launches(tg_ctx* ctx);
+/* Batches per launch sequence actually used by tg_score_stream (tg_model_cfg.superbatch after
+ * the default and the cache-pass capacity clamp); 0 before tg_model_load or for a null ctx. */
+int32_t tg_superbatch(tg_ctx* ctx);
 
 /* Per-stage device timing (the operation breakdown of Table 3):
  * when enabled, every hot-path launch is bracketed by CUDA events on its

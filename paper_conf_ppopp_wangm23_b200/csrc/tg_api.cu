@@ -661,6 +661,7 @@ const char* tg_strerror(tg_status s) {
 const char* tg_version(void) { return "libtg 0.2 sm_100a (fp32 SIMT, tf32x3/bf16 tcgen05; superbatch schedule)"; }
 
 int64_t tg_kernel_launches(tg_ctx* ctx) { return ctx ? ctx->launches : 0; }
+int32_t tg_superbatch(tg_ctx* ctx) { return (ctx && ctx->loaded) ? ctx->S : 0; }
 
 tg_status tg_graph_load(int device, const tg_graph_desc* gd, tg_ctx** out) {
   if (!gd || !out) return TG_EINVAL;
@@ -768,7 +769,7 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
   const int64_t per_layer = 4LL * D * D + 3LL * D + (int64_t)d_n * (D + d_n) + d_n + (int64_t)d_n * d_n + d_n;
   const int64_t expect = L * per_layer + 2LL * d_t + 2LL * d_n * d_n + d_n + d_n + 1;
   if (n_params != expect) return TG_EINVAL;
-  int S = cfg->superbatch ? cfg->superbatch : 16;
+  int S = cfg->superbatch ? cfg->superbatch : 32;
   // per-batch capacities: I_L = targets; I_{l-1} = C_l (k+1) <= I_l (k+1)
   int cap[TG_MAX_LAYERS + 1];
   int64_t cc = cfg->max_batch_targets;
@@ -782,10 +783,11 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     if (cap[l] > 16 * 10000) return TG_EINVAL;                   // dedup cluster bound
     if (cap[l] > kSeqCLMax * 1024 * kProbeIPT) return TG_EINVAL; // ordered cache pass bound
   }
-  // every key of a superbatch's cached level must fit the cache passes' DSMEM hash
-  // (load <= 0.6): S shrinks for large batches (batch 2,000 at k = 20 -> S = 1)
+  // every key of a superbatch's cached level must fit the cache passes' DSMEM hash:
+  // worst-case load <= 0.9 (cap assumes every target and neighbour distinct; real
+  // superbatches load it about half as much). S shrinks for large batches (2,000 -> 1).
   for (int l = 1; l < L; ++l) {
-    const int64_t fit = (int64_t)kSeqCLMax * kSeqSlotsPerCTA * 6 / 10 / cap[l];
+    const int64_t fit = (int64_t)kSeqCLMax * kSeqSlotsPerCTA * 9 / 10 / cap[l];
     if (fit < S) S = fit < 1 ? 1 : (int)fit;
   }
   if ((int64_t)cap[1] * S > ((int64_t)1 << 26)) return TG_EINVAL;

@@ -25,7 +25,7 @@ COUNTER_FIELDS = ("n", "unique", "lookups", "hits", "misses", "evicted")
 EXPORTS = ("tg_graph_load", "tg_model_load", "tg_embed_batch", "tg_score_edges", "tg_score_stream",
            "tg_cache_reset", "tg_counters_read", "tg_dedup", "tg_sample", "tg_time_encode",
            "tg_kernel_launches", "tg_free", "tg_strerror", "tg_version", "tg_profile_enable",
-           "tg_profile_read", "tg_gemm")
+           "tg_profile_read", "tg_gemm", "tg_superbatch")
 STAGES = ("prep", "dedup", "lookup", "sample", "resolve", "proj_k", "attn", "proj_v", "lnorm", "ffn1", "ffn2",
           "score", "other", "phi")
 
@@ -74,6 +74,8 @@ def lib():
         L.tg_gemm.argtypes = [vp, i32, i32, i32, i32, vp, vp, vp, i32, vp, vp]
         L.tg_kernel_launches.argtypes = [vp]
         L.tg_kernel_launches.restype = i64
+        L.tg_superbatch.argtypes = [vp]
+        L.tg_superbatch.restype = i32
         L.tg_free.argtypes = [vp]
         L.tg_free.restype = None
         L.tg_strerror.argtypes = [ctypes.c_int]
@@ -210,6 +212,10 @@ class Context:
 
     def kernel_launches(self):
         return int(lib().tg_kernel_launches(self.h))
+
+    def superbatch(self):
+        """S in use by score_stream (after the default and the capacity clamp)."""
+        return int(lib().tg_superbatch(self.h))
 
     def close(self):
         if getattr(self, "h", None):
