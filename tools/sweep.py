@@ -4,7 +4,7 @@ The paper's own variants: Fig. 6's ablation (memoization -> + dedup -> + time-en
 precompute) and Table 4's cache-limit sweep {1e4, 1e5, 1e6, 3e6} (P:L450-466,
 plus the 2e6 default of P:L380). Each row is cold-cache chronological passes over a whole
 stream through tg_score_stream (the bench's launch configuration: bf16 GEMM operands,
-superbatch 16), device-timed with CUDA events, L2 flushed before each pass; edges/s is the
+default superbatch), device-timed with CUDA events, L2 flushed before each pass; edges/s is the
 median of --passes passes. Outputs do not depend on the toggles (bit-exact invariance is a
 GPU test), so only speed and the counters move.
 
