@@ -342,6 +342,12 @@ k_probe(LevelDev lv, int S, CacheDev c, int use_cache, int has_ring, long long* 
                     (k0 == kEmptyKey) || (k0 == key) || (*(volatile long long*)(c.ipos + h) < live_lo);
                 if (reusable) {
                   if (atomicCAS(c.ikey + h, k0, kLockedKey) == k0) {
+                    __threadfence();  // re-check under the lock (ABA, see k_probe_ins)
+                    if (k0 != kEmptyKey && k0 != key && *(volatile long long*)(c.ipos + h) >= live_lo) {
+                      atomicExch(c.ikey + h, k0);
+                      h = (h + 1) & c.imask;
+                      continue;
+                    }
                     *(volatile long long*)(c.ipos + h) = pos;
                     __threadfence();
                     atomicExch(c.ikey + h, key);
@@ -815,6 +821,18 @@ __global__ void k_probe_ins(LevelDev lv, CacheDev c, int* err) { pdl_enter();
         const bool reusable = (k0 == kEmptyKey) || (k0 == key) || (*(volatile long long*)(c.ipos + h) < live_lo);
         if (reusable) {
           if (atomicCAS(c.ikey + h, k0, kLockedKey) == k0) {
+            // Re-check under the lock: the CAS only proves ikey still equals k0, not that
+            // the slot is still dead. A concurrent re-insert of the dead key k0 itself (k0
+            // evicted earlier, missed again in this superbatch) can lock, write a live
+            // position and unlock with the same key value between our ipos read and our
+            // CAS -- an ABA that used to overwrite k0's live entry (that key then missed
+            // once while still in the FIFO window). ipos only changes under the lock.
+            __threadfence();
+            if (k0 != kEmptyKey && k0 != key && *(volatile long long*)(c.ipos + h) >= live_lo) {
+              atomicExch(c.ikey + h, k0);  // live after all: release unchanged, probe on
+              h = (h + 1) & c.imask;
+              continue;
+            }
             *(volatile long long*)(c.ipos + h) = pos;
             __threadfence();
             atomicExch(c.ikey + h, key);

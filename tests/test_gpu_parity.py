@@ -287,6 +287,28 @@ def test_superbatch_invariance_bitexact(limit):
         assert counters_dict(ref_log[b], mc.n_layers) == w, b
 
 
+def test_eviction_stress_repeated():
+    """Heavy FIFO churn (limit 700 < one superbatch's misses), repeated cold passes: every pass's
+    per-batch counters equal the Alg. 1 simulator's and the scores are identical across passes.
+    Guards the index-insert ABA (a re-inserted dead key's live entry overwritten by a concurrent
+    insert that had seen the slot dead), which showed up in about 1 % of passes."""
+    cfg, s, flat = setup("config1", n_edges=4000)
+    mc = cfg.model
+    want = _sim_counters(s, flat, mc, 700)
+    from paper_conf_ppopp_wangm23_b200 import counters_dict
+    ref_sc = None
+    for it in range(12):
+        S = (1, 3, 16)[it % 3]
+        ctx = make_ctx(s, flat, mc, cache_limit=700, superbatch=S)
+        sc, log = _stream_gpu(ctx, s, mc.batch)
+        ctx.close()
+        bad = [b for b, w in enumerate(want) if counters_dict(log[b], mc.n_layers) != w]
+        assert not bad, (it, S, bad[:5])
+        if ref_sc is None:
+            ref_sc = sc
+        assert np.array_equal(sc, ref_sc), (it, S)
+
+
 # ------------------------------------------------------------- GEMM kernels
 @pytest.mark.parametrize("prec,rtol,atol", [(0, 1e-5, 1e-5), (1, 1e-5, 1e-4), (2, 2e-2, 2e-2),
                                              (3, 5e-3, 5e-3)])
