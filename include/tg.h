@@ -136,6 +136,21 @@ tg_status tg_embed_batch(tg_ctx* ctx, const int32_t* nodes, const uint32_t* ts, 
 tg_status tg_score_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, const uint32_t* ts,
                          int64_t n_edges, float* scores, void* cuda_stream);
 
+/* Link prediction with negatives (NEXT-3; the TGAT evaluation the paper's task
+ * follows, [37]): embeds nodes/ts as ONE chronological batch (one
+ * deduplicated target list, P:L239 -- e.g. src || dst || negatives, 3 x edges)
+ * and writes scores[p] = sigmoid(MLP(h[pair_a[p]], h[pair_b[p]])) (R10) for
+ * every pair of target indices (0 <= pair_a[p], pair_b[p] < n_targets).
+ * n_targets <= max_batch_targets; n_pairs <= max_batch_targets.
+ * nodes/ts/pair_a/pair_b: all host or all device; scores: either.
+ * Updates the memo cache and the counters like tg_embed_batch.
+ * Errors: TG_EINVAL (sizes, null, host pair index out of range), TG_ESTATE;
+ * a device pair index out of range sets the sticky device error bit 16
+ * (reported by tg_counters_read as TG_EDEVICE) and that pair's score is not written. */
+tg_status tg_score_pairs(tg_ctx* ctx, const int32_t* nodes, const uint32_t* ts, int64_t n_targets,
+                         const int32_t* pair_a, const int32_t* pair_b, int64_t n_pairs, float* scores,
+                         void* cuda_stream);
+
 /* The paper's inference task: the whole edge range [0, n_edges) in
  * chronological batches of `batch` edges (the last one partial, R13), one
  * tg_score_edges per batch, issued from native code without host sync

@@ -264,6 +264,39 @@ void launch_score_head(const float* z, int ldz, const long long* oidx, int M, co
   launch_k(k_score_head, dim3(blocks), dim3(256), 0, st, z, ldz, oidx, M, Wa2, ba2, dn, scores);
 }
 
+// Pair rows for tg_score_pairs (NEXT-3 link prediction with negatives): pair p scores
+// target pa[p] against target pb[p] of a single-batch target list, both resolved through
+// the batch's inverse index (DedupInvert, Alg. 1 l.20); an out-of-range index is an error.
+__global__ void k_pair_rows(const float* __restrict__ HL, int ldh, LevelDev top, int n_targets,
+                            const int32_t* __restrict__ pa, const int32_t* __restrict__ pb, int n_pairs,
+                            const float** __restrict__ rs, const float** __restrict__ rd,
+                            long long* __restrict__ oidx, int* __restrict__ m_dev, int* __restrict__ err) { pdl_enter();
+  if (blockIdx.x == 0 && threadIdx.x == 0) *m_dev = n_pairs;
+  for (int w = blockIdx.x * blockDim.x + threadIdx.x; w < n_pairs; w += gridDim.x * blockDim.x) {
+    const int a = pa[w], b = pb[w];
+    if (a < 0 || a >= n_targets || b < 0 || b >= n_targets) {
+      atomicOr(err, kErrPairIndex);
+      rs[w] = HL;
+      rd[w] = HL;
+      oidx[w] = -1;
+      continue;
+    }
+    rs[w] = HL + (size_t)(top.c_base[0] + top.inv[a]) * ldh;
+    rd[w] = HL + (size_t)(top.c_base[0] + top.inv[b]) * ldh;
+    oidx[w] = w;
+  }
+}
+
+void launch_pair_rows(const float* HL, int ldh, LevelDev top, int n_targets, const int32_t* pa, const int32_t* pb,
+                      int n_pairs, const float** rs, const float** rd, long long* oidx, int* m_dev, int* err,
+                      cudaStream_t st) {
+  int blocks = (n_pairs + 255) / 256;
+  if (blocks < 1) blocks = 1;
+  if (blocks > 1184) blocks = 1184;
+  launch_k(k_pair_rows, dim3(blocks), dim3(256), 0, st, HL, ldh, top, n_targets, pa, pb, n_pairs, rs, rd, oidx,
+           m_dev, err);
+}
+
 __global__ void k_invert(const float* __restrict__ HL, int ldh, LevelDev top, int n, int dn,
                          float* __restrict__ out) { pdl_enter();
   const long long tot = (long long)n * dn;

@@ -963,7 +963,7 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
       TRY(tc_prepare_weights(ctx->Wa1, dnp, 2 * dnp, cfg->precision, &ctx->tcWa1, ctx->owned));
       if (cfg->precision == TG_PREC_BF16)
         TRY(tc_prepare_weights(ctx->Wa1, dnp, 2 * dnp, TG_PREC_TF32, &ctx->tcWa1g, ctx->owned));
-    const size_t ne = (size_t)S * ((cfg->max_batch_targets + 1) / 2);
+    const size_t ne = std::max((size_t)S * ((cfg->max_batch_targets + 1) / 2), (size_t)cfg->max_batch_targets);
     TRY(dalloc(ctx, &ctx->sc_rs, ne));
     TRY(dalloc(ctx, &ctx->sc_rd, ne));
     TRY(dalloc(ctx, &ctx->sc_oidx, ne));
@@ -1203,6 +1203,83 @@ tg_status tg_score_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, co
   TRY(stream_edges(ctx, o.src, o.dst, o.ts, n_edges, (int)n_edges, o.out, nullptr, st));
   if (o.host_out) {
     CK(cudaMemcpyAsync(scores, o.out, n_edges * 4, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+  }
+  return TG_OK;
+}
+
+tg_status tg_score_pairs(tg_ctx* ctx, const int32_t* nodes, const uint32_t* ts, int64_t n_targets,
+                         const int32_t* pair_a, const int32_t* pair_b, int64_t n_pairs, float* scores,
+                         void* cuda_stream) {
+  if (!ctx) return TG_EINVAL;
+  if (!ctx->loaded) return TG_ESTATE;
+  if (ctx->broken) return TG_ECUDA;
+  const int64_t ne = (int64_t)ctx->cfg.max_batch_targets;  // the score workspace holds at least this many
+  if (n_targets < 0 || n_targets > ctx->cap[ctx->L] || n_pairs < 0 || n_pairs > ne ||
+      (n_targets > 0 && (!nodes || !ts)) || (n_pairs > 0 && (!pair_a || !pair_b || !scores)))
+    return TG_EINVAL;
+  if (n_pairs == 0 && n_targets == 0) return TG_OK;
+  if (n_pairs > 0 && n_targets == 0) return TG_EINVAL;
+  cudaStream_t st = (cudaStream_t)cuda_stream;
+  CK(cudaSetDevice(ctx->device));
+  const bool dev_in = is_device_ptr(nodes);
+  const bool dev_out = n_pairs == 0 || is_device_ptr(scores);
+  if (!dev_in && n_pairs > 0) {  // host pairs: range-checked here, before any launch
+    for (int64_t p = 0; p < n_pairs; ++p)
+      if (pair_a[p] < 0 || pair_a[p] >= n_targets || pair_b[p] < 0 || pair_b[p] >= n_targets) return TG_EINVAL;
+  }
+  const int32_t* dn = nodes;
+  const uint32_t* dt = ts;
+  const int32_t* da = pair_a;
+  const int32_t* db = pair_b;
+  float* dout = scores;
+  if (!dev_in || !dev_out) {
+    const size_t n8 = ((size_t)n_targets * 8 + 15) & ~(size_t)15, p8 = ((size_t)n_pairs * 8 + 15) & ~(size_t)15;
+    TRY(ensure_stage(ctx, n8 + p8 + (size_t)n_pairs * 4 + 64));
+    char* stg = (char*)ctx->stage;
+    if (!dev_in) {
+      CK(cudaMemcpyAsync(stg, nodes, n_targets * 4, cudaMemcpyHostToDevice, st));
+      CK(cudaMemcpyAsync(stg + n_targets * 4, ts, n_targets * 4, cudaMemcpyHostToDevice, st));
+      CK(cudaMemcpyAsync(stg + n8, pair_a, n_pairs * 4, cudaMemcpyHostToDevice, st));
+      CK(cudaMemcpyAsync(stg + n8 + n_pairs * 4, pair_b, n_pairs * 4, cudaMemcpyHostToDevice, st));
+      dn = (const int32_t*)stg;
+      dt = (const uint32_t*)(stg + n_targets * 4);
+      da = (const int32_t*)(stg + n8);
+      db = (const int32_t*)(stg + n8 + n_pairs * 4);
+    }
+    if (!dev_out) dout = (float*)(stg + n8 + p8);
+  }
+  // embeddings of the (deduplicated) target list: one Alg. 1 batch, cache on
+  launch_prep_nodes(dn, dt, (int)n_targets, ctx->lv[ctx->L], st);
+  TRY(launched(ctx));
+  EdgeSrc none{};
+  TRY(run_superbatch(ctx, 1, false, none, (int)n_targets, st));
+  if (n_pairs > 0) {
+    Prof pf(ctx, TG_ST_SCORE, st);
+    launch_pair_rows(ctx->HL, ctx->dnp, ctx->lv[ctx->L], (int)n_targets, da, db, (int)n_pairs, ctx->sc_rs,
+                     ctx->sc_rd, ctx->sc_oidx, ctx->sc_m, ctx->err, st);
+    GemmArgs g{};  // hidden layer of the affinity MLP over the pairs (R10)
+    g.a_rows0 = ctx->sc_rs;
+    g.K0 = ctx->dnp;
+    g.a_rows1 = ctx->sc_rd;
+    g.K = 2 * ctx->dnp;
+    g.B = ctx->Wa1;
+    g.N = ctx->dnp;
+    g.bias = ctx->ba1;
+    g.relu = 1;
+    g.C = ctx->sc_z;
+    g.ldc = ctx->dnp;
+    g.m_dev = ctx->sc_m;
+    g.m_max = (int)n_pairs;
+    if (ctx->cfg.precision == TG_PREC_BF16) launch_gemm_tc(g, ctx->tcWa1g, TG_PREC_TF32, st);
+    else if (ctx->cfg.precision != TG_PREC_FP32) launch_gemm_tc(g, ctx->tcWa1, ctx->cfg.precision, st);
+    else launch_gemm_simt(g, st);
+    launch_score_head(ctx->sc_z, ctx->dnp, ctx->sc_oidx, (int)n_pairs, ctx->Wa2, ctx->ba2, ctx->d_n, dout, st);
+    TRY(launched(ctx, 3));
+  }
+  TRY(finish(ctx, 1, nullptr, 0, st));
+  if (!dev_out) {
+    CK(cudaMemcpyAsync(scores, dout, n_pairs * 4, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
   }
   return TG_OK;

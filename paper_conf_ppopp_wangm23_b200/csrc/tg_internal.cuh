@@ -89,7 +89,7 @@ inline cudaError_t launch_k_cluster(void (*kern)(KArgs...), dim3 grid, dim3 bloc
 }
 
 // device error bits (sticky)
-enum : int { kErrNodeRange = 1, kErrIndexFull = 2, kErrDedupFull = 4, kErrEidRange = 8 };
+enum : int { kErrNodeRange = 1, kErrIndexFull = 2, kErrDedupFull = 4, kErrEidRange = 8, kErrPairIndex = 16 };
 
 __host__ __device__ inline int round4(int x) { return (x + 3) & ~3; }
 
@@ -327,6 +327,10 @@ void launch_score_rows(const float* HL, int ldh, LevelDev top, int S, EdgeSrc es
                        const float** rd, long long* oidx, int* m_dev, cudaStream_t st);
 void launch_score_head(const float* z, int ldz, const long long* oidx, int M, const float* Wa2, float ba2, int dn,
                        float* scores, cudaStream_t st);
+// Row pointers of target pairs (pa[p], pb[p]) of a single-batch target list (tg_score_pairs).
+void launch_pair_rows(const float* HL, int ldh, LevelDev top, int n_targets, const int32_t* pa, const int32_t* pb,
+                      int n_pairs, const float** rs, const float** rd, long long* oidx, int* m_dev, int* err,
+                      cudaStream_t st);
 // out[i] = H_L[q(i)] for a single-batch embed call (DedupInvert, Alg. 1 l.20).
 void launch_invert(const float* HL, int ldh, LevelDev top, int n, int dn, float* out, cudaStream_t st);
 void launch_prep_nodes(const int32_t* nodes, const uint32_t* ts, int n, LevelDev top, cudaStream_t st);

@@ -23,7 +23,7 @@ TG_NCOUNTERS = TG_CNT_TDIRECT + 1
 COUNTER_FIELDS = ("n", "unique", "lookups", "hits", "misses", "evicted")
 
 EXPORTS = ("tg_graph_load", "tg_model_load", "tg_embed_batch", "tg_score_edges", "tg_score_stream",
-           "tg_cache_reset", "tg_counters_read", "tg_dedup", "tg_sample", "tg_time_encode",
+           "tg_score_pairs", "tg_cache_reset", "tg_counters_read", "tg_dedup", "tg_sample", "tg_time_encode",
            "tg_kernel_launches", "tg_free", "tg_strerror", "tg_version", "tg_profile_enable",
            "tg_profile_read", "tg_gemm", "tg_superbatch")
 STAGES = ("prep", "dedup", "lookup", "sample", "resolve", "proj_k", "attn", "proj_v", "lnorm", "ffn1", "ffn2",
@@ -64,6 +64,7 @@ def lib():
         L.tg_embed_batch.argtypes = [vp, vp, vp, i64, vp, vp]
         L.tg_score_edges.argtypes = [vp, vp, vp, vp, i64, vp, vp]
         L.tg_score_stream.argtypes = [vp, vp, vp, vp, i64, i32, vp, vp, vp]
+        L.tg_score_pairs.argtypes = [vp, vp, vp, i64, vp, vp, i64, vp, vp]
         L.tg_cache_reset.argtypes = [vp, i64]
         L.tg_counters_read.argtypes = [vp, vp, i32]
         L.tg_dedup.argtypes = [vp, vp, vp, i64, vp, vp, vp, vp, vp]
@@ -82,7 +83,7 @@ def lib():
         L.tg_strerror.restype = ctypes.c_char_p
         L.tg_version.restype = ctypes.c_char_p
         for f in ("tg_graph_load", "tg_model_load", "tg_embed_batch", "tg_score_edges", "tg_score_stream",
-                  "tg_cache_reset", "tg_counters_read", "tg_dedup", "tg_sample", "tg_time_encode",
+                  "tg_score_pairs", "tg_cache_reset", "tg_counters_read", "tg_dedup", "tg_sample", "tg_time_encode",
                   "tg_profile_enable", "tg_profile_read", "tg_gemm"):
             getattr(L, f).restype = ctypes.c_int
         _lib = L
@@ -163,6 +164,11 @@ class Context:
     def score_edges(self, src, dst, ts, scores, stream=None):
         _check(lib().tg_score_edges(self.h, _ptr(src), _ptr(dst), _ptr(ts), int(src.shape[0]), _ptr(scores),
                                     _stream(stream)), "tg_score_edges")
+        return scores
+
+    def score_pairs(self, nodes, ts, pair_a, pair_b, scores, stream=None):
+        _check(lib().tg_score_pairs(self.h, _ptr(nodes), _ptr(ts), int(nodes.shape[0]), _ptr(pair_a), _ptr(pair_b),
+                                    int(pair_a.shape[0]), _ptr(scores), _stream(stream)), "tg_score_pairs")
         return scores
 
     def score_stream(self, src, dst, ts, batch, scores, batch_counters=None, stream=None):

@@ -167,6 +167,41 @@ def test_embed_parity(name, L, prec):
         assert ok, (rep, err, nbad)
 
 
+@pytest.mark.parametrize("prec", [0, 2])
+@pytest.mark.parametrize("name", ["tiny", "config1"])
+def test_score_pairs_negatives(name, prec):
+    """NEXT-3: link prediction with negatives ([37]). One batch's target list is
+    src || dst || neg at the edge times (3B targets, one dedup), scored as positive pairs
+    (src, dst) and negative pairs (src, neg); both compared with the oracle's embed + score."""
+    cfg, s, flat = setup(name)
+    mc = cfg.model
+    ctx = make_ctx(s, flat, mc, max_targets=600, precision=prec)
+    o = make_oracle(s, flat, mc)
+    rng = np.random.default_rng(11)
+    B = 200 if name != "config1" else 40
+    for rep, lo in enumerate((0, B, B)):                # third call: repeated batch, cache hits
+        src, dst, ts = s.src[lo:lo + B], s.dst[lo:lo + B], s.ts[lo:lo + B]
+        neg = rng.integers(1, s.n_nodes + 1, B)        # seeded uniform negative sampler
+        nodes = np.concatenate([src, dst, neg]).astype(np.int32)
+        tt = np.concatenate([ts, ts, ts]).astype(np.uint32)
+        pa = np.concatenate([np.arange(B), np.arange(B)]).astype(np.int32)
+        pb = np.concatenate([B + np.arange(B), 2 * B + np.arange(B)]).astype(np.int32)
+        if rep == 1:                                    # host buffers through the same call
+            got = np.zeros(2 * B, np.float32)
+            ctx.score_pairs(nodes, tt.view(np.int32), pa, pb, got)
+        else:
+            out = torch.zeros(2 * B, dtype=torch.float32, device="cuda")
+            ctx.score_pairs(dev(nodes), dev(tt.view(np.int32)), dev(pa), dev(pb), out)
+            torch.cuda.synchronize()
+            got = out.cpu().numpy()
+        h = o.embed(mc.n_layers, nodes, tt.astype(np.int64))
+        ref = o.score(h[pa], h[pb])
+        ok, err, nbad = close(got, ref, *TOL[prec])
+        assert ok, (rep, err, nbad)
+    with pytest.raises(Exception):                      # host pair index out of range
+        ctx.score_pairs(nodes, tt.view(np.int32), pa, np.full_like(pb, 3 * B), np.zeros(2 * B, np.float32))
+
+
 def test_embed_empty_and_single():
     cfg, s, flat = setup("tiny")
     ctx = make_ctx(s, flat, cfg.model)
