@@ -178,7 +178,7 @@ def test_score_pairs_negatives(name, prec):
     ctx = make_ctx(s, flat, mc, max_targets=600, precision=prec)
     o = make_oracle(s, flat, mc)
     rng = np.random.default_rng(11)
-    B = 200 if name != "config1" else 40
+    B = min(200 if name != "config1" else 40, s.n_edges // 2)
     for rep, lo in enumerate((0, B, B)):                # third call: repeated batch, cache hits
         src, dst, ts = s.src[lo:lo + B], s.dst[lo:lo + B], s.ts[lo:lo + B]
         neg = rng.integers(1, s.n_nodes + 1, B)        # seeded uniform negative sampler
