@@ -1,29 +1,36 @@
-"""Benchmark: TGAT inference edges/s over a Reddit-shaped stream (BASELINE.json).
+"""Benchmark: TGAT inference edges/s over a Reddit-shaped stream (BASELINE.json configs[2]).
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--config reddit]
-                    [--precision fp32|tf32x3|bf16] [--impl ours|reference]
+                    [--precision tf32x3|bf16|fp32|tf32] [--scaling strong|weak]
+                    [--impl ours|reference]
 
-A *step* is one full chronological pass (batches of 200 edges) over
-the rank's stream, cold cache (tg_cache_reset, as in the paper's runs), i.e.
-the whole hot path S1-S16 per batch. For N > 1 (torchrun, NCCL), one process
-per GPU:
-  --scaling weak   (default) every rank processes its own Reddit-shaped stream
-                   (independent seed): fixed work per GPU;
-  --scaling strong the single stream is sharded into contiguous batch ranges
-                   [r*nb/N, (r+1)*nb/N) (north_star's deployment).
-NCCL only gathers the scores and all-reduces the counters at the end of a
-pass; there is no per-batch collective (batches are independent).
+A *step* is one full chronological pass (batches of 200 edges) over the rank's
+share of the stream, cold cache (tg_cache_reset, as in the paper's runs), i.e. the whole
+hot path S1-S16 of SURVEY 8(a) for every batch.
 
---impl reference times the oracle (oracle/, plain float64 CPU TGAT, the
-paper's baseline role) on the host cores on a bounded sample of the same
-workload (rank 0 only).
+Headline precision: tf32x3 -- the fp32-level tensor-core mode (3-term tf32 split, fp32
+accumulate, fp32 activations between the GEMMs; parity 1e-5 + 1e-4|ref|, R17). The paper
+computes in fp32. The same line carries a second measurement in bf16 GEMM operands
+(`"bf16"` key, parity rtol 2e-2) for context.
+
+Multi-GPU (north_star): one process per GPU. `--gpus N` without a torchrun
+environment re-executes itself through torch.distributed.run (127.0.0.1); under torchrun
+WORLD_SIZE must equal --gpus.
+  --scaling strong (default) the stream is sharded into contiguous batch ranges
+                   [r*nb/N, (r+1)*nb/N) (north_star's partition; each shard starts cold);
+  --scaling weak   every rank processes its own Reddit-shaped stream (independent seed).
+NCCL only gathers the scores and all-reduces the counters at the end of a pass; there is no
+per-batch collective (batches are independent given the graph).
+
+--impl reference times the oracle (oracle/, plain float64 CPU TGAT, the paper's baseline
+role) on the host cores on a bounded sample of the same workload (rank 0 only).
 """
 import argparse
 import json
 import os
+import socket
 import subprocess
 import sys
-import threading
 import time
 
 import numpy as np
@@ -32,6 +39,13 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 PEAKS_FALLBACK = {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}
+# nominal dense tensor peaks of B200 (B200_PROFILING.md), used only as ratios to the measured
+# bf16 peak: tf32 = bf16 x 1.1 / 2.25; the tf32x3 mode issues 3 tf32 MMAs per fp32-level product
+NOMINAL_TF = {"bf16": 2250.0, "tf32": 1100.0}
+PAPER_CONTEXT = ("TGOpt (PPoPP'23) geomean inference speedup over the official TGAT: 4.9x on 2x Xeon Gold "
+                 "6348 (56 cores, 2.6 GHz), 2.9x on 1x Tesla V100 16 GB (AWS p3.2xlarge) (P:L13, P:L376); "
+                 "derived paper throughput on jodie-lastfm ~14.8k edges/s (V100, Table 3). Context, not target: "
+                 "different hardware, real datasets, trained weights.")
 
 
 def load_peaks():
@@ -43,6 +57,25 @@ def load_peaks():
     d = dict(PEAKS_FALLBACK)
     d["source"] = "fallback (B200_PROFILING.md)"
     return d
+
+
+def tensor_peak(peaks, prec, sustained=True):
+    """Effective TFLOP/s of an fp32-level (or bf16) product in the given mode."""
+    bf = peaks.get("bf16_tflops_sustained" if sustained else "bf16_tflops", peaks["bf16_tflops"])
+    if prec == "bf16":
+        return bf
+    tf32 = bf * NOMINAL_TF["tf32"] / NOMINAL_TF["bf16"]
+    return tf32 / 3.0 if prec == "tf32x3" else tf32
+
+
+def cpu_model():
+    try:
+        for l in open("/proc/cpuinfo"):
+            if l.startswith("model name"):
+                return l.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
 
 
 # ---------------------------------------------------------------- clocks
@@ -99,16 +132,26 @@ class ClockSampler:
 
 
 # --------------------------------------------------------- reference arm
-def run_reference(args, cfg):
-    """The oracle (plain float64 CPU TGAT, no TGOpt optimisations) on host cores."""
+def _oracle(cfg, name):
     from synth import make_stream, make_params
     from oracle.tgat import Model, TemporalGraph, TGAT
-    from threadpoolctl import threadpool_info
     mc = cfg.model
-    s = make_stream(args.config)
+    s = make_stream(name)
     flat = make_params(mc.n_layers, mc.n_heads, s.d_n, s.d_e)
     o = TGAT(Model(flat, mc.n_layers, mc.n_heads, s.d_n, s.d_e), TemporalGraph(s.n_nodes, s.src, s.dst, s.ts),
              s.node_feat, s.edge_feat, mc.n_neighbors)
+    return s, o
+
+
+def _threads():
+    from threadpoolctl import threadpool_info
+    return int(max([d.get("num_threads", 1) for d in threadpool_info()] + [1]))
+
+
+def run_reference(args, cfg):
+    """The oracle (plain float64 CPU TGAT, no TGOpt optimisations) on host cores."""
+    mc = cfg.model
+    s, o = _oracle(cfg, args.config)
     nb = (s.n_edges + mc.batch - 1) // mc.batch
     total = args.warmup + args.steps
     picks = np.linspace(0, nb - 1, total).astype(int)
@@ -121,29 +164,24 @@ def run_reference(args, cfg):
         if i >= args.warmup:
             times.append(dt)
             edges += hi - lo
-    cores = max([d.get("num_threads", 1) for d in threadpool_info()] + [1])
     val = edges / sum(times)
-    sample = f"{args.steps} stratified batches of {mc.batch} edges of the {args.config} stream (1 batch per step)"
+    sample = (f"{args.steps} stratified batches of {mc.batch} edges of the {args.config} stream (1 batch per "
+              f"step; float64 NumPy/OpenBLAS oracle, not an fp32 C++ program)")
     line = {"impl": "reference", "metric": "edges_per_sec", "value": val, "unit": "edges/s", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * float(np.mean(times)),
             "higher_is_better": True, "scaling": "none", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic", "config": {"workload": args.config, "batch": mc.batch,
                                             "n_layers": mc.n_layers, "k": mc.n_neighbors, "sample": sample},
-            "cpu_baseline": {"value": val, "unit": "edges/s", "cores": cores, "kind": "oracle", "sample": sample},
+            "cpu_baseline": {"value": val, "unit": "edges/s", "cores": _threads(), "cpu_model": cpu_model(),
+                             "kind": "oracle", "sample": sample},
             "e2e": {"value": val, "unit": "edges/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
 
 def cpu_baseline(cfg, name, seconds=15.0):
     """Oracle edges/s on a bounded sample (rank 0, N = 1): stratified batches until ~`seconds`."""
-    from synth import make_stream, make_params
-    from oracle.tgat import Model, TemporalGraph, TGAT
-    from threadpoolctl import threadpool_info
     mc = cfg.model
-    s = make_stream(name)
-    flat = make_params(mc.n_layers, mc.n_heads, s.d_n, s.d_e)
-    o = TGAT(Model(flat, mc.n_layers, mc.n_heads, s.d_n, s.d_e), TemporalGraph(s.n_nodes, s.src, s.dst, s.ts),
-             s.node_feat, s.edge_feat, mc.n_neighbors)
+    s, o = _oracle(cfg, name)
     nb = (s.n_edges + mc.batch - 1) // mc.batch
     order = np.linspace(0, nb - 1, 16).astype(int)
     t_all, e_all, used = 0.0, 0, []
@@ -156,67 +194,104 @@ def cpu_baseline(cfg, name, seconds=15.0):
         used.append(int(b))
         if t_all > seconds:
             break
-    cores = max([d.get("num_threads", 1) for d in threadpool_info()] + [1])
-    return {"value": e_all / t_all, "unit": "edges/s", "cores": int(cores), "kind": "oracle",
-            "sample": f"{len(used)} stratified batches {used} of {mc.batch} edges ({e_all} edges, {t_all:.1f} s)"}
+    return {"value": e_all / t_all, "unit": "edges/s", "cores": _threads(), "cpu_model": cpu_model(),
+            "kind": "oracle",
+            "sample": (f"{len(used)} stratified batches {used} of {mc.batch} edges ({e_all} edges, {t_all:.1f} s); "
+                       f"float64 NumPy/OpenBLAS oracle (oracle/tgat.py)")}
 
 
-# ---------------------------------------------------------------- main
-def main():
-    ap = argparse.ArgumentParser()
-    ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=5)
-    ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", default="reddit")
-    ap.add_argument("--precision", default="bf16", choices=["fp32", "tf32x3", "bf16", "tf32"])
-    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"])
-    ap.add_argument("--superbatch", type=int, default=0)
-    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--no-profile", action="store_true")
-    args = ap.parse_args()
+# ---------------------------------------------------------- roofline
+def model_dims(s, mc):
+    d_n, d_e = s.d_n, s.d_e
+    D = d_n + d_e + d_n
+    return d_n, d_e, D, mc.n_neighbors, mc.n_heads
 
-    from synth import get_config
-    cfg = get_config(args.config)
-    mc = cfg.model
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
 
-    if args.impl == "reference":
-        if rank == 0:
-            run_reference(args, cfg)
-        return
+def flops_spec(s, mc):
+    """F_M of SURVEY 8(d): one M + FFN in the paper's form (per-neighbour K/V projections)."""
+    d_n, d_e, D, k, H = model_dims(s, mc)
+    return 2 * D * D + 4 * k * D * D + 4 * k * D + 2 * D * D + 2 * (D + d_n) * d_n + 2 * d_n * d_n
 
-    import dataclasses
+
+def flops_absorbed(s, mc):
+    """The same embedding in the absorbed form this build runs: G1..G4 plus the
+    per-neighbour dot products / weighted sums of the attention kernel."""
+    d_n, d_e, D, k, H = model_dims(s, mc)
+    g1 = 2 * (H * D) * d_n
+    g2 = 2 * D * (H * D)
+    g3 = 2 * d_n * (D + d_n)
+    g4 = 2 * d_n * d_n
+    attn = 4 * H * k * D
+    return {"G1": g1, "G2": g2, "G3": g3, "G4": g4, "attn": attn, "total": g1 + g2 + g3 + g4 + attn}
+
+
+def gather_bytes(s, mc):
+    """SURVEY 8(d) unit: (k+1)(d_n + d_e) * 4 B gathered per computed embedding (Phi rows come
+    from L2 or are computed)."""
+    d_n, d_e, D, k, H = model_dims(s, mc)
+    return (k + 1) * (d_n + d_e) * 4
+
+
+def front_bytes(per, L, k, d_n):
+    """SURVEY 8(d)'s dedup/probe/sample/store traffic of one batch from its counters."""
+    b = 0
+    for l in range(1, L + 1):
+        b += 30 * per[f"l{l}_n"]                       # dedup entry (key read, hash, inv write)
+        b += 24 * per[f"l{l}_lookups"]                 # cache probe
+        b += (k * 12 + 120) * per[f"l{l}_misses"]      # sampled target: k (node, eid, t) + search
+        if l < L:
+            b += (d_n * 4 + 8) * per[f"l{l}_misses"]   # CacheStore payload + key
+    return b
+
+
+def ideal_time(per_batch, s, mc, peaks, prec):
+    """End-to-end ideal time = sum_b max(F_b / P_tensor, B_b / BW_HBM), from the
+    measured per-batch counters, in both formulations (paper form and absorbed form)."""
+    L, k = mc.n_layers, mc.n_neighbors
+    bw = peaks["hbm_gbs"] * 1e9
+    pt = tensor_peak(peaks, prec) * 1e12
+    fs, fa, gb = flops_spec(s, mc), flops_absorbed(s, mc)["total"], gather_bytes(s, mc)
+    t_spec = t_abs = 0.0
+    F_spec = F_abs = B = 0
+    for p in per_batch:
+        m = sum(p[f"l{l}_misses"] for l in range(1, L + 1))
+        bb = m * gb + front_bytes(p, L, k, s.d_n)
+        t_spec += max(m * fs / pt, bb / bw)
+        t_abs += max(m * fa / pt, bb / bw)
+        F_spec += m * fs
+        F_abs += m * fa
+        B += bb
+    return {"ideal_ms_paper_form": 1e3 * t_spec, "ideal_ms_absorbed_form": 1e3 * t_abs,
+            "flops_paper_form": F_spec, "flops_absorbed_form": F_abs, "bytes": B,
+            "tensor_peak_tflops": pt / 1e12, "hbm_gbs": bw / 1e9}
+
+
+def traffic_record(config, prec):
+    """Measured DRAM bytes per launch of the dominant kernel from the committed ncu capture of the
+    same build (profiles/traffic.json: {config: {prec: {kernel: {...}}}}), stamped with its S and
+    targets per launch; None if not captured."""
+    p = os.path.join(ROOT, "profiles", "traffic.json")
+    if not os.path.exists(p):
+        return None
+    return json.load(open(p)).get(config, {}).get(prec)
+
+
+# ---------------------------------------------------------------- one precision arm
+def measure(args, prec_name, s, flat, mc, ctx_kw, shard, world, rank, local, dist, steps, warmup,
+            profile=True):
     import torch
-    import torch.distributed as dist
-    from synth import make_stream, make_params
     from paper_conf_ppopp_wangm23_b200 import (Context, TG_NCOUNTERS, counters_dict, TG_PREC_FP32,
                                               TG_PREC_TF32X3, TG_PREC_BF16, TG_PREC_TF32)
-    from paper_conf_ppopp_wangm23_b200.shard import shard_batches, gather_scores, reduce_counters
-
-    torch.cuda.set_device(local)
-    if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    prec = {"fp32": TG_PREC_FP32, "tf32x3": TG_PREC_TF32X3, "bf16": TG_PREC_BF16, "tf32": TG_PREC_TF32}[args.precision]
-
-    if args.scaling == "weak" and world > 1:
-        s = make_stream(dataclasses.replace(cfg.stream, seed=cfg.stream.seed + 7919 * rank))
-    else:
-        s = make_stream(args.config)
-    flat = make_params(mc.n_layers, mc.n_heads, s.d_n, s.d_e)
+    from paper_conf_ppopp_wangm23_b200.shard import gather_scores, reduce_counters
+    prec = {"fp32": TG_PREC_FP32, "tf32x3": TG_PREC_TF32X3, "bf16": TG_PREC_BF16, "tf32": TG_PREC_TF32}[prec_name]
+    b0, b1, e0, e1 = shard
     B = mc.batch
-    if args.scaling == "strong":
-        b0, b1, e0, e1 = shard_batches(s.n_edges, B, rank, world)
-    else:
-        b0, b1, e0, e1 = 0, (s.n_edges + B - 1) // B, 0, s.n_edges
     E_rank = e1 - e0
     E_job = s.n_edges if args.scaling == "strong" else s.n_edges * world
     ctx = Context.from_stream(s, device=local)
     ctx.load_model(flat, n_layers=mc.n_layers, n_heads=mc.n_heads, n_neighbors=mc.n_neighbors,
                    max_batch_targets=2 * B, cache_limit=mc.cache_limit, time_window=mc.time_window,
-                   precision=prec, superbatch=args.superbatch)
+                   precision=prec, superbatch=args.superbatch, **ctx_kw)
     dev = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
     src, dst, ts = dev(s.src[e0:e1]), dev(s.dst[e0:e1]), dev(s.ts[e0:e1].view(np.int32))
     scores = torch.zeros(E_rank, dtype=torch.float32, device="cuda")
@@ -242,17 +317,17 @@ def main():
         collect(sc)
         return launches
 
-    for _ in range(args.warmup):
+    for _ in range(warmup):
         step()
     torch.cuda.synchronize()
     # ---- timed region: K passes, L2 flushed before each, events on the launching stream
-    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
     launches = 0
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
     with ClockSampler(local) as clk:
-        for i in range(args.steps):
+        for i in range(steps):
             flush.zero_()
             ev[i][0].record(stream)
             launches += step()
@@ -267,7 +342,7 @@ def main():
         tt = torch.tensor([t_rank], dtype=torch.float64, device="cuda")
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         t_max = float(tt.item())
-    value = args.steps * E_job / t_max
+    value = steps * E_job / t_max
 
     # ---- per-batch counters of the last pass (hit rates, dedup ratios)
     lg = log.cpu().numpy().reshape(nbr, TG_NCOUNTERS)
@@ -280,16 +355,28 @@ def main():
     def rate(a, b):
         return a / b if b else None
 
-    hit_mean = float(np.mean([p["l1_hits"] / p["l1_lookups"] for p in per if p["l1_lookups"]]))
+    L = mc.n_layers
+    cached = range(1, L)
+    hit_mean = {f"l{l}": float(np.mean([p[f"l{l}_hits"] / p[f"l{l}_lookups"] for p in per if p[f"l{l}_lookups"]]))
+                for l in cached}
+    win = []                                     # Fig. 7: hit rate over 10-batch windows
+    for w0 in range(0, len(per) - 9):
+        hh = sum(p["l1_hits"] for p in per[w0:w0 + 10])
+        ll = sum(p["l1_lookups"] for p in per[w0:w0 + 10])
+        if ll:
+            win.append(hh / ll)
     stats = {
-        "l1_hit_rate_mean_of_batches": hit_mean,
-        "l1_hit_rate_global": rate(tot["l1_hits"], tot["l1_lookups"]),
+        "hit_rate_mean_of_batches": hit_mean,
+        "hit_rate_global": {f"l{l}": rate(tot[f"l{l}_hits"], tot[f"l{l}_lookups"]) for l in cached},
+        "l1_hit_rate_10batch_window": ({"min": float(np.min(win)), "median": float(np.median(win)),
+                                        "max": float(np.max(win)), "first": float(win[0]),
+                                        "last": float(win[-1])} if win else None),
         "dedup_ratio": {f"l{l}": rate(tot[f"l{l}_n"] - tot[f"l{l}_unique"], tot[f"l{l}_n"])
-                        for l in range(1, mc.n_layers + 1)},
-        "l0_dup_ratio_na": "layer 0 is not deduplicated (P:L239)",
+                        for l in range(1, L + 1)},
+        "l0_dup_ratio_na": "layer 0 is not deduplicated (P:L239); see profiles/*/calibration.json",
         "time_table_hit_rate": rate(tot["t_table"], tot["t_table"] + tot["t_direct"]),
-        "computed_embeddings": {f"l{l}": tot[f"l{l}_misses"] for l in range(1, mc.n_layers + 1)},
-        "cache_evictions": tot["l1_evicted"],
+        "computed_embeddings": {f"l{l}": tot[f"l{l}_misses"] for l in range(1, L + 1)},
+        "cache_evictions": tot["l1_evicted"] if L > 1 else 0,
     }
 
     # ---- e2e: same metric through the public API with pinned HOST buffers
@@ -298,7 +385,7 @@ def main():
     hs_ts = torch.from_numpy(np.ascontiguousarray(s.ts[e0:e1].view(np.int32))).pin_memory()
     hs_sc = torch.zeros(E_rank, dtype=torch.float32).pin_memory()
     e2e_t = []
-    for i in range(args.steps + 1):
+    for i in range(steps + 1):
         if world > 1:
             dist.barrier()
         flush.zero_()
@@ -306,7 +393,8 @@ def main():
         t0 = time.perf_counter()
         ctx.cache_reset()
         ctx.score_stream(hs_src, hs_dst, hs_ts, B, hs_sc, None, stream=stream)  # H2D in, D2H out, synced
-        collect(hs_sc.cuda(non_blocking=False)) if world > 1 else None
+        if world > 1:
+            collect(hs_sc.cuda(non_blocking=False))
         t1 = time.perf_counter() - t0
         if i:
             e2e_t.append(t1)
@@ -315,14 +403,14 @@ def main():
         tt = torch.tensor([e2e_rank], dtype=torch.float64, device="cuda")
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         e2e_rank = float(tt.item())
-    e2e_val = args.steps * E_job / e2e_rank
+    e2e_val = steps * E_job / e2e_rank
     assert np.array_equal(hs_sc.numpy(), scores.cpu().numpy()), "host-buffer path disagrees with device path"
 
-    # ---- per-stage device timing (separate profiled pass of the same workload)
+    # ---- per-stage device timing (separate profiled pass of the same workload) + roofline
     peaks = load_peaks()
-    roof = None
-    stages = None
-    if not args.no_profile:
+    ms_step = 1e3 * t_max / steps
+    roof, kernels, stages, ideal = None, None, None, None
+    if profile:
         ctx.profile(True)
         ctx.cache_reset()
         ctx.score_stream(src, dst, ts, B, scores, None, stream=stream)
@@ -330,50 +418,178 @@ def main():
         stages = ctx.profile_read()
         ctx.profile(False)
         c = ctx.counters()
-        D = s.d_n + s.d_e + s.d_n
-        k = mc.n_neighbors
-        n_targets = sum(c[f"l{l}_misses"] for l in range(1, mc.n_layers + 1))
-        # algorithmic bytes of the attention kernel per computed target:
-        # neighbour rows h_j + e_ij, Phi rows (table or computed), u in and c out (2 x H x D),
-        # per-slot metadata (row ptr 8 + eid 4 + node 4 + t 4 B)
-        per_target = k * (s.d_n + s.d_e) * 4 + k * s.d_n * 4 + 2 * mc.n_heads * D * 4 + k * 20
+        n_targets = sum(c[f"l{l}_misses"] for l in range(1, L + 1))
+        d_n, d_e, D, k, H = model_dims(s, mc)
+        fa = flops_absorbed(s, mc)
+        tpk = tensor_peak(peaks, prec_name)
+        kernels = {}
+        # attention (gather-bound): SURVEY 8(d) bytes (k+1)(d_n+d_e)*4 per computed target
         attn_ms, attn_n = stages["attn"]
-        achieved = (n_targets * per_target) / (attn_ms / 1e3) / 1e9
+        gb = gather_bytes(s, mc)
+        act = 2 if prec_name == "bf16" else 4
+        absorbed_io = k * (d_n + d_e) * 4 + H * D * 4 + H * D * act  # neighbour rows + u in + c out
+        kernels["k_attn_g"] = {"bound": "hbm", "unit": "GB/s", "peak": peaks["hbm_gbs"],
+                               "bytes_per_target": gb, "targets": n_targets, "launches": attn_n,
+                               "avg_launch_us": 1e3 * attn_ms / max(1, attn_n),
+                               "achieved": n_targets * gb / (attn_ms / 1e3) / 1e9,
+                               "achieved_absorbed_io": n_targets * absorbed_io / (attn_ms / 1e3) / 1e9,
+                               "absorbed_io_bytes_per_target": absorbed_io,
+                               "share_of_step": attn_ms / ms_step}
+        for st_name, g in (("proj_k", "G1"), ("proj_v", "G2"), ("ffn1", "G3"), ("ffn2", "G4")):
+            t_ms, n_l = stages[st_name]
+            kernels[f"k_gemm_tc {g}" if prec_name != "fp32" else f"k_gemm_simt {g}"] = {
+                "bound": "tensor", "unit": "TFLOP/s", "peak": tpk, "flops_per_target": fa[g], "targets": n_targets,
+                "launches": n_l, "avg_launch_us": 1e3 * t_ms / max(1, n_l),
+                "achieved": n_targets * fa[g] / (t_ms / 1e3) / 1e12, "share_of_step": t_ms / ms_step}
+        for v in kernels.values():
+            v["frac"] = v["achieved"] / v["peak"]
+        dom = max(kernels, key=lambda n: kernels[n]["share_of_step"])
+        dk = kernels[dom]
+        tr = traffic_record(args.config, prec_name)
         traffic = None
-        tp = os.path.join(ROOT, "profiles", "attn_traffic_bytes_per_launch.json")
-        if os.path.exists(tp):
-            traffic = json.load(open(tp)).get(args.config)
-        roof = {"kernel": "k_attn", "bound": "hbm", "achieved": achieved, "peak": peaks["hbm_gbs"],
-                "unit": "GB/s", "frac": achieved / peaks["hbm_gbs"], "traffic": traffic,
-                "peak_source": peaks["source"], "bytes_per_target": per_target, "targets": n_targets,
-                "launches": attn_n, "avg_launch_us": 1e3 * attn_ms / max(1, attn_n),
-                "stage_share_of_step": attn_ms / max(1e-9, sum(v[0] for v in stages.values()))}
+        if tr and dom in tr:
+            traffic = {k2: tr[dom][k2] for k2 in tr[dom]}
+        roof = {"kernel": dom, "bound": dk["bound"], "achieved": dk["achieved"], "peak": dk["peak"],
+                "unit": dk["unit"], "frac": dk["frac"],
+                "traffic": (traffic or {}).get("dram_bytes_per_launch"),
+                "traffic_record": traffic,
+                "peak_source": peaks["source"] + ("" if dk["bound"] == "hbm" else
+                                                  f" bf16_tflops_sustained x tf32/bf16 nominal ratio"
+                                                  f"{' / 3 passes' if prec_name == 'tf32x3' else ''}"),
+                "launches": dk["launches"], "avg_launch_us": dk["avg_launch_us"],
+                "share_of_step": dk["share_of_step"]}
+        ideal = ideal_time(per, s, mc, peaks, prec_name)
+        ideal["measured_ms"] = ms_step
+        ideal["frac_paper_form"] = ideal["ideal_ms_paper_form"] / ms_step
+        ideal["frac_absorbed_form"] = ideal["ideal_ms_absorbed_form"] / ms_step
+        ideal["note"] = ("per-batch counters of this rank's pass; F from SURVEY 8(d) F_M (paper form) and "
+                         "from the G1-G4 + attention flops this build executes (absorbed form)")
+    out = {"value": value, "ms_per_step": ms_step, "launches": int(launches), "clocks": clk.summary(),
+           "e2e": {"value": e2e_val, "unit": "edges/s", "h2d_bytes_per_step": 12 * E_rank,
+                   "d2h_bytes_per_step": 4 * E_rank},
+           "stats": stats, "superbatch": ctx.superbatch(), "roofline": roof, "roofline_kernels": kernels,
+           "e2e_roofline": ideal,
+           "stages_ms": {k2: round(v[0], 3) for k2, v in stages.items()} if stages else None,
+           "E_rank": E_rank, "E_job": E_job}
+    ctx.close()
+    del flush
+    torch.cuda.empty_cache()
+    return out
+
+
+def _free_port():
+    so = socket.socket()
+    so.bind(("127.0.0.1", 0))
+    p = so.getsockname()[1]
+    so.close()
+    return p
+
+
+# ---------------------------------------------------------------- main
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="reddit")
+    ap.add_argument("--precision", default="tf32x3", choices=["tf32x3", "bf16", "fp32", "tf32"])
+    ap.add_argument("--second-precision", default="bf16",
+                    help="also measure this precision into the same line ('none' to skip)")
+    ap.add_argument("--scaling", default="strong", choices=["strong", "weak"])
+    ap.add_argument("--superbatch", type=int, default=0)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-profile", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        ap.error("--warmup must be >= 3 (timing rules)")
+
+    world = int(os.environ.get("WORLD_SIZE", "0"))
+    if args.gpus > 1 and world == 0:
+        # spawn one rank per GPU on this node (north_star: one process per GPU, NCCL)
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+               "--master-addr=127.0.0.1", f"--master-port={_free_port()}", os.path.abspath(__file__),
+               *sys.argv[1:]]
+        sys.exit(subprocess.call(cmd))
+    world = max(world, 1)
+    if world != args.gpus:
+        raise SystemExit(f"WORLD_SIZE={world} but --gpus {args.gpus}")
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+
+    from synth import get_config
+    cfg = get_config(args.config)
+    mc = cfg.model
+    if args.impl == "reference":
+        if rank == 0:
+            run_reference(args, cfg)
+        return
+
+    import dataclasses
+    import torch
+    import torch.distributed as dist
+    from synth import make_stream, make_params
+    from paper_conf_ppopp_wangm23_b200.shard import shard_batches
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    if args.scaling == "weak" and world > 1:
+        s = make_stream(dataclasses.replace(cfg.stream, seed=cfg.stream.seed + 7919 * rank))
+    else:
+        s = make_stream(args.config)
+    flat = make_params(mc.n_layers, mc.n_heads, s.d_n, s.d_e)
+    B = mc.batch
+    if args.scaling == "strong":
+        shard = shard_batches(s.n_edges, B, rank, world)
+    else:
+        shard = (0, (s.n_edges + B - 1) // B, 0, s.n_edges)
+
+    precs = [args.precision] + ([args.second_precision] if args.second_precision not in ("none", args.precision)
+                                else [])
+    res = {}
+    for p in precs:
+        res[p] = measure(args, p, s, flat, mc, {}, shard, world, rank, local, dist, args.steps, args.warmup,
+                         profile=not args.no_profile)
+    h = res[args.precision]
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(cfg, args.config)
 
     if rank == 0:
-        line = {"metric": "edges_per_sec", "value": value, "unit": "edges/s", "n_gpus": world,
-                "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t_max / args.steps,
+        dtype = {"fp32": "f32", "tf32x3": "tf32x3", "bf16": "bf16", "tf32": "tf32"}
+        line = {"metric": "edges_per_sec", "value": h["value"], "unit": "edges/s", "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": h["ms_per_step"],
                 "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None,
-                "dtype": {"fp32": "f32", "tf32x3": "tf32x3", "bf16": "bf16", "tf32": "tf32"}[args.precision],
-                "data": "synthetic",
+                "dtype": dtype[args.precision],
+                "data": "synthetic (seeded Reddit-shaped stream, synth/; random-init weights seed 1234)",
                 "config": {"workload": args.config, "n_edges": s.n_edges, "n_nodes": s.n_nodes,
-                           "edges_per_rank": E_rank, "batch": B, "n_layers": mc.n_layers, "heads": mc.n_heads,
+                           "edges_per_rank": h["E_rank"], "batch": B, "n_layers": mc.n_layers, "heads": mc.n_heads,
                            "k": mc.n_neighbors, "d_n": s.d_n, "d_e": s.d_e, "cache_limit": mc.cache_limit,
                            "time_window": mc.time_window, "opts": "dedup+cache+ttable",
-                           "superbatch": ctx.superbatch(),
+                           "superbatch": h["superbatch"],
                            "parallelism": (f"independent streams x{world}" if args.scaling == "weak"
-                                           else f"batch-range shards x{world}"),
+                                           else f"contiguous batch-range shards x{world}"),
+                           "precision_note": ("tf32x3: 3-term tf32 tensor-core products with fp32 accumulation, "
+                                              "fp32 activations (fp32-level, parity 1e-5 + 1e-4|ref|)"
+                                              if args.precision == "tf32x3" else args.precision),
                            "l2": "flushed (256 MB write) before every timed step; inputs > L2",
                            "step": "one cold-cache chronological pass over the rank's batches"},
-                "e2e": {"value": e2e_val, "unit": "edges/s", "h2d_bytes_per_step": 12 * E_rank,
-                        "d2h_bytes_per_step": 4 * E_rank},
-                "gpu_launches": int(launches),
-                "roofline": roof, "cpu_baseline": cpu, "clocks": clk.summary(), "stats": stats,
-                "stages_ms": {k2: round(v[0], 3) for k2, v in stages.items()} if stages else None,
-                "peaks": {k2: peaks[k2] for k2 in ("hbm_gbs", "bf16_tflops", "source") if k2 in peaks}}
+                "e2e": h["e2e"], "gpu_launches": h["launches"],
+                "roofline": h["roofline"], "roofline_kernels": h["roofline_kernels"],
+                "e2e_roofline": h["e2e_roofline"],
+                "cpu_baseline": cpu, "clocks": h["clocks"], "stats": h["stats"], "stages_ms": h["stages_ms"],
+                "paper_context": PAPER_CONTEXT}
+        for p in precs[1:]:
+            r = res[p]
+            line[p] = {"value": r["value"], "ms_per_step": r["ms_per_step"], "dtype": dtype[p], "e2e": r["e2e"],
+                       "gpu_launches": r["launches"], "clocks": r["clocks"], "roofline": r["roofline"],
+                       "e2e_roofline": r["e2e_roofline"], "stages_ms": r["stages_ms"],
+                       "superbatch": r["superbatch"]}
+        peaks = load_peaks()
+        line["peaks"] = {k2: peaks[k2] for k2 in ("hbm_gbs", "bf16_tflops", "bf16_tflops_sustained", "source")
+                         if k2 in peaks}
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()

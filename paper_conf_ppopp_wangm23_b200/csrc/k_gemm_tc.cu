@@ -95,7 +95,14 @@ tg_status tc_prepare_weights(const float* W, int N, int K, int precision, TcWeig
   // N tiles of <= 256 columns: each A tile is re-read once per N tile, and the
   // kernel is bound by L2 -> SM operand traffic at these sizes
   // (narrow GEMMs, N <= 256, keep two N tiles for parallelism instead)
-  const int ntn = (N > 256 && tc_acc_cols(precision) == 256) ? (N + 255) / 256 : (N + 127) / 128;
+  int ntn = (N > 256 && tc_acc_cols(precision) == 256) ? (N + 255) / 256 : (N + 127) / 128;
+  // tf32x3 keeps a [big | small] accumulator pair per buffer: N tiles <= 128 keep the
+  // epilogue double-buffered (4 x 128 TMEM columns); wider tiles run single-buffered
+  static const int x3_bn = [] {
+    const char* e = getenv("TG_X3_BN");
+    return e ? atoi(e) : 256;
+  }();
+  if (precision == TG_PREC_TF32X3 && x3_bn > 0 && x3_bn < 256) ntn = (N + x3_bn - 1) / x3_bn;
   int BN = (N + ntn - 1) / ntn;
   BN = (BN + 15) & ~15;
   const int epc = tc_epc(precision);
@@ -319,6 +326,16 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   // the compiler keeps the shared address space (LDS/STS, not generic LD/ST)
   unsigned char* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   const int BN = w.BN;
+  // TMEM accumulators (512 columns allocated). tf32x3: each buffer holds [big | small]
+  // (BNc = round32(BN) columns each): ah.bh accumulates into `big`, the correction terms
+  // ah.bl + al.bh into `small`, summed in fp32 by the epilogue -- the tensor core's fp32
+  // accumulation truncates at every MMA (error ~ steps x ulp(|acc|)), so keeping the
+  // 2K/8 correction MMAs out of the large accumulator cuts that error 3x. Double-buffered
+  // when 4 BNc <= 512, else one buffer. Other modes: two 256-column buffers.
+  const int BNc = (BN + 31) & ~31;
+  const uint32_t buf_cols = PLANES == 2 ? 2u * BNc : (uint32_t)tc_acc_cols(PREC);
+  const uint32_t small_off = PLANES == 2 ? (uint32_t)BNc : 0u;
+  const uint32_t nbuf = (PLANES == 2 && 4 * BNc > 512) ? 1u : 2u;
   const uint32_t a_plane = TC_BM * 128;
   const uint32_t b_plane = (uint32_t)BN * 128;
   const uint32_t stage_bytes = PLANES * (a_plane + b_plane);
@@ -534,10 +551,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       const uint32_t idesc = umma_idesc(PREC, BN);
       uint32_t gk = 0, tc = 0;
       for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++tc) {
-        const uint32_t acc = tc & 1;
-        mbar_wait(&tempty[acc], ((tc >> 1) & 1) ^ 1);  // epilogue drained this accumulator
+        const uint32_t acc = tc % nbuf;
+        mbar_wait(&tempty[acc], ((tc / nbuf) & 1) ^ 1);  // epilogue drained this accumulator
         asm volatile("tcgen05.fence::after_thread_sync;\n");
-        const uint32_t dtm = tmem + acc * tc_acc_cols(PREC);
+        const uint32_t dtm = tmem + acc * buf_cols;
         for (int kb = 0; kb < nkb; ++kb, ++gk) {
           const int s = gk % stages;
           mbar_wait(&full[s], (gk / stages) & 1);
@@ -551,8 +568,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
             const uint32_t acc0 = (kb > 0 || kk > 0) ? 1u : 0u;
             mma_issue<PREC>(dtm, umma_desc(aH + kk * 32), umma_desc(bH + kk * 32), idesc, acc0);
             if (PLANES == 2) {
-              mma_issue<PREC>(dtm, umma_desc(aH + kk * 32), umma_desc(bH + b_plane + kk * 32), idesc, 1u);
-              mma_issue<PREC>(dtm, umma_desc(aH + a_plane + kk * 32), umma_desc(bH + kk * 32), idesc, 1u);
+              mma_issue<PREC>(dtm + small_off, umma_desc(aH + kk * 32), umma_desc(bH + b_plane + kk * 32), idesc,
+                              acc0);
+              mma_issue<PREC>(dtm + small_off, umma_desc(aH + a_plane + kk * 32), umma_desc(bH + kk * 32), idesc,
+                              1u);
             }
           }
           asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n" ::"r"(
@@ -603,12 +622,12 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++tc) {
       const int tm = t / ntn, tn = t - tm * ntn;
       const int m0 = tm * TC_BM, n0 = tn * BN;
-      const uint32_t acc = tc & 1, par = tc & 1;
+      const uint32_t acc = tc % nbuf, par = tc & 1;
       const int er = m0 + rloc;
       unsigned short* hrow = er < M ? g.c_h + (size_t)er * g.ldc_h : nullptr;
-      mbar_wait(&tfull[acc], (tc >> 1) & 1);
+      mbar_wait(&tfull[acc], (tc / nbuf) & 1);
       asm volatile("tcgen05.fence::after_thread_sync;\n");
-      const uint32_t tacc = tmem + acc * tc_acc_cols(PREC) + ((uint32_t)(quad * 32) << 16);
+      const uint32_t tacc = tmem + acc * buf_cols + ((uint32_t)(quad * 32) << 16);
       // ---- pass 1: row statistics of this thread's column chunks
       float sn = 0.f, sm = 0.f, sM = 0.f;
       for (int c0 = 16 * half; c0 < BN; c0 += 32) {
@@ -712,7 +731,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++tc) {
       const int tm = t / w.ntn, tn = t - tm * w.ntn;
       const int m0 = tm * TC_BM, n0 = tn * BN;
-      const uint32_t acc = tc & 1;
+      const uint32_t acc = tc % nbuf;
       const int er = m0 + quad * 32 + lane;
       float* orow = nullptr;
       unsigned short* hrow = nullptr;
@@ -721,14 +740,23 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         else if (g.C) orow = g.C + (size_t)er * g.ldc;
         if (g.c_h) hrow = g.c_h + (size_t)er * g.ldc_h;
       }
-      mbar_wait(&tfull[acc], (tc >> 1) & 1);
+      mbar_wait(&tfull[acc], (tc / nbuf) & 1);
       if (tc == 0 && warp == 6 && lane == 0) TCT(5, clock64());
       asm volatile("tcgen05.fence::after_thread_sync;\n");
       bool released = false;
       for (int c0 = 16 * half; c0 < BN; c0 += 32) {
         uint32_t v[16];
-        tmem_ld16(tmem + acc * tc_acc_cols(PREC) + ((uint32_t)(quad * 32) << 16) + (uint32_t)c0, v);
-        asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
+        const uint32_t tq = tmem + acc * buf_cols + ((uint32_t)(quad * 32) << 16) + (uint32_t)c0;
+        tmem_ld16(tq, v);
+        if (PLANES == 2) {  // + the correction accumulator (fp32 RN add)
+          uint32_t vs[16];
+          tmem_ld16(tq + small_off, vs);
+          asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
+#pragma unroll
+          for (int j = 0; j < 16; ++j) v[j] = __float_as_uint(__uint_as_float(v[j]) + __uint_as_float(vs[j]));
+        } else {
+          asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
+        }
         if (c0 + 32 >= BN) {  // this warp's last chunk: hand the accumulator back
           asm volatile("tcgen05.fence::before_thread_sync;\n");
           mbar_arrive(&tempty[acc]);

@@ -25,6 +25,7 @@ class StreamConfig:
     zipf_item: float = 1.2
     session_mean: float = 6.0
     gap_scale: float = 30.0  # Pareto scale (s) of intra-session gaps -> power-law dt near 0 (Fig. 4)
+    min_gap: int = 0         # minimum intra-session gap (s): a node's consecutive events differ in t
 
 
 @dataclass(frozen=True)

@@ -62,7 +62,7 @@ def _session_times(cfg: StreamConfig, rng, n_events):
     sess = np.repeat(np.arange(lens.size), lens)
     starts = rng.integers(0, cfg.max_t + 1, size=lens.size).astype(np.float64)
     # Pareto(alpha=1.2) gaps, scale gap_scale seconds, floored to integer seconds
-    gaps = np.floor(cfg.gap_scale * (rng.pareto(1.2, size=total)))
+    gaps = np.floor(cfg.gap_scale * (rng.pareto(1.2, size=total))) + cfg.min_gap
     first = np.r_[0, np.cumsum(lens)[:-1]]
     gaps[first] = 0.0
     # cumulative gap inside each session

@@ -13,7 +13,12 @@ from synth import make_stream
 from tests.gpu_helpers import close, setup, make_ctx, make_oracle
 
 pytestmark = pytest.mark.gpu
+# (rtol, atol) for embeddings: fp32-level modes at north_star's 1e-4 / 1e-5 (R17); bf16 / 1-pass tf32
+# GEMM operands at rtol 2e-2 with atol 2e-2 (R22: bf16 rounding of K ~ 10^2..10^3 products leaves
+# absolute errors up to ~1.5e-2 on O(1) embedding elements near zero, tools/parity_errors.py)
 TOL = {0: (1e-4, 1e-5), 1: (1e-4, 1e-5), 2: (2e-2, 2e-2), 3: (2e-2, 2e-2)}  # fp32/tf32x3/bf16/tf32
+# scores (sigmoid outputs): rtol only in every mode, with the fp32 atol 1e-5 as the floor (R22)
+SCORE_TOL = {0: (1e-4, 1e-5), 1: (1e-4, 1e-5), 2: (2e-2, 1e-5), 3: (2e-2, 1e-5)}
 
 
 @pytest.fixture(scope="module", autouse=True)
@@ -196,7 +201,7 @@ def test_score_pairs_negatives(name, prec):
             got = out.cpu().numpy()
         h = o.embed(mc.n_layers, nodes, tt.astype(np.int64))
         ref = o.score(h[pa], h[pb])
-        ok, err, nbad = close(got, ref, *TOL[prec])
+        ok, err, nbad = close(got, ref, *SCORE_TOL[prec])
         assert ok, (rep, err, nbad)
     with pytest.raises(Exception):                      # host pair index out of range
         ctx.score_pairs(nodes, tt.view(np.int32), pa, np.full_like(pb, 3 * B), np.zeros(2 * B, np.float32))
@@ -268,7 +273,7 @@ def test_stream_scores_parity(name, prec):
     for b in picks:
         lo, hi = b * mc.batch, min((b + 1) * mc.batch, s.n_edges)
         _, ref = o.infer_batch(s.src[lo:hi], s.dst[lo:hi], s.ts[lo:hi])
-        ok, err, nbad = close(scores[lo:hi], ref, *TOL[prec])
+        ok, err, nbad = close(scores[lo:hi], ref, *SCORE_TOL[prec])
         assert ok, (b, err, nbad)
 
 
@@ -345,7 +350,7 @@ def test_eviction_stress_repeated():
 
 
 # ------------------------------------------------------------- GEMM kernels
-@pytest.mark.parametrize("prec,rtol,atol", [(0, 1e-5, 1e-5), (1, 1e-5, 1e-4), (2, 2e-2, 2e-2),
+@pytest.mark.parametrize("prec,rtol,atol", [(0, 1e-5, 1e-5), (1, 1e-5, 1e-5), (2, 2e-2, 2e-2),
                                              (3, 5e-3, 5e-3)])
 @pytest.mark.parametrize("M,N,K", [(1, 16, 8), (130, 176, 172), (6400, 1032, 172), (700, 516, 1032),
                                    (257, 172, 688)])

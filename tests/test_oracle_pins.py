@@ -319,3 +319,98 @@ def test_fifo_cache_semantics():
     assert [c.live(k) for k in (1, 2, 3, 4)] == [False, True, True, True]
     assert c.store([5, 6, 7, 8], None) == 3    # n > limit: the newest `limit` survive (R11)
     assert [c.live(k) for k in (4, 5, 6, 7, 8)] == [False, False, True, True, True]
+
+
+# ------------------------------------------------ TimeEncode window counters (Sec. 4.3)
+def _brute_deltas(bt, l, i, t, out):
+    """Every dt = t - t_j that computing h(l, i, t) encodes, by literal recursion over the
+    edge-scan sampler of tests/_bruteforce.py (no dedup, no memo: the baseline of P:L140)."""
+    if l == 0:
+        return
+    _brute_deltas(bt, l - 1, i, t, out)
+    for (j, e, tj) in bt.neighbours(i, t):
+        out.append(t - tj)                  # padding slot: t_j = 0, dt = t (R7)
+        _brute_deltas(bt, l - 1, j, tj, out)
+
+
+def _window_setup():
+    cfg, s, flat, m, g, t = _setup("tiny_bip")
+    mc = cfg.model
+    bt = BruteTGAT(flat, mc.n_layers, mc.n_heads, s.d_n, s.d_e, s.src, s.dst, s.ts,
+                   s.node_feat, s.edge_feat, mc.n_neighbors)
+    return cfg, s, t, bt
+
+
+def test_time_table_counter_baseline_matches_bruteforce_window():
+    """Phi(dt) comes from the precomputed window iff 0 <= dt < W. With dedup and cache
+    off every target of the (k+1)^L expansion is computed, so the per-batch table/direct counts
+    are the brute-force count of dt < W over the expansion. W is set to a dt that occurs, so an
+    off-by-one (dt <= W) changes the count."""
+    cfg, s, t, bt = _window_setup()
+    mc = cfg.model
+    nb = 4
+    deltas = []
+    per_batch = []
+    for b in range(nb):
+        lo, hi = b * mc.batch, min((b + 1) * mc.batch, s.n_edges)
+        d = []
+        for (i, tt) in list(zip(s.src[lo:hi], s.ts[lo:hi])) + list(zip(s.dst[lo:hi], s.ts[lo:hi])):
+            _brute_deltas(bt, mc.n_layers, int(i), int(tt), d)
+        per_batch.append(d)
+        deltas += d
+    pos = sorted(x for x in deltas if x > 0)
+    W = pos[len(pos) // 2]
+    assert sum(1 for x in deltas if x == W) > 0
+    for win in (W, W + 1):
+        sim = TGOptSim(t, time_window=win, dedup=False, cache=False, ttable=True, compute=False)
+        for b in range(nb):
+            lo, hi = b * mc.batch, min((b + 1) * mc.batch, s.n_edges)
+            sim.reset_counters()
+            sim.infer_batch(s.src[lo:hi], s.dst[lo:hi], s.ts[lo:hi])
+            c = sim.counters()
+            want_tab = sum(1 for x in per_batch[b] if 0 <= x < win)
+            assert c["t_table"] == want_tab, (win, b)
+            assert c["t_direct"] == len(per_batch[b]) - want_tab
+    # table off: everything direct
+    sim = TGOptSim(t, time_window=W, dedup=False, cache=False, ttable=False, compute=False)
+    sim.infer_batch(s.src[:mc.batch], s.dst[:mc.batch], s.ts[:mc.batch])
+    assert sim.counters()["t_table"] == 0 and sim.counters()["t_direct"] == len(per_batch[0])
+
+
+def test_time_table_counter_with_memo_matches_key_universe():
+    """With dedup and an unbounded cache (L = 2), a layer-2 target is computed once per batch
+    per distinct (i, t) and a layer-1 key once per stream (the key-universe argument), so
+    the stream's table count is the brute-force dt < W count over exactly those targets."""
+    cfg, s, t, bt = _window_setup()
+    mc = cfg.model
+    assert mc.n_layers == 2
+    W = mc.time_window
+    k = mc.n_neighbors
+    sim = TGOptSim(t, cache_limit=10**9, time_window=W, compute=False)
+    seen1 = set()
+    want_tab = want_all = 0
+
+    def count(i, tt):
+        nonlocal want_tab, want_all
+        for (j, e, tj) in bt.neighbours(i, tt):
+            want_all += 1
+            want_tab += 1 if 0 <= tt - tj < W else 0
+
+    for lo in range(0, s.n_edges, mc.batch):
+        hi = min(lo + mc.batch, s.n_edges)
+        sim.infer_batch(s.src[lo:hi], s.dst[lo:hi], s.ts[lo:hi])
+        top = []
+        for (i, tt) in list(zip(s.src[lo:hi], s.ts[lo:hi])) + list(zip(s.dst[lo:hi], s.ts[lo:hi])):
+            if (int(i), int(tt)) not in top:
+                top.append((int(i), int(tt)))
+        for (i, tt) in top:                      # layer 2: every distinct target of the batch
+            count(i, tt)
+        for (i, tt) in top:                      # layer 1: keys never computed before
+            for key in [(i, tt)] + [(j, tj) for (j, e, tj) in bt.neighbours(i, tt)]:
+                if key not in seen1:
+                    seen1.add(key)
+                    count(*key)
+    c = sim.counters()
+    assert c["l1_misses"] == len(seen1)
+    assert c["t_table"] == want_tab and c["t_direct"] == want_all - want_tab
+    assert 0 < want_tab < want_all
