@@ -64,6 +64,8 @@ def tensor_peak(peaks, prec, sustained=True):
     bf = peaks.get("bf16_tflops_sustained" if sustained else "bf16_tflops", peaks["bf16_tflops"])
     if prec == "bf16":
         return bf
+    if prec == "f16x3":          # fp16 runs at the bf16 rate; 3 MMAs per fp32-level product
+        return bf / 3.0
     tf32 = bf * NOMINAL_TF["tf32"] / NOMINAL_TF["bf16"]
     return tf32 / 3.0 if prec == "tf32x3" else tf32
 
@@ -281,9 +283,10 @@ def measure(args, prec_name, s, flat, mc, ctx_kw, shard, world, rank, local, dis
             profile=True):
     import torch
     from paper_conf_ppopp_wangm23_b200 import (Context, TG_NCOUNTERS, counters_dict, TG_PREC_FP32,
-                                              TG_PREC_TF32X3, TG_PREC_BF16, TG_PREC_TF32)
+                                              TG_PREC_TF32X3, TG_PREC_BF16, TG_PREC_TF32, TG_PREC_F16X3)
     from paper_conf_ppopp_wangm23_b200.shard import gather_scores, reduce_counters
-    prec = {"fp32": TG_PREC_FP32, "tf32x3": TG_PREC_TF32X3, "bf16": TG_PREC_BF16, "tf32": TG_PREC_TF32}[prec_name]
+    prec = {"fp32": TG_PREC_FP32, "tf32x3": TG_PREC_TF32X3, "bf16": TG_PREC_BF16, "tf32": TG_PREC_TF32,
+            "f16x3": TG_PREC_F16X3}[prec_name]
     b0, b1, e0, e1 = shard
     B = mc.batch
     E_rank = e1 - e0
@@ -454,8 +457,9 @@ def measure(args, prec_name, s, flat, mc, ctx_kw, shard, world, rank, local, dis
                 "traffic": (traffic or {}).get("dram_bytes_per_launch"),
                 "traffic_record": traffic,
                 "peak_source": peaks["source"] + ("" if dk["bound"] == "hbm" else
-                                                  f" bf16_tflops_sustained x tf32/bf16 nominal ratio"
-                                                  f"{' / 3 passes' if prec_name == 'tf32x3' else ''}"),
+                                                  (" bf16_tflops_sustained / 3 passes" if prec_name == "f16x3"
+                                                   else " bf16_tflops_sustained x tf32/bf16 nominal ratio"
+                                                   f"{' / 3 passes' if prec_name == 'tf32x3' else ''}")),
                 "launches": dk["launches"], "avg_launch_us": dk["avg_launch_us"],
                 "share_of_step": dk["share_of_step"]}
         ideal = ideal_time(per, s, mc, peaks, prec_name)
@@ -492,7 +496,7 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="reddit")
-    ap.add_argument("--precision", default="tf32x3", choices=["tf32x3", "bf16", "fp32", "tf32"])
+    ap.add_argument("--precision", default="tf32x3", choices=["tf32x3", "f16x3", "bf16", "fp32", "tf32"])
     ap.add_argument("--second-precision", default="bf16",
                     help="also measure this precision into the same line ('none' to skip)")
     ap.add_argument("--scaling", default="strong", choices=["strong", "weak"])
@@ -558,7 +562,7 @@ def main():
         cpu = cpu_baseline(cfg, args.config)
 
     if rank == 0:
-        dtype = {"fp32": "f32", "tf32x3": "tf32x3", "bf16": "bf16", "tf32": "tf32"}
+        dtype = {"fp32": "f32", "tf32x3": "tf32x3", "bf16": "bf16", "tf32": "tf32", "f16x3": "f16x3"}
         line = {"metric": "edges_per_sec", "value": h["value"], "unit": "edges/s", "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": h["ms_per_step"],
                 "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None,

@@ -60,7 +60,12 @@ typedef struct tg_ctx tg_ctx; /* opaque; one per device */
 #define TG_PREC_TF32X3 1  /* tcgen05 kind::tf32, 3-term hi/lo split: fp32-level error */
 #define TG_PREC_BF16  2   /* tcgen05 kind::f16 bf16 operands, fp32 accumulate: rtol 2e-2 */
 #define TG_PREC_TF32  3   /* tcgen05 kind::tf32 one pass (A streamed raw fp32, B rna-tf32): rtol 2e-2 class */
-#define TG_PREC_LAST  TG_PREC_TF32
+#define TG_PREC_F16X3 4   /* tcgen05 kind::f16, fp16 operands with the 3-term hi/lo split (11 + 11 bits, as
+                           * TF32X3) at twice the tf32 rate: fp32-level error (parity 1e-5 + 1e-4|ref|).
+                           * Weights are scaled per row by exact powers of two; activations entering a
+                           * projection must satisfy |a| < 65504, else the sticky device error bit 32 is set
+                           * (tg_counters_read returns TG_EDEVICE) -- use TG_PREC_TF32X3 for such data. */
+#define TG_PREC_LAST  TG_PREC_F16X3
 
 /* ------------------------------------------------------------------------ */
 /* Graph: a CTDG edge stream with static node/edge features.        */

@@ -19,7 +19,14 @@
 // TG_PREC_TF32X3: kind::tf32 with the 3-term split a.b ~ ah.bh + ah.bl + al.bh
 // (ah = rna_tf32(a), al = rna_tf32(a - ah)): fp32-level accuracy on tensor
 // cores. TG_PREC_BF16: kind::f16 with bf16 operands, fp32 accumulation.
+// TG_PREC_F16X3: kind::f16 with fp16 operands and the same 3-term split
+// (ah = rn_f16(a), al = rn_f16(a - ah); 11 + 11 significant bits like tf32 hi/lo)
+// at twice the tf32 MMA rate and half the shared-memory bytes per product. fp16's
+// exponent range is handled by an exact power-of-two scale per weight row (host,
+// undone per output column in the epilogue); activations must satisfy |a| < 65504
+// (checked by the producers: sticky device error kErrF16Range otherwise).
 #include <cuda_bf16.h>
+#include <cuda_fp16.h>
 
 #include <cstdio>
 #include <cstdlib>
@@ -40,8 +47,10 @@ constexpr int TC_MAXSTAGES = 8;
 __host__ __device__ constexpr int tc_acc_cols(int) { return 256; }
 __host__ __device__ constexpr int tc_ctas_per_sm(int) { return 1; }
 
-__host__ __device__ inline int tc_epc(int prec) { return prec == TG_PREC_BF16 ? 64 : 32; }  // elems / 128B
-__host__ __device__ inline int tc_planes(int prec) { return prec == TG_PREC_TF32X3 ? 2 : 1; }
+__host__ __device__ inline int tc_epc(int prec) {  // elements per 128 B
+  return (prec == TG_PREC_BF16 || prec == TG_PREC_F16X3) ? 64 : 32;
+}
+__host__ __device__ inline int tc_planes(int prec) { return (prec == TG_PREC_TF32X3 || prec == TG_PREC_F16X3) ? 2 : 1; }
 
 // offset of 16-byte chunk c of row r inside a 128B-swizzled K-major tile
 __host__ __device__ inline unsigned sw128(int r, int c) {
@@ -102,7 +111,8 @@ tg_status tc_prepare_weights(const float* W, int N, int K, int precision, TcWeig
     const char* e = getenv("TG_X3_BN");
     return e ? atoi(e) : 256;
   }();
-  if (precision == TG_PREC_TF32X3 && x3_bn > 0 && x3_bn < 256) ntn = (N + x3_bn - 1) / x3_bn;
+  if ((precision == TG_PREC_TF32X3 || precision == TG_PREC_F16X3) && x3_bn > 0 && x3_bn < 256)
+    ntn = (N + x3_bn - 1) / x3_bn;
   int BN = (N + ntn - 1) / ntn;
   BN = (BN + 15) & ~15;
   const int epc = tc_epc(precision);
@@ -113,6 +123,24 @@ tg_status tc_prepare_weights(const float* W, int N, int K, int precision, TcWeig
   std::vector<float> w((size_t)N * K);
   if (cudaMemcpy(w.data(), W, w.size() * 4, cudaMemcpyDeviceToHost) != cudaSuccess) return TG_ECUDA;
   std::vector<unsigned char> img(total, 0);
+  // F16X3: exact power-of-two scale per weight row n so that max_k |W[n,k]| 2^e lies in
+  // [2^14, 2^15) -- the hi and lo fp16 parts then stay normal for every element within
+  // 2^-14 of the row maximum; the epilogue multiplies output column n by 2^-e
+  std::vector<float> colscale;
+  if (precision == TG_PREC_F16X3) {
+    colscale.assign((size_t)ntn * BN, 1.f);
+    for (int n = 0; n < N; ++n) {
+      float mx = 0.f;
+      for (int k = 0; k < K; ++k) mx = std::max(mx, std::fabs(w[(size_t)n * K + k]));
+      if (mx > 0.f && std::isfinite(mx)) {
+        int e = 0;
+        std::frexp(mx, &e);  // mx = f 2^e, f in [0.5, 1): mx 2^(15 - e) in [2^14, 2^15)
+        const int s = 15 - e;
+        for (int k = 0; k < K; ++k) w[(size_t)n * K + k] = std::ldexp(w[(size_t)n * K + k], s);
+        colscale[n] = std::ldexp(1.f, -s);
+      }
+    }
+  }
   for (int tn = 0; tn < ntn; ++tn)
     for (int kb = 0; kb < nkb; ++kb) {
       unsigned char* base = img.data() + ((size_t)tn * nkb + kb) * planes * plane_bytes;
@@ -120,7 +148,19 @@ tg_status tc_prepare_weights(const float* W, int N, int K, int precision, TcWeig
         const int n = tn * BN + r;
         for (int c = 0; c < 8; ++c) {
           unsigned char* dst0 = base + sw128(r, c);
-          if (precision == TG_PREC_BF16) {
+          if (precision == TG_PREC_F16X3) {
+            uint16_t vh[8], vl[8];
+            for (int e = 0; e < 8; ++e) {
+              const int kk = kb * epc + c * 8 + e;
+              const float x = (n < N && kk < K) ? w[(size_t)n * K + kk] : 0.f;
+              const __half h = __float2half_rn(x);
+              const __half l = __float2half_rn(x - __half2float(h));
+              memcpy(&vh[e], &h, 2);
+              memcpy(&vl[e], &l, 2);
+            }
+            memcpy(dst0, vh, 16);
+            memcpy(dst0 + plane_bytes, vl, 16);
+          } else if (precision == TG_PREC_BF16) {
             uint16_t v[8];
             for (int e = 0; e < 8; ++e) {
               const int kk = kb * epc + c * 8 + e;
@@ -147,6 +187,14 @@ tg_status tc_prepare_weights(const float* W, int N, int K, int precision, TcWeig
   if (cudaMemcpy(d, img.data(), total, cudaMemcpyHostToDevice) != cudaSuccess) return TG_ECUDA;
   out->hi = d;
   out->lo = nullptr;
+  out->colscale = nullptr;
+  if (!colscale.empty()) {
+    void* cs = nullptr;
+    if (cudaMalloc(&cs, colscale.size() * 4) != cudaSuccess) return TG_ENOMEM;
+    owned.push_back(cs);
+    if (cudaMemcpy(cs, colscale.data(), colscale.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) return TG_ECUDA;
+    out->colscale = reinterpret_cast<float*>(cs);
+  }
   out->N = N;
   out->K = K;
   out->Np = ntn * BN;
@@ -175,7 +223,7 @@ __device__ __forceinline__ uint64_t umma_desc(uint32_t saddr) {
 __device__ __forceinline__ uint32_t umma_idesc(int prec, int N) {
   uint32_t d = 0;
   d |= 1u << 4;                                         // D = f32
-  const uint32_t fmt = prec == TG_PREC_BF16 ? 1u : 2u;  // bf16 : tf32
+  const uint32_t fmt = prec == TG_PREC_BF16 ? 1u : prec == TG_PREC_F16X3 ? 0u : 2u;  // bf16 : f16 : tf32
   d |= fmt << 7;                                        // A format
   d |= fmt << 10;                                       // B format
   d |= (uint32_t)(N >> 3) << 17;                        // N / 8
@@ -185,7 +233,7 @@ __device__ __forceinline__ uint32_t umma_idesc(int prec, int N) {
 
 template <int PREC>
 __device__ __forceinline__ void mma_issue(uint32_t tmem, uint64_t da, uint64_t db, uint32_t idesc, uint32_t acc) {
-  if (PREC == TG_PREC_BF16) {
+  if (PREC == TG_PREC_BF16 || PREC == TG_PREC_F16X3) {
     asm volatile(
         "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
         "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}\n" ::"r"(tmem),
@@ -318,8 +366,8 @@ template <int PREC>
 __global__ void __launch_bounds__(TC_THREADS, 1)
     k_gemm_tc(GemmArgs g, TcWeights w, int stages, const __grid_constant__ CUtensorMap tmA, int a_tma,
               const __grid_constant__ CUtensorMap tmA2, int a2_kb0, int a2_x0) {
-  constexpr int EPC = PREC == TG_PREC_BF16 ? 64 : 32;
-  constexpr int PLANES = PREC == TG_PREC_TF32X3 ? 2 : 1;
+  constexpr int EPC = (PREC == TG_PREC_BF16 || PREC == TG_PREC_F16X3) ? 64 : 32;
+  constexpr int PLANES = (PREC == TG_PREC_TF32X3 || PREC == TG_PREC_F16X3) ? 2 : 1;
   constexpr int NV = EPC / 4;  // float4 loads per row per k-block
   extern __shared__ __align__(1024) unsigned char smem_raw[];
   // 1024-byte alignment (128B swizzle atoms) by an integer offset from smem_raw, so
@@ -477,7 +525,27 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         const int s = gk % stages;
         mbar_wait(&empty[s], ((gk / stages) & 1) ^ 1);
         unsigned char* sA = smem + s * stage_bytes;
-        if (PREC == TG_PREC_BF16) {
+        if (PREC == TG_PREC_F16X3) {
+          bool big = false;
+#pragma unroll
+          for (int c = 0; c < 8; ++c) {
+            const float4 x0 = regs[2 * c], x1 = regs[2 * c + 1];
+            const float xs[8] = {x0.x, x0.y, x0.z, x0.w, x1.x, x1.y, x1.z, x1.w};
+            uint32_t hv[4], lv[4];
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+              const __half2 h = __floats2half2_rn(xs[2 * e], xs[2 * e + 1]);
+              const float2 hf = __half22float2(h);
+              const __half2 l = __floats2half2_rn(xs[2 * e] - hf.x, xs[2 * e + 1] - hf.y);
+              big |= !(fabsf(xs[2 * e]) < 65504.f) | !(fabsf(xs[2 * e + 1]) < 65504.f);
+              hv[e] = *reinterpret_cast<const uint32_t*>(&h);
+              lv[e] = *reinterpret_cast<const uint32_t*>(&l);
+            }
+            *reinterpret_cast<uint4*>(sA + sw128(tid, c)) = make_uint4(hv[0], hv[1], hv[2], hv[3]);
+            *reinterpret_cast<uint4*>(sA + a_plane + sw128(tid, c)) = make_uint4(lv[0], lv[1], lv[2], lv[3]);
+          }
+          if (big && g.err) atomicOr(g.err, kErrF16Range);
+        } else if (PREC == TG_PREC_BF16) {
 #pragma unroll
           for (int c = 0; c < 8; ++c) {
             const float4 x0 = regs[2 * c], x1 = regs[2 * c + 1];
@@ -774,10 +842,18 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         const bool cpad = cl < BN && c >= g.N && c < g.ldc_h;  // bf16 zero padding [N, ldc_h)
         float4 b4 = make_float4(0.f, 0.f, 0.f, 0.f);
         if (cin && g.bias) b4 = *reinterpret_cast<const float4*>(g.bias + c);
+        float4 s4 = make_float4(1.f, 1.f, 1.f, 1.f);  // F16X3: undo the weight-row scale (exact)
+        if (PREC == TG_PREC_F16X3 && cl < BN) s4 = *reinterpret_cast<const float4*>(w.colscale + n0 + cl);
 #pragma unroll
         for (int i = 0; i < 4; ++i) {
           const int r = rq + 8 * i;
           float4 x = *reinterpret_cast<const float4*>(stg + r * TC_STG_LD + 4 * cq);
+          if (PREC == TG_PREC_F16X3) {
+            x.x *= s4.x;
+            x.y *= s4.y;
+            x.z *= s4.z;
+            x.w *= s4.w;
+          }
           x.x += b4.x;
           x.y += b4.y;
           x.z += b4.z;
@@ -925,6 +1001,14 @@ void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaSt
     }
     launch_k(k_gemm_tc<TG_PREC_TF32>, dim3(grid), dim3(TC_THREADS), smem, st, g, w, stages, tm, a_tma, tm2,
              a2_kb0, a2_x0);
+  } else if (precision == TG_PREC_F16X3) {
+    static size_t set = 0;
+    if (smem > set) {
+      cudaFuncSetAttribute(k_gemm_tc<TG_PREC_F16X3>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      set = smem;
+    }
+    launch_k(k_gemm_tc<TG_PREC_F16X3>, dim3(grid), dim3(TC_THREADS), smem, st, g, w, stages, tm, 0, tm2,
+             1 << 30, 0);
   } else {
     static size_t set = 0;
     if (smem > set) {

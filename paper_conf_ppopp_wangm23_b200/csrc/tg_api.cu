@@ -223,6 +223,7 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   const int* m_dev = lv.n_c_total;
   // G1: u = P h^(l-1) + bu  (target-side K projection with W_q and 1/sqrt(d_k) folded)
   GemmArgs g1{};
+  g1.err = ctx->err;
   g1.a_rows0 = lv.hs_row;
   g1.K0 = g1.K = ctx->dnp;
   g1.B = w.P;
@@ -343,6 +344,7 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   TRY(launched(ctx));
   // G2: y = F c + b_fc  (W_v and W_fc folded; the residual q of Eq. 4 is added by the LayerNorm)
   GemmArgs g2{};
+  g2.err = ctx->err;
   g2.a_base0 = ctx->c;
   g2.lda0 = HDp;
   g2.K0 = g2.K = HDp;
@@ -389,6 +391,7 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   }
   // G3: z = ReLU(W1 [r || h^(l-1)] + b1)  (Eq. 7)
   GemmArgs g3{};
+  g3.err = ctx->err;
   g3.a_base0 = ctx->r;
   g3.lda0 = ctx->Dp;
   g3.K0 = ctx->Dp;
@@ -417,6 +420,7 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   TRY(launched(ctx));
   // G4: h = W2 z + b2 -> ring slot (CacheStore payload, Alg. 3 l.8-10) or H_L
   GemmArgs g4{};
+  g4.err = ctx->err;
   g4.a_base0 = ctx->z;
   g4.lda0 = ctx->dnp;
   g4.K0 = g4.K = ctx->dnp;
@@ -605,6 +609,7 @@ tg_status stream_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, cons
       launch_score_rows(ctx->HL, ctx->dnp, ctx->lv[ctx->L], S, es, ctx->sc_rs, ctx->sc_rd, ctx->sc_oidx, ctx->sc_m,
                         st);
       GemmArgs g{};  // hidden layer of the affinity MLP: ReLU(W_a1 [h_src || h_dst] + b_a1)
+      g.err = ctx->err;
       g.a_rows0 = ctx->sc_rs;
       g.K0 = ctx->dnp;
       g.a_rows1 = ctx->sc_rd;
@@ -1259,6 +1264,7 @@ tg_status tg_score_pairs(tg_ctx* ctx, const int32_t* nodes, const uint32_t* ts, 
     launch_pair_rows(ctx->HL, ctx->dnp, ctx->lv[ctx->L], (int)n_targets, da, db, (int)n_pairs, ctx->sc_rs,
                      ctx->sc_rd, ctx->sc_oidx, ctx->sc_m, ctx->err, st);
     GemmArgs g{};  // hidden layer of the affinity MLP over the pairs (R10)
+    g.err = ctx->err;
     g.a_rows0 = ctx->sc_rs;
     g.K0 = ctx->dnp;
     g.a_rows1 = ctx->sc_rd;
@@ -1433,6 +1439,7 @@ tg_status tg_gemm(tg_ctx* ctx, int32_t precision, int32_t M, int32_t N, int32_t 
   if (!ctx->gemm_m) TRY(dalloc(ctx, &ctx->gemm_m, 1));
   launch_set_int(ctx->gemm_m, M, st);  // stream-ordered (device count as on the hot path)
   GemmArgs g{};
+  g.err = ctx->err;
   g.a_base0 = A;
   g.lda0 = K;
   g.K0 = g.K = K;

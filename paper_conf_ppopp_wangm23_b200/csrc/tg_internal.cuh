@@ -89,7 +89,8 @@ inline cudaError_t launch_k_cluster(void (*kern)(KArgs...), dim3 grid, dim3 bloc
 }
 
 // device error bits (sticky)
-enum : int { kErrNodeRange = 1, kErrIndexFull = 2, kErrDedupFull = 4, kErrEidRange = 8, kErrPairIndex = 16 };
+enum : int { kErrNodeRange = 1, kErrIndexFull = 2, kErrDedupFull = 4, kErrEidRange = 8, kErrPairIndex = 16,
+             kErrF16Range = 32 };
 
 __host__ __device__ inline int round4(int x) { return (x + 3) & ~3; }
 
@@ -308,6 +309,7 @@ struct GemmArgs {
   const float* ln_g;
   const float* ln_b;
   int ln_dn, ln_de, ln_dt, ln_s1, ln_s2;
+  int* err;                     // sticky device error word (F16X3 range check), may be null
 };
 void launch_gemm_simt(const GemmArgs& g, cudaStream_t st);
 

@@ -17,6 +17,7 @@ struct TcWeights {
   int BN = 0;              // N tile (multiple of 16, <= 256)
   int ntn = 0;             // N tiles
   int nkb = 0;             // K blocks of 128 bytes
+  float* colscale = nullptr;  // F16X3: per output column 2^-e undoing the weight-row scale [ntn * BN]
 };
 
 // Dense A operand loaded by TMA tensor copies (cp.async.bulk.tensor.2d, 128B

@@ -14,7 +14,7 @@ _PKG = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("TG_LIB") or os.path.join(_PKG, "libtg.so")
 
 TG_OPT_DEDUP, TG_OPT_CACHE, TG_OPT_TTABLE, TG_OPT_ALL = 1, 2, 4, 7
-TG_PREC_FP32, TG_PREC_TF32X3, TG_PREC_BF16, TG_PREC_TF32 = 0, 1, 2, 3
+TG_PREC_FP32, TG_PREC_TF32X3, TG_PREC_BF16, TG_PREC_TF32, TG_PREC_F16X3 = 0, 1, 2, 3, 4
 TG_MAX_LAYERS = 4
 TG_CNT_PER_LAYER = 6
 TG_CNT_TTABLE = (TG_MAX_LAYERS + 1) * TG_CNT_PER_LAYER
