@@ -481,6 +481,20 @@ def measure(args, prec_name, s, flat, mc, ctx_kw, shard, world, rank, local, dis
     return out
 
 
+def spawn_cmd(argv, gpus, port):
+    """One rank per GPU on this node through torch.distributed.run (127.0.0.1 rendezvous)."""
+    return [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={gpus}",
+            "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *argv]
+
+
+def check_world(world_env, gpus):
+    """WORLD_SIZE (0 = unset) against --gpus: returns the world size, raises on a mismatch."""
+    world = max(int(world_env), 1)
+    if world != gpus:
+        raise SystemExit(f"WORLD_SIZE={world} but --gpus {gpus}")
+    return world
+
+
 def _free_port():
     so = socket.socket()
     so.bind(("127.0.0.1", 0))
@@ -511,13 +525,8 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "0"))
     if args.gpus > 1 and world == 0:
         # spawn one rank per GPU on this node (north_star: one process per GPU, NCCL)
-        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
-               "--master-addr=127.0.0.1", f"--master-port={_free_port()}", os.path.abspath(__file__),
-               *sys.argv[1:]]
-        sys.exit(subprocess.call(cmd))
-    world = max(world, 1)
-    if world != args.gpus:
-        raise SystemExit(f"WORLD_SIZE={world} but --gpus {args.gpus}")
+        sys.exit(subprocess.call(spawn_cmd(sys.argv[1:], args.gpus, _free_port())))
+    world = check_world(world, args.gpus)
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
 

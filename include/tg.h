@@ -54,6 +54,11 @@ typedef struct tg_ctx tg_ctx; /* opaque; one per device */
 #define TG_OPT_CACHE  2u  /* memo cache at layers 1..L-1 (Sec. 4.2)    */
 #define TG_OPT_TTABLE 4u  /* precomputed Phi(dt) window [0, W) (Sec. 4.3)      */
 #define TG_OPT_ALL    7u
+/* Storage location of the memo cache (NEXT-2; the paper's design choice, Table 5):
+ * the FIFO payload ring of every cached layer lives in pinned, mapped host memory (read
+ * and written by the kernels over PCIe / C2C); the index stays in HBM. Outputs and counters
+ * are unchanged; only speed and bytes moved differ. Not part of TG_OPT_ALL. */
+#define TG_OPT_HOST_CACHE 8u
 
 /* Arithmetic of the dense projections. */
 #define TG_PREC_FP32  0   /* fp32 FFMA (CUDA cores): rtol 1e-4 / atol 1e-5 vs oracle */
@@ -147,7 +152,7 @@ tg_status tg_score_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, co
  * and writes scores[p] = sigmoid(MLP(h[pair_a[p]], h[pair_b[p]])) (R10) for
  * every pair of target indices (0 <= pair_a[p], pair_b[p] < n_targets).
  * n_targets <= max_batch_targets; n_pairs <= max_batch_targets.
- * nodes/ts/pair_a/pair_b: all host or all device; scores: either.
+ * nodes/ts/pair_a/pair_b: all host or all device (a mix is TG_EINVAL); scores: either.
  * Updates the memo cache and the counters like tg_embed_batch.
  * Errors: TG_EINVAL (sizes, null, host pair index out of range), TG_ESTATE;
  * a device pair index out of range sets the sticky device error bit 16
@@ -157,15 +162,28 @@ tg_status tg_score_pairs(tg_ctx* ctx, const int32_t* nodes, const uint32_t* ts, 
                          void* cuda_stream);
 
 /* The paper's inference task: the whole edge range [0, n_edges) in
- * chronological batches of `batch` edges (the last one partial, R13), one
- * tg_score_edges per batch, issued from native code without host sync
- * (batch chain captured once into a CUDA graph when possible).
- * src/dst/ts: either, [n_edges]; scores: either, [n_edges].
+ * chronological batches of `batch` edges (the last one partial, R13), with the
+ * per-batch semantics of tg_score_edges, issued from native code as superbatches
+ * of S batches (tg_superbatch) on two internal streams without host sync.
+ * src/dst/ts: all host or all device (a mix is TG_EINVAL), [n_edges]; scores:
+ * either, [n_edges].
  * batch_counters: optional device int64 [n_batches x TG_NCOUNTERS] that
  * receives each batch's counters (NULL = not recorded). */
 tg_status tg_score_stream(tg_ctx* ctx, const int32_t* src, const int32_t* dst, const uint32_t* ts,
                           int64_t n_edges, int32_t batch, float* scores, int64_t* batch_counters,
                           void* cuda_stream);
+
+/* Link-prediction evaluation with negatives over the whole stream (NEXT-3; the TGAT
+ * evaluation protocol the paper's task follows, [37]): like tg_score_stream, but
+ * batch b's target list is src || dst || neg at the edge times (3 x batch targets, ONE
+ * deduplicated Alg. 1 batch) and it writes scores[e] = p(src_e, dst_e) and
+ * scores[n_edges + e] = p(src_e, neg_e) (R10). neg[e] (1..n_nodes) is the caller's seeded
+ * negative destination of edge e -- an input, not part of the method. Requires
+ * 3 x batch <= max_batch_targets. src/dst/ts/neg: all host or all device (a mix is
+ * TG_EINVAL); scores: either, [2 x n_edges]. Errors as tg_score_stream. */
+tg_status tg_score_stream_neg(tg_ctx* ctx, const int32_t* src, const int32_t* dst, const uint32_t* ts,
+                              const int32_t* neg, int64_t n_edges, int32_t batch, float* scores,
+                              int64_t* batch_counters, void* cuda_stream);
 
 /* Empties the memo cache (all layers) and zeroes the counters; new_limit >= 0
  * replaces the item limit (must be <= the limit given to tg_model_load), < 0

@@ -209,22 +209,26 @@ void launch_layernorm(const float* y, float* r, int Dp, int dn, int dnp, int de,
 // p_e = sigmoid(W_a2 ReLU(W_a1 [h_src || h_dst] + b_a1) + b_a2) (R10) as
 // (1) row resolution through each batch's inverse index (DedupInvert),
 // (2) the hidden layer as a projection GEMM over the S*B edges, (3) a warp
-// per edge for the W_a2 dot product and the sigmoid.
+// per edge for the W_a2 dot product and the sigmoid. With negatives (es.neg,
+// NEXT-3) rows S*B.. score (src_e, neg_e) into scores[n_edges + e].
 __global__ void k_score_rows(const float* __restrict__ HL, int ldh, LevelDev top, int S, EdgeSrc es,
                              const float** __restrict__ rs, const float** __restrict__ rd,
                              long long* __restrict__ oidx, int* __restrict__ m_dev) { pdl_enter();
-  const int tot = S * es.B;
+  const int half = S * es.B;
+  const int tot = es.neg ? 2 * half : half;
   if (blockIdx.x == 0 && threadIdx.x == 0) *m_dev = tot;
   for (int w = blockIdx.x * blockDim.x + threadIdx.x; w < tot; w += gridDim.x * blockDim.x) {
-    const int b = w / es.B, e = w - b * es.B;
+    const int ng = w >= half;
+    const int wp = w - ng * half;
+    const int b = wp / es.B, e = wp - b * es.B;
     const int64_t lo = es.e0 + (int64_t)b * es.B;
     const int64_t rem = es.n_edges - lo;
     const int Bb = (int)(rem < es.B ? (rem < 0 ? 0 : rem) : es.B);
     if (e < Bb) {
       const size_t seg = (size_t)b * top.cap;
       rs[w] = HL + (size_t)(top.c_base[b] + top.inv[seg + e]) * ldh;
-      rd[w] = HL + (size_t)(top.c_base[b] + top.inv[seg + Bb + e]) * ldh;
-      oidx[w] = lo + e;
+      rd[w] = HL + (size_t)(top.c_base[b] + top.inv[seg + (ng ? 2 : 1) * Bb + e]) * ldh;
+      oidx[w] = (ng ? es.n_edges : 0) + lo + e;
     } else {  // past the stream end: any valid row, result discarded
       rs[w] = HL;
       rd[w] = HL;
@@ -235,7 +239,7 @@ __global__ void k_score_rows(const float* __restrict__ HL, int ldh, LevelDev top
 
 void launch_score_rows(const float* HL, int ldh, LevelDev top, int S, EdgeSrc es, const float** rs,
                        const float** rd, long long* oidx, int* m_dev, cudaStream_t st) {
-  int blocks = (S * es.B + 255) / 256;
+  int blocks = ((es.neg ? 2 : 1) * S * es.B + 255) / 256;
   if (blocks < 1) blocks = 1;
   launch_k(k_score_rows, dim3(blocks), dim3(256), 0, st, HL, ldh, top, S, es, rs, rd, oidx, m_dev);
 }

@@ -70,15 +70,16 @@ k_dedup(LevelDev lv, int edge_mode, EdgeSrc es, long long* cnt, int layer, int* 
   int Bb = 0, n;
   if (edge_mode) {
     Bb = batch_edges(es, b, elo);
-    n = 2 * Bb;  // targets src || dst at the edge time
+    n = (es.neg ? 3 : 2) * Bb;  // targets src || dst (|| neg) at the edge time
   } else {
     n = lv.n_in[b];
   }
   const size_t seg = (size_t)b * lv.cap;
   auto item = [&](int i, int32_t& node, uint32_t& t) {
     if (edge_mode) {
-      const int64_t e = elo + (i < Bb ? i : i - Bb);
-      node = i < Bb ? es.src[e] : es.dst[e];
+      const int part = i < Bb ? 0 : (i < 2 * Bb ? 1 : 2);
+      const int64_t e = elo + (i - part * Bb);
+      node = part == 0 ? es.src[e] : (part == 1 ? es.dst[e] : es.neg[e]);
       t = es.ts[e];
     } else {
       node = lv.in_node[seg + i];
@@ -187,7 +188,7 @@ __global__ void k_dedup_off(LevelDev lv, int S, int edge_mode, EdgeSrc es, long 
     int Bb = 0, n;
     if (edge_mode) {
       Bb = batch_edges(es, b, elo);
-      n = 2 * Bb;
+      n = (es.neg ? 3 : 2) * Bb;
     } else {
       n = lv.n_in[b];
     }
@@ -196,8 +197,9 @@ __global__ void k_dedup_off(LevelDev lv, int S, int edge_mode, EdgeSrc es, long 
       int32_t node;
       uint32_t t;
       if (edge_mode) {
-        const int64_t e = elo + (i < Bb ? i : i - Bb);
-        node = i < Bb ? es.src[e] : es.dst[e];
+        const int part = i < Bb ? 0 : (i < 2 * Bb ? 1 : 2);
+        const int64_t e = elo + (i - part * Bb);
+        node = part == 0 ? es.src[e] : (part == 1 ? es.dst[e] : es.neg[e]);
         t = es.ts[e];
       } else {
         node = lv.in_node[seg + i];
@@ -411,6 +413,35 @@ k_probe(LevelDev lv, int S, CacheDev c, int use_cache, int has_ring, long long* 
 //      global index (key -> head0 + q), skipping keys re-missed later.
 // The newest copy of a key is always first on its probe chain (an insert
 // takes the first dead or empty slot), so lookups stop at the first match.
+__device__ __forceinline__ int sbh_pre(const LevelDev& lv, int S, int* s_pre) {
+  if (threadIdx.x == 0) {
+    int a = 0;
+    for (int b = 0; b < S; ++b) {
+      s_pre[b] = a;
+      a += lv.n_u[b];
+    }
+    s_pre[S] = a;
+  }
+  __syncthreads();
+  return s_pre[S];
+}
+__device__ __forceinline__ int sbh_batch(const int* s_pre, int S, int j) {  // last b with pre[b] <= j
+  int lo = 0, hi = S - 1;
+  while (lo < hi) {
+    const int mid = (lo + hi + 1) >> 1;
+    if (s_pre[mid] <= j) lo = mid; else hi = mid - 1;
+  }
+  return lo;
+}
+__device__ __forceinline__ unsigned long long sbh_mask(const CacheDev& c, int NT) {
+  unsigned long long T = 1024;
+  while (T < 2ull * (unsigned long long)NT && T <= c.sb_mask) T <<= 1;
+  return (T > c.sb_mask + 1 ? c.sb_mask + 1 : T) - 1;
+}
+__device__ __forceinline__ bool sbh_evfree(const CacheDev& c, int NT) {
+  return __ldcg(c.state + 1) + NT <= __ldcg(c.state + 2);
+}
+
 __global__ void k_probe_pre(LevelDev lv, int S, CacheDev c) { pdl_enter();
   // an index rebuild (launch_index_maint, just before) left its filled-slot count in state[7]
   if (blockIdx.x == 0 && threadIdx.x == 0 &&
@@ -419,7 +450,19 @@ __global__ void k_probe_pre(LevelDev lv, int S, CacheDev c) { pdl_enter();
   if (blockIdx.x == 0 && threadIdx.x == 0 && c.occ_report) {  // one 64-bit store: consistent pair
     const unsigned long long occ = (unsigned long long)c.state[3] & ((1ull << 40) - 1);
     *(volatile unsigned long long*)c.occ_report = ((unsigned long long)(c.report_sb + 1) << 40) | occ;
+    if (c.size_report)  // live size at superbatch start (host bound for the eviction-free schedule)
+      *(volatile unsigned long long*)c.size_report =
+          ((unsigned long long)(c.report_sb + 1) << 40) | ((unsigned long long)c.state[1] & ((1ull << 40) - 1));
     __threadfence_system();
+  }
+  if (c.sb_key) {  // clear the superbatch-scoped hash of the grid-wide pass (k_sbh_*)
+    __shared__ int s_pre[kMaxS + 1];
+    const unsigned long long T = sbh_mask(c, sbh_pre(lv, S, s_pre)) + 1;
+    for (unsigned long long h = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; h < T;
+         h += (unsigned long long)gridDim.x * blockDim.x) {
+      c.sb_key[h] = kEmptyKey;
+      c.sb_val[h] = 0xFFFFFFFFu;
+    }
   }
   const int tot = S * lv.cap;
   for (int idx = blockIdx.x * blockDim.x + threadIdx.x; idx < tot; idx += gridDim.x * blockDim.x) {
@@ -459,6 +502,12 @@ k_probe_seq(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err)
   const unsigned rank = cluster.block_rank();
   const int tid = threadIdx.x;
   if (c.state[5] == 1) return;  // the eviction-free parallel pass handled this superbatch
+  // the host runs superbatches that may evict with S small enough for this DSMEM hash
+  // (tg_model_load: S_small); a larger one would overflow it -- report, never mis-count
+  if ((long long)S * lv.cap * 10 > (long long)CL * kSeqSlots * 9) {
+    if (rank == 0 && tid == 0) atomicOr(err, kErrIndexFull);
+    return;
+  }
   for (int s = tid; s < kSeqSlots; s += blockDim.x) skey[s] = kEmptyKey;
   if (rank == 0 && tid == 0) {
     s_head = __ldcg(c.state + 0);
@@ -585,161 +634,166 @@ k_probe_seq(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err)
 // the start or inserted during the superbatch can leave the FIFO window, so
 // the sequential outcome is closed-form: the occurrence of a key in batch b
 // hits iff an earlier batch of the superbatch holds the same key, or the key
-// is live in the index at superbatch start. One cluster pass over the
-// concatenated unique lists (j = batch-major order, the order of Alg. 1's
-// lookups) finds first occurrences (DSMEM hash, min position), ranks the
-// misses with an ordered scan (their FIFO positions are head0 + q) and hands
-// every later occurrence the ring slot of its first one.
-__global__ void __launch_bounds__(kSeqThreads, 1)
-k_probe_par(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err) { pdl_enter();
-  extern __shared__ __align__(16) unsigned char smem[];
-  unsigned long long* skey = reinterpret_cast<unsigned long long*>(smem);
-  unsigned* sval = reinterpret_cast<unsigned*>(skey + kSeqSlots);  // min j, later: ring slot
+// is live in the index at superbatch start. Over the concatenated unique lists
+// (j = batch-major order, the order of Alg. 1's lookups), grid-wide on every SM,
+// with a superbatch-scoped hash table in global memory (cleared by k_probe_pre):
+//   k_sbh_insert  every key: claim a table slot (CAS on the key), atomicMin(j);
+//   k_sbh_count   misses = first occurrences not live at superbatch start, per
+//                 contiguous block of j;
+//   k_sbh_assign  ordered rank q of every miss (block offset + block scan): its
+//                 FIFO position is head0 + q; first occurrences publish their slot;
+//   k_sbh_finish  later occurrences take the slot of their first; per-batch
+//                 compute-list bounds, counters and the FIFO state.
+// If eviction is possible the four kernels return at once and the ordered pass
+// (k_probe_seq) handles the superbatch.
+__global__ void k_sbh_insert(LevelDev lv, int S, CacheDev c, int* err) { pdl_enter();
+  __shared__ int s_pre[kMaxS + 1];
+  const int NT = sbh_pre(lv, S, s_pre);
+  const bool ef = sbh_evfree(c, NT);
+  if (blockIdx.x == 0 && threadIdx.x == 0) c.state[5] = ef ? 1 : 0;
+  if (!ef) return;
+  const unsigned long long tmask = sbh_mask(c, NT);
+  for (int j = blockIdx.x * blockDim.x + threadIdx.x; j < NT; j += gridDim.x * blockDim.x) {
+    const int b = sbh_batch(s_pre, S, j);
+    const size_t idx = (size_t)b * lv.cap + (j - s_pre[b]);
+    const unsigned long long key = tkey(lv.u_node[idx], lv.u_ts[idx]);
+    unsigned long long h = mix64(key) & tmask;
+    int hs = -1;
+    for (unsigned long long pr = 0; pr <= tmask; ++pr) {
+      const unsigned long long old = atomicCAS(c.sb_key + h, kEmptyKey, key);
+      if (old == kEmptyKey || old == key) {
+        atomicMin(c.sb_val + h, (unsigned)j);
+        hs = (int)h;
+        break;
+      }
+      h = (h + 1) & tmask;
+    }
+    if (hs < 0) atomicOr(err, kErrDedupFull);
+    c.sb_h[idx] = hs;
+  }
+}
+
+// miss test of entry j (first occurrence, not live at superbatch start)
+__device__ __forceinline__ bool sbh_first(const LevelDev& lv, const CacheDev& c, size_t idx, int j) {
+  const int h = c.sb_h[idx];
+  return h >= 0 && __ldcg(c.sb_val + h) == (unsigned)j;
+}
+
+__global__ void __launch_bounds__(kSbhThreads) k_sbh_count(LevelDev lv, int S, CacheDev c) { pdl_enter();
   __shared__ int s_pre[kMaxS + 1];
   __shared__ int s_warp[32];
-  __shared__ int s_total;
-  cg::cluster_group cluster = cg::this_cluster();
-  const unsigned CL = cluster.num_blocks();
-  const unsigned rank = cluster.block_rank();
-  const int tid = threadIdx.x;
-  const long long head0 = __ldcg(c.state + 0), size0 = __ldcg(c.state + 1), limit = __ldcg(c.state + 2);
-  if (tid == 0) {
-    int a = 0;
-    for (int b = 0; b < S; ++b) {
-      s_pre[b] = a;
-      a += lv.n_u[b];
-    }
-    s_pre[S] = a;
-  }
-  __syncthreads();
-  const int NT = s_pre[S];
-  if (size0 + NT > limit) {  // eviction possible: the ordered pass handles this superbatch
-    if (rank == 0 && tid == 0) c.state[5] = 0;
-    return;                  // uniform over the cluster (same inputs everywhere)
-  }
-  for (int s = tid; s < kSeqSlots; s += blockDim.x) {
-    skey[s] = kEmptyKey;
-    sval[s] = 0xFFFFFFFFu;
-  }
-  const long long live_lo = head0 - size0;
-  const unsigned long long tmask = (unsigned long long)CL * kSeqSlots - 1ull;
-  cluster.sync();
-  const int chunk = (NT + (int)CL - 1) / (int)CL;
-  const int cbeg = min(NT, (int)rank * chunk), cend = min(NT, cbeg + chunk);
-  const int ipt = (chunk + (int)blockDim.x - 1) / (int)blockDim.x;
-  const int tbeg = cbeg + tid * ipt;
-  unsigned hs[kDedupIPT];
-  int jb[kDedupIPT];
-  // ---- first occurrences (min j per key)
+  const int NT = sbh_pre(lv, S, s_pre);
+  if (__ldcg(c.state + 5) != 1) return;
+  const long long live_lo = __ldcg(c.state + 0) - __ldcg(c.state + 1);
+  const int j0 = blockIdx.x * kSbhChunk + threadIdx.x * kSbhItems;
+  int m = 0;
 #pragma unroll
-  for (int j = 0; j < kDedupIPT; ++j) {
-    hs[j] = 0xFFFFFFFFu;
-    jb[j] = 0;
-    const int i = tbeg + j;
-    if (j < ipt && i < cend) {
-      int b = 0;
-      while (b + 1 < S && s_pre[b + 1] <= i) ++b;
-      jb[j] = b;
-      const size_t idx = (size_t)b * lv.cap + (i - s_pre[b]);
-      const unsigned long long key = tkey(lv.u_node[idx], lv.u_ts[idx]);
-      unsigned long long h = mix64(key) & tmask;
-      for (unsigned long long pr = 0; pr <= tmask; ++pr) {
-        unsigned long long* kp = cluster.map_shared_rank(skey, (unsigned)(h / kSeqSlots)) + (h % kSeqSlots);
-        const unsigned long long old = atomicCAS(kp, kEmptyKey, key);
-        if (old == kEmptyKey || old == key) {
-          atomicMin(cluster.map_shared_rank(sval, (unsigned)(h / kSeqSlots)) + (h % kSeqSlots), (unsigned)i);
-          hs[j] = (unsigned)h;
-          break;
-        }
-        h = (h + 1) & tmask;
+  for (int e = 0; e < kSbhItems; ++e) {
+    const int j = j0 + e;
+    if (j < NT) {
+      const int b = sbh_batch(s_pre, S, j);
+      const size_t idx = (size_t)b * lv.cap + (j - s_pre[b]);
+      if (sbh_first(lv, c, idx, j)) {
+        const long long p = __ldcg(lv.p0 + idx);
+        m += !(p >= 0 && p >= live_lo);
       }
-      if (hs[j] == 0xFFFFFFFFu) atomicOr(err, kErrDedupFull);
     }
   }
-  cluster.sync();
-  // ---- misses = first occurrences not live at superbatch start; ordered rank
-  unsigned firstmask = 0, missmask = 0;
-  int m_local = 0;
+  int tot;
+  block_excl_scan(m, s_warp, tot);
+  if (threadIdx.x == 0) c.sb_blk[blockIdx.x] = tot;
+}
+
+__global__ void __launch_bounds__(kSbhThreads) k_sbh_assign(LevelDev lv, int S, CacheDev c) { pdl_enter();
+  __shared__ int s_pre[kMaxS + 1];
+  __shared__ int s_warp[32];
+  __shared__ int s_off;
+  const int NT = sbh_pre(lv, S, s_pre);
+  if (__ldcg(c.state + 5) != 1) return;
+  const long long head0 = __ldcg(c.state + 0);
+  const long long live_lo = head0 - __ldcg(c.state + 1);
+  if (threadIdx.x == 0) {
+    int o = 0;
+    for (int q = 0; q < (int)blockIdx.x; ++q) o += __ldcg(c.sb_blk + q);
+    s_off = o;
+  }
+  const int j0 = blockIdx.x * kSbhChunk + threadIdx.x * kSbhItems;
+  unsigned first = 0, miss = 0;
+  int m = 0;
 #pragma unroll
-  for (int j = 0; j < kDedupIPT; ++j) {
-    const int i = tbeg + j;
-    if (j < ipt && i < cend && hs[j] != 0xFFFFFFFFu) {
-      const unsigned h = hs[j];
-      if (*(cluster.map_shared_rank(sval, h / kSeqSlots) + (h % kSeqSlots)) == (unsigned)i) {
-        firstmask |= 1u << j;
-        const size_t idx = (size_t)jb[j] * lv.cap + (i - s_pre[jb[j]]);
+  for (int e = 0; e < kSbhItems; ++e) {
+    const int j = j0 + e;
+    if (j < NT) {
+      const int b = sbh_batch(s_pre, S, j);
+      const size_t idx = (size_t)b * lv.cap + (j - s_pre[b]);
+      if (sbh_first(lv, c, idx, j)) {
+        first |= 1u << e;
         const long long p = __ldcg(lv.p0 + idx);
         if (!(p >= 0 && p >= live_lo)) {
-          missmask |= 1u << j;
-          ++m_local;
+          miss |= 1u << e;
+          ++m;
         }
       }
     }
   }
-  int tot_cta;
-  const int excl = block_excl_scan(m_local, s_warp, tot_cta);
-  if (tid == 0) s_total = tot_cta;
-  cluster.sync();  // first-decisions done everywhere (sval may be overwritten now)
-  int before = 0;
-  for (unsigned r = 0; r < rank; ++r) before += *cluster.map_shared_rank(&s_total, r);
-  int q = before + excl;
+  int tot;
+  const int excl = block_excl_scan(m, s_warp, tot);  // (syncs: s_off visible)
+  int q = s_off + excl;
 #pragma unroll
-  for (int j = 0; j < kDedupIPT; ++j) {
-    if (firstmask & (1u << j)) {
-      const int i = tbeg + j;
-      const int b = jb[j];
-      const int u = i - s_pre[b];
-      const size_t idx = (size_t)b * lv.cap + u;
-      long long sl;
-      if (missmask & (1u << j)) {
-        lv.c_b[q] = b;
-        lv.c_u[q] = u;
-        lv.c_node[q] = lv.u_node[idx];
-        lv.c_ts[q] = lv.u_ts[idx];
-        lv.sup[q] = 0;
-        sl = (head0 + q) % c.rcap;
-        ++q;
-      } else {
-        sl = __ldcg(lv.p0 + idx) % c.rcap;
-      }
-      lv.slot[idx] = sl;
-      const unsigned h = hs[j];
-      *(cluster.map_shared_rank(sval, h / kSeqSlots) + (h % kSeqSlots)) = (unsigned)sl;
+  for (int e = 0; e < kSbhItems; ++e) {
+    if (!(first & (1u << e))) continue;
+    const int j = j0 + e;
+    const int b = sbh_batch(s_pre, S, j);
+    const int u = j - s_pre[b];
+    const size_t idx = (size_t)b * lv.cap + u;
+    long long sl;
+    if (miss & (1u << e)) {
+      lv.c_b[q] = b;
+      lv.c_u[q] = u;
+      lv.c_node[q] = lv.u_node[idx];
+      lv.c_ts[q] = lv.u_ts[idx];
+      lv.sup[q] = 0;
+      sl = (head0 + q) % c.rcap;
+      ++q;
+    } else {
+      sl = __ldcg(lv.p0 + idx) % c.rcap;
     }
+    lv.slot[idx] = sl;
+    c.sb_slot[c.sb_h[idx]] = sl;
   }
-  cluster.sync();
-  // ---- later occurrences: the slot of the first one; per-batch bookkeeping
-#pragma unroll
-  for (int j = 0; j < kDedupIPT; ++j) {
-    const int i = tbeg + j;
-    if (j < ipt && i < cend && hs[j] != 0xFFFFFFFFu && !(firstmask & (1u << j))) {
-      const unsigned h = hs[j];
-      const size_t idx = (size_t)jb[j] * lv.cap + (i - s_pre[jb[j]]);
-      lv.slot[idx] = *(cluster.map_shared_rank(sval, h / kSeqSlots) + (h % kSeqSlots));
-    }
+}
+
+__global__ void k_sbh_finish(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int nblk) { pdl_enter();
+  __shared__ int s_pre[kMaxS + 1];
+  __shared__ int s_M;
+  const int NT = sbh_pre(lv, S, s_pre);
+  if (__ldcg(c.state + 5) != 1) return;
+  // later occurrences: the slot of the first one (Alg. 1 l.8 hit inside the superbatch)
+  for (int j = blockIdx.x * blockDim.x + threadIdx.x; j < NT; j += gridDim.x * blockDim.x) {
+    const int b = sbh_batch(s_pre, S, j);
+    const size_t idx = (size_t)b * lv.cap + (j - s_pre[b]);
+    if (!sbh_first(lv, c, idx, j)) lv.slot[idx] = __ldcg(c.sb_slot + c.sb_h[idx]);
   }
-  if (rank == CL - 1 && tid == 0) {
-    const int M = before + tot_cta;  // last CTA: total misses
-    *lv.n_c_total = M;
-    c.state[4] = head0;
-    c.state[0] = head0 + M;
-    c.state[1] = size0 + M;
-    c.state[5] = 1;
+  if (blockIdx.x != 0) return;
+  if (threadIdx.x == 0) {
+    int M = 0;
+    for (int q = 0; q < nblk; ++q) M += __ldcg(c.sb_blk + q);
+    s_M = M;
   }
-  cluster.sync();  // remote smem reads done; n_c per batch needs every miss counted
-  if (rank == 0 && tid < S) {
-    // misses of batch b = misses with j in [pre[b], pre[b+1]); recount from the compute list
-    const int b = tid;
-    const int M = *lv.n_c_total;
+  __syncthreads();
+  const int M = s_M;
+  if (threadIdx.x < S) {
+    // misses of batch b = misses with j in [pre[b], pre[b+1]): bounds in the compute list
+    const int b = threadIdx.x;
     int lo = 0, hi = M;  // first q with c_b[q] >= b
     while (lo < hi) {
       const int mid = (lo + hi) >> 1;
-      if (lv.c_b[mid] < b) lo = mid + 1; else hi = mid;
+      if (__ldcg(lv.c_b + mid) < b) lo = mid + 1; else hi = mid;
     }
     int lo2 = lo, hi2 = M;  // first q with c_b[q] > b
     while (lo2 < hi2) {
       const int mid = (lo2 + hi2) >> 1;
-      if (lv.c_b[mid] <= b) lo2 = mid + 1; else hi2 = mid;
+      if (__ldcg(lv.c_b + mid) <= b) lo2 = mid + 1; else hi2 = mid;
     }
     const int n = s_pre[b + 1] - s_pre[b], m = lo2 - lo;
     lv.c_base[b] = lo;
@@ -748,6 +802,14 @@ k_probe_par(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err)
     cnt_add(cnt, b, L6 + 2, n);      // lookups
     cnt_add(cnt, b, L6 + 3, n - m);  // hits
     cnt_add(cnt, b, L6 + 4, m);      // misses
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const long long head0 = c.state[0], size0 = c.state[1];
+    *lv.n_c_total = M;
+    c.state[4] = head0;
+    c.state[0] = head0 + M;
+    c.state[1] = size0 + M;
   }
 }
 
@@ -946,18 +1008,21 @@ int launch_probe(LevelDev lv, int S, const CacheDev* cache, long long* cnt, int 
   // cluster large enough for every key of the superbatch to be an in-SB miss (load <= 0.6)
   int cl = 1;
   while (cl < kSeqCL && (long long)cl * kSeqSlots * 6 / 10 < (long long)S * lv.cap) cl <<= 1;
-  static bool attr2 = false;
-  if (!attr2) {
-    cudaFuncSetAttribute(k_probe_par, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    cudaFuncSetAttribute(k_probe_par, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
-    attr2 = true;
-  }
-  launch_k_cluster(k_probe_par, dim3(cl), dim3(kSeqThreads), smem, st, cl, lv, S, c, cnt, layer, err);
+  // eviction-free superbatches: grid-wide pass (k_sbh_*); otherwise the ordered pass
+  const int nj = S * lv.cap;
+  int gb = (nj + 255) / 256;
+  if (gb > 148 * 8) gb = 148 * 8;
+  const int nblk = (nj + kSbhChunk - 1) / kSbhChunk;
+  launch_k(k_sbh_insert, dim3(gb), dim3(256), 0, st, lv, S, c, err);
+  launch_k(k_sbh_count, dim3(nblk), dim3(kSbhThreads), 0, st, lv, S, c);
+  launch_k(k_sbh_assign, dim3(nblk), dim3(kSbhThreads), 0, st, lv, S, c);
+  launch_k(k_sbh_finish, dim3(gb), dim3(256), 0, st, lv, S, c, cnt, layer, nblk);
+  if (cl > kSeqCL) cl = kSeqCL;
   launch_k_cluster(k_probe_seq, dim3(cl), dim3(kSeqThreads), smem, st, cl, lv, S, c, cnt, layer, err);
   int ib = (S * lv.cap + 255) / 256;
   if (ib > 148 * 4) ib = 148 * 4;
   launch_k(k_probe_ins, dim3(ib), dim3(256), 0, st, lv, c, err);
-  return 4;
+  return 7;
 }
 
 // ------------------------------------------------------------------ NghLookup

@@ -68,12 +68,22 @@ constexpr int TC_EPI_BYTES = TC_EPI_WARPS * 32 * TC_STG_LD * 4;
 constexpr int TC_LN_MAXTN = 4;
 constexpr int TC_LN_BYTES = (2 * 128 + 2 * TC_LN_MAXTN * 128) * 16 + 4 * 256 * 4;  // + bias, gamma, beta, valid
 
-static inline int tc_stages(int prec, int BN, int ln = 0) {
+// Shared-memory plan: `stages` operand stages plus, when the generic fp32 A producer runs,
+// `stg` staging units of 16 KB (its cp.async look-ahead ring, up to 4 units) -- as many
+// staging units as fit beside 2 stages, then as many stages as fit beside those.
+constexpr int TC_STG_UNIT = TC_BM * 128;
+static inline void tc_plan(int prec, int BN, int ln, bool generic, int* stages, int* stg) {
   const size_t st = (size_t)tc_planes(prec) * ((size_t)TC_BM * 128 + (size_t)BN * 128);
   const size_t budget = (tc_ctas_per_sm(prec) == 1 ? 205 * 1024 : 100 * 1024) - (ln ? TC_LN_BYTES : 0);
-  int s = (int)(budget / st);
+  int d = 0;  // 0: no room beside 2 stages -> the producers load synchronously
+  if (generic) {
+    d = budget > 2 * st ? (int)((budget - 2 * st) / TC_STG_UNIT) : 0;
+    d = d > 4 ? 4 : d;
+  }
+  int s = (int)((budget - (size_t)d * TC_STG_UNIT) / st);
   if (s > TC_MAXSTAGES) s = TC_MAXSTAGES;
-  return s < 2 ? 2 : s;
+  *stages = s < 2 ? 2 : s;
+  *stg = d;
 }
 
 // ------------------------------------------------------------ host: weights
@@ -364,11 +374,10 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t* v) {
 
 template <int PREC>
 __global__ void __launch_bounds__(TC_THREADS, 1)
-    k_gemm_tc(GemmArgs g, TcWeights w, int stages, const __grid_constant__ CUtensorMap tmA, int a_tma,
+    k_gemm_tc(GemmArgs g, TcWeights w, int stages, int stg, const __grid_constant__ CUtensorMap tmA, int a_tma,
               const __grid_constant__ CUtensorMap tmA2, int a2_kb0, int a2_x0) {
   constexpr int EPC = (PREC == TG_PREC_BF16 || PREC == TG_PREC_F16X3) ? 64 : 32;
   constexpr int PLANES = (PREC == TG_PREC_TF32X3 || PREC == TG_PREC_F16X3) ? 2 : 1;
-  constexpr int NV = EPC / 4;  // float4 loads per row per k-block
   extern __shared__ __align__(1024) unsigned char smem_raw[];
   // 1024-byte alignment (128B swizzle atoms) by an integer offset from smem_raw, so
   // the compiler keeps the shared address space (LDS/STS, not generic LD/ST)
@@ -506,85 +515,140 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       }
     }
   } else if (warp < 4) {
-    // ===================== A producers
-    uint32_t gk = 0;
-    for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
-      const int tm = t / w.ntn;
-      const int row = tm * TC_BM + tid;
-      const bool rv = row < M;
-      const float* r0 = nullptr;
-      const float* r1 = nullptr;
-      if (rv) {
-        r0 = g.a_rows0 ? g.a_rows0[row] : g.a_base0 + (size_t)row * g.lda0;
-        if (g.K0 < g.K) r1 = g.a_rows1 ? g.a_rows1[row] : g.a_base1 + (size_t)row * g.lda1;
+    // ===================== A producers (fp32 rows: gathered through row pointers or dense),
+    // converted on the fly. Loads run ahead through a per-thread cp.async staging ring of
+    // `stg` units (a unit = 32 fp32 = 128 B of the thread's own row; UPK units per k-block),
+    // so up to stg x 16 KB per CTA are in flight without holding registers: the producers
+    // are bound by L2 latency otherwise (one k-block of register prefetch measured ~1.4 us
+    // per k-block at ~35% tensor-pipe activity). Each thread reads back only what it
+    // copied itself (cp.async.wait_group), so no cross-thread synchronisation is needed.
+    constexpr int UPK = EPC / 32;
+    unsigned char* sring = smem + stages * stage_bytes + TC_BAR_BYTES + TC_EPI_BYTES + (g.ln ? TC_LN_BYTES : 0);
+    const int D = stg;
+    const int upt = nkb * UPK;  // units per tile
+    // issue cursor: tile it_t (this CTA's sequence), unit it_u within the tile
+    int it_t = blockIdx.x, it_u = 0;
+    const float* ir0 = nullptr;
+    const float* ir1 = nullptr;
+    bool irv = false;
+    auto rows_of = [&](int tt) {
+      const int row = (tt / w.ntn) * TC_BM + tid;
+      irv = tt < ntiles && row < M;
+      ir0 = ir1 = nullptr;
+      if (irv) {
+        ir0 = g.a_rows0 ? g.a_rows0[row] : g.a_base0 + (size_t)row * g.lda0;
+        if (g.K0 < g.K) ir1 = g.a_rows1 ? g.a_rows1[row] : g.a_base1 + (size_t)row * g.lda1;
       }
-      float4 regs[NV];
+    };
+    rows_of(it_t);
+    const void* dummy = w.hi;  // valid global address for zero-byte (zero-fill) copies
+    auto issue = [&](int slot) {
+      if (it_t < ntiles) {
+        const uint32_t dst = smem_u32(sring + (size_t)slot * (TC_BM * 128) + tid * 128);
+        const int col0 = it_u * 32;
 #pragma unroll
-      for (int v = 0; v < NV; ++v) regs[v] = rv ? tc_load4(g, r0, r1, v * 4) : make_float4(0.f, 0.f, 0.f, 0.f);
+        for (int c = 0; c < 8; ++c) {
+          const int col = col0 + 4 * c;
+          const bool ok = irv && col < g.K;
+          const void* src = !ok ? dummy : (const void*)(col < g.K0 ? ir0 + col : ir1 + (col - g.K0));
+          asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(dst + ((c ^ (tid & 7)) << 4)),
+                       "l"(src), "r"(ok ? 16 : 0)
+                       : "memory");
+        }
+        if (++it_u == upt) {
+          it_u = 0;
+          it_t += gridDim.x;
+          rows_of(it_t);
+        }
+      }
+      asm volatile("cp.async.commit_group;\n" ::: "memory");  // (empty past the last tile)
+    };
+    for (int i = 0; i < D; ++i) issue(i);
+    uint32_t gk = 0, gu = 0;
+    for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+      if (D == 0) rows_of(t);  // no room for staging (widest N tiles): blocking loads
       for (int kb = 0; kb < nkb; ++kb, ++gk) {
         const int s = gk % stages;
         mbar_wait(&empty[s], ((gk / stages) & 1) ^ 1);
         unsigned char* sA = smem + s * stage_bytes;
-        if (PREC == TG_PREC_F16X3) {
-          bool big = false;
+        bool big = false;
 #pragma unroll
-          for (int c = 0; c < 8; ++c) {
-            const float4 x0 = regs[2 * c], x1 = regs[2 * c + 1];
-            const float xs[8] = {x0.x, x0.y, x0.z, x0.w, x1.x, x1.y, x1.z, x1.w};
-            uint32_t hv[4], lv[4];
+        for (int h = 0; h < UPK; ++h, ++gu) {
+          // unit gu is the oldest of the D outstanding groups
+          float4 x[8];
+          const int slot = D > 0 ? (int)(gu % (uint32_t)D) : 0;
+          if (D == 0) {
 #pragma unroll
-            for (int e = 0; e < 4; ++e) {
-              const __half2 h = __floats2half2_rn(xs[2 * e], xs[2 * e + 1]);
-              const float2 hf = __half22float2(h);
-              const __half2 l = __floats2half2_rn(xs[2 * e] - hf.x, xs[2 * e + 1] - hf.y);
-              big |= !(fabsf(xs[2 * e]) < 65504.f) | !(fabsf(xs[2 * e + 1]) < 65504.f);
-              hv[e] = *reinterpret_cast<const uint32_t*>(&h);
-              lv[e] = *reinterpret_cast<const uint32_t*>(&l);
+            for (int c = 0; c < 8; ++c)
+              x[c] = irv ? tc_load4(g, ir0, ir1, (kb * UPK + h) * 32 + 4 * c) : make_float4(0.f, 0.f, 0.f, 0.f);
+          } else {
+            if (D == 1) asm volatile("cp.async.wait_group 0;\n" ::: "memory");
+            else if (D == 2) asm volatile("cp.async.wait_group 1;\n" ::: "memory");
+            else if (D == 3) asm volatile("cp.async.wait_group 2;\n" ::: "memory");
+            else asm volatile("cp.async.wait_group 3;\n" ::: "memory");
+            const unsigned char* src = sring + (size_t)slot * (TC_BM * 128) + tid * 128;
+#pragma unroll
+            for (int c = 0; c < 8; ++c) x[c] = *reinterpret_cast<const float4*>(src + ((c ^ (tid & 7)) << 4));
+          }
+          if (PREC == TG_PREC_F16X3) {
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+              const float xs[8] = {x[2 * j].x, x[2 * j].y, x[2 * j].z, x[2 * j].w,
+                                   x[2 * j + 1].x, x[2 * j + 1].y, x[2 * j + 1].z, x[2 * j + 1].w};
+              uint32_t hv[4], lv[4];
+#pragma unroll
+              for (int e = 0; e < 4; ++e) {
+                const __half2 hh = __floats2half2_rn(xs[2 * e], xs[2 * e + 1]);
+                const float2 hf = __half22float2(hh);
+                const __half2 ll = __floats2half2_rn(xs[2 * e] - hf.x, xs[2 * e + 1] - hf.y);
+                big |= !(fabsf(xs[2 * e]) < 65504.f) | !(fabsf(xs[2 * e + 1]) < 65504.f);
+                hv[e] = *reinterpret_cast<const uint32_t*>(&hh);
+                lv[e] = *reinterpret_cast<const uint32_t*>(&ll);
+              }
+              const int c = h * 4 + j;
+              *reinterpret_cast<uint4*>(sA + sw128(tid, c)) = make_uint4(hv[0], hv[1], hv[2], hv[3]);
+              *reinterpret_cast<uint4*>(sA + a_plane + sw128(tid, c)) = make_uint4(lv[0], lv[1], lv[2], lv[3]);
             }
-            *reinterpret_cast<uint4*>(sA + sw128(tid, c)) = make_uint4(hv[0], hv[1], hv[2], hv[3]);
-            *reinterpret_cast<uint4*>(sA + a_plane + sw128(tid, c)) = make_uint4(lv[0], lv[1], lv[2], lv[3]);
-          }
-          if (big && g.err) atomicOr(g.err, kErrF16Range);
-        } else if (PREC == TG_PREC_BF16) {
+          } else if (PREC == TG_PREC_BF16) {
 #pragma unroll
-          for (int c = 0; c < 8; ++c) {
-            const float4 x0 = regs[2 * c], x1 = regs[2 * c + 1];
-            __nv_bfloat162 p0 = __floats2bfloat162_rn(x0.x, x0.y), p1 = __floats2bfloat162_rn(x0.z, x0.w);
-            __nv_bfloat162 p2 = __floats2bfloat162_rn(x1.x, x1.y), p3 = __floats2bfloat162_rn(x1.z, x1.w);
-            uint4 u;
-            u.x = *reinterpret_cast<uint32_t*>(&p0);
-            u.y = *reinterpret_cast<uint32_t*>(&p1);
-            u.z = *reinterpret_cast<uint32_t*>(&p2);
-            u.w = *reinterpret_cast<uint32_t*>(&p3);
-            *reinterpret_cast<uint4*>(sA + sw128(tid, c)) = u;
-          }
-        } else {
+            for (int j = 0; j < 4; ++j) {
+              const float4 x0 = x[2 * j], x1 = x[2 * j + 1];
+              __nv_bfloat162 p0 = __floats2bfloat162_rn(x0.x, x0.y), p1 = __floats2bfloat162_rn(x0.z, x0.w);
+              __nv_bfloat162 p2 = __floats2bfloat162_rn(x1.x, x1.y), p3 = __floats2bfloat162_rn(x1.z, x1.w);
+              uint4 u;
+              u.x = *reinterpret_cast<uint32_t*>(&p0);
+              u.y = *reinterpret_cast<uint32_t*>(&p1);
+              u.z = *reinterpret_cast<uint32_t*>(&p2);
+              u.w = *reinterpret_cast<uint32_t*>(&p3);
+              *reinterpret_cast<uint4*>(sA + sw128(tid, h * 4 + j)) = u;
+            }
+          } else {
 #pragma unroll
-          for (int c = 0; c < 8; ++c) {
-            const float4 x = regs[c];
-            float4 hi, lo;
-            hi.x = rna_tf32(x.x);
-            hi.y = rna_tf32(x.y);
-            hi.z = rna_tf32(x.z);
-            hi.w = rna_tf32(x.w);
-            *reinterpret_cast<float4*>(sA + sw128(tid, c)) = hi;
-            if (PLANES == 2) {
-              lo.x = rna_tf32(x.x - hi.x);
-              lo.y = rna_tf32(x.y - hi.y);
-              lo.z = rna_tf32(x.z - hi.z);
-              lo.w = rna_tf32(x.w - hi.w);
-              *reinterpret_cast<float4*>(sA + a_plane + sw128(tid, c)) = lo;
+            for (int c = 0; c < 8; ++c) {
+              const float4 xv = x[c];
+              float4 hi, lo;
+              hi.x = rna_tf32(xv.x);
+              hi.y = rna_tf32(xv.y);
+              hi.z = rna_tf32(xv.z);
+              hi.w = rna_tf32(xv.w);
+              *reinterpret_cast<float4*>(sA + sw128(tid, c)) = hi;
+              if (PLANES == 2) {
+                lo.x = rna_tf32(xv.x - hi.x);
+                lo.y = rna_tf32(xv.y - hi.y);
+                lo.z = rna_tf32(xv.z - hi.z);
+                lo.w = rna_tf32(xv.w - hi.w);
+                *reinterpret_cast<float4*>(sA + a_plane + sw128(tid, c)) = lo;
+              }
             }
           }
+          if (D > 0) issue(slot);  // refill the slot just consumed: unit gu + D
         }
+        if (PREC == TG_PREC_F16X3 && big && g.err) atomicOr(g.err, kErrF16Range);
         asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");  // generic -> async proxy
         mbar_arrive(&full[s]);
-        if (kb + 1 < nkb && rv) {  // prefetch the next k-block while this one is consumed
-#pragma unroll
-          for (int v = 0; v < NV; ++v) regs[v] = tc_load4(g, r0, r1, (kb + 1) * EPC + v * 4);
-        }
       }
     }
+    asm volatile("cp.async.wait_group 0;\n" ::: "memory");
   } else if (warp == 4) {
     // ===================== B producer (TMA bulk copies of weight tile images)
     if (lane == 0) {
@@ -901,10 +965,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;\n" ::"r"(tmem), "r"(2 * tc_acc_cols(PREC)));
 }
 
-static size_t tc_smem(int prec, int BN, int stages, int ln = 0) {
+static size_t tc_smem(int prec, int BN, int stages, int stg, int ln = 0) {
   const size_t planes = tc_planes(prec);
   size_t s = 1024 + (size_t)stages * planes * ((size_t)TC_BM * 128 + (size_t)BN * 128) + TC_BAR_BYTES + TC_EPI_BYTES +
-             (ln ? TC_LN_BYTES : 0);
+             (ln ? TC_LN_BYTES : 0) + (size_t)stg * TC_STG_UNIT;
   // tf32x3: one CTA per SM (it allocates all 512 TMEM columns; a second
   // co-resident CTA would block in tcgen05.alloc until the first one exits).
   const size_t one_per_sm = 120 * 1024;
@@ -950,8 +1014,12 @@ void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaSt
   const CUtensorMap& tm2 = two ? ta2->map : zero_map;
   if (!two) a2_kb0 = 1 << 30;
   const int ln = g.ln ? 1 : 0;
-  const int stages = tc_stages(precision, w.BN, ln);
-  const size_t smem = tc_smem(precision, w.BN, stages, ln);
+  // the generic fp32 A producer (cp.async staging) runs unless A comes by TMA, as raw fp32
+  // (one-pass tf32) or as a dense bf16 activation
+  const bool generic = !a_tma && precision != TG_PREC_TF32 && !(precision == TG_PREC_BF16 && g.a_h);
+  int stages = 2, stg = 0;
+  tc_plan(precision, w.BN, ln, generic, &stages, &stg);
+  const size_t smem = tc_smem(precision, w.BN, stages, stg, ln);
   const int tiles = ((g.m_max + TC_BM - 1) / TC_BM) * w.ntn;
   int slots = 148 * tc_ctas_per_sm(precision);
   if (ln) slots = slots / w.ntn * w.ntn;  // whole clusters; a cluster walks the M tiles in lockstep
@@ -988,10 +1056,10 @@ void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaSt
       if (max_cl > 0 && grid > max_cl * w.ntn) grid = max_cl * w.ntn;
     }
     if (ln)
-      launch_k_cluster(k_gemm_tc<TG_PREC_BF16>, dim3(grid), dim3(TC_THREADS), smem, st, w.ntn, g, w, stages, tm,
+      launch_k_cluster(k_gemm_tc<TG_PREC_BF16>, dim3(grid), dim3(TC_THREADS), smem, st, w.ntn, g, w, stages, stg, tm,
                        a_tma, tm2, a2_kb0, a2_x0);
     else
-      launch_k(k_gemm_tc<TG_PREC_BF16>, dim3(grid), dim3(TC_THREADS), smem, st, g, w, stages, tm, a_tma, tm2,
+      launch_k(k_gemm_tc<TG_PREC_BF16>, dim3(grid), dim3(TC_THREADS), smem, st, g, w, stages, stg, tm, a_tma, tm2,
                a2_kb0, a2_x0);
   } else if (precision == TG_PREC_TF32) {
     static size_t set = 0;
@@ -999,7 +1067,7 @@ void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaSt
       cudaFuncSetAttribute(k_gemm_tc<TG_PREC_TF32>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       set = smem;
     }
-    launch_k(k_gemm_tc<TG_PREC_TF32>, dim3(grid), dim3(TC_THREADS), smem, st, g, w, stages, tm, a_tma, tm2,
+    launch_k(k_gemm_tc<TG_PREC_TF32>, dim3(grid), dim3(TC_THREADS), smem, st, g, w, stages, stg, tm, a_tma, tm2,
              a2_kb0, a2_x0);
   } else if (precision == TG_PREC_F16X3) {
     static size_t set = 0;
@@ -1007,7 +1075,7 @@ void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaSt
       cudaFuncSetAttribute(k_gemm_tc<TG_PREC_F16X3>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       set = smem;
     }
-    launch_k(k_gemm_tc<TG_PREC_F16X3>, dim3(grid), dim3(TC_THREADS), smem, st, g, w, stages, tm, 0, tm2,
+    launch_k(k_gemm_tc<TG_PREC_F16X3>, dim3(grid), dim3(TC_THREADS), smem, st, g, w, stages, stg, tm, 0, tm2,
              1 << 30, 0);
   } else {
     static size_t set = 0;
@@ -1015,7 +1083,7 @@ void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaSt
       cudaFuncSetAttribute(k_gemm_tc<TG_PREC_TF32X3>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       set = smem;
     }
-    launch_k(k_gemm_tc<TG_PREC_TF32X3>, dim3(grid), dim3(TC_THREADS), smem, st, g, w, stages, tm, 0, tm2,
+    launch_k(k_gemm_tc<TG_PREC_TF32X3>, dim3(grid), dim3(TC_THREADS), smem, st, g, w, stages, stg, tm, 0, tm2,
              1 << 30, 0);
   }
 }

@@ -49,6 +49,9 @@ struct tg_ctx {
   bool loaded = false;
   tg_model_cfg cfg{};
   int L = 0, H = 0, k = 0, d_n = 0, d_e = 0, d_t = 0, dnp = 0, dep = 0, dtp = 0, Dp = 0, W = 0, S = 1;
+  // superbatch sizes: S (workspaces; superbatches the host can prove eviction-free) and
+  // S_small (superbatches that may evict: the ordered pass's DSMEM hash bounds it)
+  int S_small = 1;
   LayerW lw[TG_MAX_LAYERS];
   float *omega = nullptr, *phi = nullptr, *table = nullptr;
   float *Wa1 = nullptr, *ba1 = nullptr, *Wa2 = nullptr;
@@ -72,6 +75,9 @@ struct tg_ctx {
   int64_t limit0 = 0;
   long long idx_bound[TG_MAX_LAYERS + 1]{};  // host upper bound on occupied index slots (rebuild trigger)
   unsigned long long* occ_h = nullptr;       // host-mapped [TG_MAX_LAYERS + 1] occupancy reports
+  unsigned long long* size_h = nullptr;      // host-mapped [TG_MAX_LAYERS + 1] live-size reports
+  long long extra_keys = 0;                  // layer-L targets that need not be edge endpoints
+  long long ins_bound[TG_MAX_LAYERS + 1]{};  // sum of S x cap over superbatches since the reset
   long long sb_count = 0;                    // superbatches issued since the last cache reset
   long long targets_issued = 0;              // layer-L targets issued since the last cache reset
   // compute workspace
@@ -114,6 +120,7 @@ struct tg_ctx {
   void* stage = nullptr;
   size_t stage_bytes = 0;
   std::vector<void*> owned;
+  std::vector<void*> owned_host;  // pinned host allocations (TG_OPT_HOST_CACHE rings)
 };
 
 namespace {
@@ -460,8 +467,12 @@ tg_status run_front(tg_ctx* ctx, int S, bool edge_mode, const EdgeSrc& es, int n
   const bool cache_on = ctx->cfg.opts & TG_OPT_CACHE;
   const int use_table = (ctx->cfg.opts & TG_OPT_TTABLE) ? 1 : 0;
   long long* cnt = ctx->cnt_sb;
-  ctx->targets_issued += edge_mode ? 2 * std::min<int64_t>((int64_t)S * es.B, es.n_edges - es.e0)
+  ctx->targets_issued += edge_mode ? (es.neg ? 3 : 2) * std::min<int64_t>((int64_t)S * es.B, es.n_edges - es.e0)
                                    : (long long)S * n_max_top;
+  // keys outside the 2E + 1 edge-endpoint universe: negatives, arbitrary embed targets
+  ctx->extra_keys += edge_mode ? (es.neg ? std::min<int64_t>((int64_t)S * es.B, es.n_edges - es.e0) : 0)
+                               : (long long)S * n_max_top;
+  for (int l = 1; l < L; ++l) ctx->ins_bound[l] += (long long)S * ctx->cap[l];
   // ---- top-down (Alg. 1 l.5-12): dedup, lookup/compaction, sampling
   {
     Prof pf(ctx, TG_ST_DEDUP, st);
@@ -506,6 +517,7 @@ tg_status run_front(tg_ctx* ctx, int S, bool edge_mode, const EdgeSrc& es, int n
           if (b < ctx->idx_bound[l - 1]) ctx->idx_bound[l - 1] = b;
         }
         cd.occ_report = ctx->occ_h ? ctx->occ_h + (l - 1) : nullptr;
+        cd.size_report = ctx->size_h ? ctx->size_h + (l - 1) : nullptr;
         cd.report_sb = ctx->sb_count;
         if (ctx->idx_bound[l - 1] * kIndexRebuildDen > slots * kIndexRebuildNum) {
           Prof pf(ctx, TG_ST_LOOKUP, st);
@@ -562,6 +574,28 @@ tg_status run_front(tg_ctx* ctx, int S, bool edge_mode, const EdgeSrc& es, int n
   return TG_OK;
 }
 
+// Can the next superbatch of S batches be proven eviction-free on the host, without a
+// device sync (then it may use the large S: the grid-wide lookup pass has no S bound)?
+// Upper bounds on the live FIFO size of each cached level at its start: the key universe
+// (with dedup every live item is a distinct key, and every cached key is an edge endpoint
+// <i, t_e>, <0, 0> or an extra target), the inserts issued since the reset, and
+// the latest device report (k_probe_pre) plus the inserts issued after it.
+bool sb_eviction_free(tg_ctx* ctx, int S) {
+  if (!(ctx->cfg.opts & TG_OPT_CACHE)) return true;
+  const long long limit = ctx->cfg.cache_limit;
+  for (int l = 1; l < ctx->L; ++l) {
+    const long long per_sb = (long long)ctx->S * ctx->cap[l];
+    long long b = ctx->ins_bound[l];
+    if (ctx->cfg.opts & TG_OPT_DEDUP) b = std::min(b, 2 * ctx->g.E + 1 + ctx->extra_keys);
+    const unsigned long long rep = ctx->size_h ? *(volatile unsigned long long*)&ctx->size_h[l] : 0ull;
+    const long long sb_obs = (long long)(rep >> 40) - 1;
+    if (sb_obs >= 0 && sb_obs <= ctx->sb_count)
+      b = std::min(b, (long long)(rep & ((1ull << 40) - 1)) + (ctx->sb_count - sb_obs) * per_sb);
+    if (b + (long long)S * ctx->cap[l] > limit) return false;
+  }
+  return true;
+}
+
 // Bottom-up half (Alg. 1 l.13-18): M and FFN, layer by layer over all S batches.
 tg_status run_back(tg_ctx* ctx, cudaStream_t st) {
   for (int l = 1; l <= ctx->L; ++l) TRY(run_layer(ctx, l, st));
@@ -581,8 +615,8 @@ tg_status finish(tg_ctx* ctx, int S, long long* log, int64_t row0, cudaStream_t 
   return launched(ctx);
 }
 
-tg_status stream_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, const uint32_t* ts, int64_t n_edges,
-                       int batch, float* scores, long long* log, cudaStream_t st) {
+tg_status stream_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, const uint32_t* ts, const int32_t* neg,
+                       int64_t n_edges, int batch, float* scores, long long* log, cudaStream_t st) {
   const int64_t nb = (n_edges + batch - 1) / batch;
   // Two-set pipeline: superbatch i's front half runs on ctx->fst into level set
   // i % 2 as soon as superbatch i-2's layers released that set, overlapping the
@@ -592,14 +626,15 @@ tg_status stream_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, cons
   CK(cudaEventRecord(ctx->ev_in, st));
   CK(cudaStreamWaitEvent(ctx->fst, ctx->ev_in, 0));
   int64_t sb = 0;
-  for (int64_t b0 = 0; b0 < nb; b0 += ctx->S, ++sb) {
-    const int S = (int)std::min<int64_t>(ctx->S, nb - b0);
+  for (int64_t b0 = 0, S = 0; b0 < nb; b0 += S, ++sb) {
+    S = std::min<int64_t>(sb_eviction_free(ctx, ctx->S) ? ctx->S : ctx->S_small, nb - b0);
     const int set = (int)(sb & 1);
-    EdgeSrc es{src, dst, ts, n_edges, b0 * batch, batch};
+    EdgeSrc es{src, dst, ts, neg, n_edges, b0 * batch, batch};
+    const int per_edge = neg ? 3 : 2;  // targets per edge: src || dst (|| neg, NEXT-3)
     select_set(ctx, set);
     if (sb >= 2) CK(cudaStreamWaitEvent(ctx->fst, ctx->ev_back[set], 0));
     static const bool one_stream = getenv("TG_ONE_STREAM") != nullptr;  // debug: no overlap
-    TRY(run_front(ctx, S, true, es, 2 * batch, one_stream ? st : ctx->fst));
+    TRY(run_front(ctx, S, true, es, per_edge * batch, one_stream ? st : ctx->fst));
     if (one_stream) CK(cudaEventRecord(ctx->ev_front[set], st));
     CK(cudaEventRecord(ctx->ev_front[set], ctx->fst));
     CK(cudaStreamWaitEvent(st, ctx->ev_front[set], 0));
@@ -621,11 +656,11 @@ tg_status stream_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, cons
       g.C = ctx->sc_z;
       g.ldc = ctx->dnp;
       g.m_dev = ctx->sc_m;
-      g.m_max = S * batch;
+      g.m_max = (neg ? 2 : 1) * S * batch;
       if (ctx->cfg.precision == TG_PREC_BF16) launch_gemm_tc(g, ctx->tcWa1g, TG_PREC_TF32, st);
       else if (ctx->cfg.precision != TG_PREC_FP32) launch_gemm_tc(g, ctx->tcWa1, ctx->cfg.precision, st);
       else launch_gemm_simt(g, st);
-      launch_score_head(ctx->sc_z, ctx->dnp, ctx->sc_oidx, S * batch, ctx->Wa2, ctx->ba2, ctx->d_n, scores, st);
+      launch_score_head(ctx->sc_z, ctx->dnp, ctx->sc_oidx, g.m_max, ctx->Wa2, ctx->ba2, ctx->d_n, scores, st);
     }
     TRY(launched(ctx, 3));
     TRY(finish(ctx, S, log, b0, st));
@@ -639,7 +674,7 @@ tg_status stream_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, cons
 }
 
 struct Staged {
-  const int32_t *src = nullptr, *dst = nullptr;
+  const int32_t *src = nullptr, *dst = nullptr, *neg = nullptr;
   const uint32_t* ts = nullptr;
   float* out = nullptr;
   bool host_out = false;
@@ -774,7 +809,12 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
   const int64_t per_layer = 4LL * D * D + 3LL * D + (int64_t)d_n * (D + d_n) + d_n + (int64_t)d_n * d_n + d_n;
   const int64_t expect = L * per_layer + 2LL * d_t + 2LL * d_n * d_n + d_n + d_n + 1;
   if (n_params != expect) return TG_EINVAL;
-  int S = cfg->superbatch ? cfg->superbatch : 32;
+  static const int s_default = [] {
+    const char* e = getenv("TG_SB_DEFAULT");  // experiments: default superbatch
+    const int v = e ? atoi(e) : 0;
+    return v > 0 && v <= kMaxS ? v : 64;
+  }();
+  int S = cfg->superbatch ? cfg->superbatch : s_default;
   // per-batch capacities: I_L = targets; I_{l-1} = C_l (k+1) <= I_l (k+1)
   int cap[TG_MAX_LAYERS + 1];
   int64_t cc = cfg->max_batch_targets;
@@ -788,17 +828,34 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     if (cap[l] > 16 * 10000) return TG_EINVAL;                   // dedup cluster bound
     if (cap[l] > kSeqCLMax * 1024 * kProbeIPT) return TG_EINVAL; // ordered cache pass bound
   }
-  // every key of a superbatch's cached level must fit the cache passes' DSMEM hash:
-  // worst-case load <= 0.9 (cap assumes every target and neighbour distinct; real
-  // superbatches load it about half as much). S shrinks for large batches (2,000 -> 1).
+  // Superbatches that may evict run the ordered cache pass, whose DSMEM hash must hold
+  // every key of the superbatch's cached level at a worst-case load <= 0.9 (cap assumes
+  // every target and neighbour distinct): S_small (batch 200 / k = 20: 28; batch 2,000: 1).
+  // Superbatches the host proves eviction-free run the grid-wide pass (global-memory
+  // hash) and use S, bounded by the grid-wide pass and a ~40 GB workspace budget.
+  int S_small = S;
   for (int l = 1; l < L; ++l) {
     const int64_t fit = (int64_t)kSeqCLMax * kSeqSlotsPerCTA * 9 / 10 / cap[l];
-    if (fit < S) S = fit < 1 ? 1 : (int)fit;
+    if (fit < S_small) S_small = fit < 1 ? 1 : (int)fit;
+  }
+  {
+    const int64_t HDp_ = (int64_t)H * (round4(d_n) + round4(d_e) + round4(d_t)), Dp_ = HDp_ / H;
+    auto ws = [&](int64_t s) {  // device bytes that grow with S (both level sets)
+      int64_t b = 0, mx = 0;
+      for (int l = 1; l <= L; ++l) {
+        b += 2 * s * cap[l] * (72 + 24 * (int64_t)k);
+        mx = std::max<int64_t>(mx, s * cap[l]);
+        if (l < L) b += s * cap[l] * 4 * 20 + s * cap[l] * 4;  // grid-wide lookup table (2x pow2) + slots
+      }
+      return b + mx * 4 * (2 * HDp_ + 2 * Dp_ + round4(d_n)) + mx * 2 * (HDp_ + Dp_ + 2 * round4(d_n));
+    };
+    while (S > S_small && (ws(S) > (40ll << 30) || (int64_t)cap[1] * S > (int64_t)kSbhMaxBlocks * kSbhChunk)) --S;
   }
   if ((int64_t)cap[1] * S > ((int64_t)1 << 26)) return TG_EINVAL;
   if (cudaSetDevice(ctx->device) != cudaSuccess) return TG_ECUDA;
   ctx->cfg = *cfg;
   ctx->S = S;
+  ctx->S_small = S_small;
   ctx->L = L;
   ctx->H = H;
   ctx->k = k;
@@ -968,7 +1025,8 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
       TRY(tc_prepare_weights(ctx->Wa1, dnp, 2 * dnp, cfg->precision, &ctx->tcWa1, ctx->owned));
       if (cfg->precision == TG_PREC_BF16)
         TRY(tc_prepare_weights(ctx->Wa1, dnp, 2 * dnp, TG_PREC_TF32, &ctx->tcWa1g, ctx->owned));
-    const size_t ne = std::max((size_t)S * ((cfg->max_batch_targets + 1) / 2), (size_t)cfg->max_batch_targets);
+    // score rows of a superbatch: S x batch positive (+ S x batch negative) pairs, batch <= targets / 2
+    const size_t ne = (size_t)S * cfg->max_batch_targets;
     TRY(dalloc(ctx, &ctx->sc_rs, ne));
     TRY(dalloc(ctx, &ctx->sc_rd, ne));
     TRY(dalloc(ctx, &ctx->sc_oidx, ne));
@@ -1025,8 +1083,30 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     while (icap < 4ull * (unsigned long long)(cfg->cache_limit + (long long)S * cap[l])) icap <<= 1;
     TRY(dalloc(ctx, &cd.ikey, icap));
     TRY(dalloc(ctx, &cd.ipos, icap));
-    TRY(dalloc(ctx, &cd.ring, (size_t)rcap * dnp));
+    if (cfg->opts & TG_OPT_HOST_CACHE) {  // NEXT-2: payload ring in pinned, mapped host memory
+      void* hp = nullptr;
+      if (cudaHostAlloc(&hp, (size_t)rcap * dnp * sizeof(float), cudaHostAllocMapped) != cudaSuccess) {
+        cudaGetLastError();
+        return TG_ENOMEM;
+      }
+      ctx->owned_host.push_back(hp);
+      void* dp = nullptr;
+      CK(cudaHostGetDevicePointer(&dp, hp, 0));
+      cd.ring = reinterpret_cast<float*>(dp);
+    } else {
+      TRY(dalloc(ctx, &cd.ring, (size_t)rcap * dnp));
+    }
     TRY(dalloc(ctx, &cd.rkey, (size_t)rcap));
+    {  // grid-wide eviction-free lookup pass: superbatch-scoped hash, >= 2x its entries
+      unsigned long long T = 1024;
+      while (T < 2ull * (unsigned long long)S * cap[l]) T <<= 1;
+      TRY(dalloc(ctx, &cd.sb_key, T));
+      TRY(dalloc(ctx, &cd.sb_val, T));
+      TRY(dalloc(ctx, &cd.sb_slot, T));
+      TRY(dalloc(ctx, &cd.sb_h, (size_t)S * cap[l]));
+      TRY(dalloc(ctx, &cd.sb_blk, kSbhMaxBlocks));
+      cd.sb_mask = T - 1;
+    }
     cd.imask = icap - 1;
     cd.rcap = rcap;
     cd.state = ctx->cache_state + 8 * l;
@@ -1076,7 +1156,9 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
         const long long hrows = l == 1 ? ctx->g.V + 1 : ctx->cache[l - 1].rcap;
         const float* tb = ctx->phi_pre ? ctx->phi_buf[set] : ctx->table;
         const long long trows = ctx->phi_pre ? rows : Wrows;
-        if (attn_make_rows_map(hb, dnp, ctx->g.ldn, hrows, &m.h) == TG_OK &&
+        // host-resident cache rings are read with per-thread loads (CTA attention kernel), not TMA
+        const bool host_rows = l > 1 && (cfg->opts & TG_OPT_HOST_CACHE);
+        if (!host_rows && attn_make_rows_map(hb, dnp, ctx->g.ldn, hrows, &m.h) == TG_OK &&
             attn_make_rows_map(ctx->Ef, ctx->dep, ctx->g.lde, ctx->g.E + 1, &m.e) == TG_OK &&
             attn_make_rows_map(tb, ctx->dtp, ctx->dtp, trows, &m.t) == TG_OK)
           m.valid = 1;
@@ -1100,6 +1182,8 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
   if (!ctx->occ_h) {
     CK(cudaHostAlloc(&ctx->occ_h, (TG_MAX_LAYERS + 1) * sizeof(unsigned long long), cudaHostAllocMapped));
     memset(ctx->occ_h, 0, (TG_MAX_LAYERS + 1) * sizeof(unsigned long long));
+    CK(cudaHostAlloc(&ctx->size_h, (TG_MAX_LAYERS + 1) * sizeof(unsigned long long), cudaHostAllocMapped));
+    memset(ctx->size_h, 0, (TG_MAX_LAYERS + 1) * sizeof(unsigned long long));
   }
   CK(cudaDeviceSynchronize());
   ctx->loaded = true;
@@ -1121,9 +1205,12 @@ tg_status tg_cache_reset(tg_ctx* ctx, int64_t new_limit) {
     CK(cudaMemcpy(cd.state, st, sizeof(st), cudaMemcpyHostToDevice));
     ctx->idx_bound[l] = 0;
     if (ctx->occ_h) ctx->occ_h[l] = 0;
+    if (ctx->size_h) ctx->size_h[l] = 0;
+    ctx->ins_bound[l] = 0;
   }
   ctx->sb_count = 0;
   ctx->targets_issued = 0;
+  ctx->extra_keys = 0;
   CK(cudaMemset(ctx->cnt_total, 0, TG_NCOUNTERS * sizeof(long long)));
   CK(cudaMemset(ctx->cnt_sb, 0, (size_t)kMaxS * TG_NCOUNTERS * sizeof(long long)));
   CK(cudaMemset(ctx->err, 0, 2 * sizeof(int)));
@@ -1169,17 +1256,23 @@ tg_status tg_embed_batch(tg_ctx* ctx, const int32_t* nodes, const uint32_t* ts, 
   return TG_OK;
 }
 
+// Host buffers are staged through the context's device buffer; every array is checked
+// separately (all inputs host or all device: a mix is rejected with TG_EINVAL).
 static tg_status stage_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, const uint32_t* ts,
-                             int64_t n_edges, float* scores, cudaStream_t st, Staged& o) {
+                             const int32_t* neg, int64_t n_edges, float* scores, cudaStream_t st, Staged& o) {
   const bool dev_in = is_device_ptr(src);
+  if (is_device_ptr(dst) != dev_in || is_device_ptr(ts) != dev_in || (neg && is_device_ptr(neg) != dev_in))
+    return TG_EINVAL;
   const bool dev_out = is_device_ptr(scores);
+  const int64_t n_out = (neg ? 2 : 1) * n_edges;
   o.src = src;
   o.dst = dst;
   o.ts = ts;
+  o.neg = neg;
   o.out = scores;
   o.host_out = !dev_out;
   if (dev_in && dev_out) return TG_OK;
-  TRY(ensure_stage(ctx, (size_t)n_edges * 16 + 64));
+  TRY(ensure_stage(ctx, (size_t)n_edges * 16 + (size_t)n_out * 4 + 64));
   char* stg = (char*)ctx->stage;
   if (!dev_in) {  // host -> device copies of this call's inputs (H2D)
     CK(cudaMemcpyAsync(stg, src, n_edges * 4, cudaMemcpyHostToDevice, st));
@@ -1188,8 +1281,12 @@ static tg_status stage_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst
     o.src = (const int32_t*)stg;
     o.dst = (const int32_t*)(stg + n_edges * 4);
     o.ts = (const uint32_t*)(stg + n_edges * 8);
+    if (neg) {
+      CK(cudaMemcpyAsync(stg + n_edges * 12, neg, n_edges * 4, cudaMemcpyHostToDevice, st));
+      o.neg = (const int32_t*)(stg + n_edges * 12);
+    }
   }
-  if (!dev_out) o.out = (float*)(stg + n_edges * 12);
+  if (!dev_out) o.out = (float*)(stg + n_edges * 16);
   return TG_OK;
 }
 
@@ -1204,8 +1301,8 @@ tg_status tg_score_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, co
   cudaStream_t st = (cudaStream_t)cuda_stream;
   CK(cudaSetDevice(ctx->device));
   Staged o;
-  TRY(stage_edges(ctx, src, dst, ts, n_edges, scores, st, o));
-  TRY(stream_edges(ctx, o.src, o.dst, o.ts, n_edges, (int)n_edges, o.out, nullptr, st));
+  TRY(stage_edges(ctx, src, dst, ts, nullptr, n_edges, scores, st, o));
+  TRY(stream_edges(ctx, o.src, o.dst, o.ts, nullptr, n_edges, (int)n_edges, o.out, nullptr, st));
   if (o.host_out) {
     CK(cudaMemcpyAsync(scores, o.out, n_edges * 4, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
@@ -1228,6 +1325,9 @@ tg_status tg_score_pairs(tg_ctx* ctx, const int32_t* nodes, const uint32_t* ts, 
   cudaStream_t st = (cudaStream_t)cuda_stream;
   CK(cudaSetDevice(ctx->device));
   const bool dev_in = is_device_ptr(nodes);
+  // every input array is checked: a host/device mix would make a kernel dereference host memory
+  if (is_device_ptr(ts) != dev_in || (n_pairs > 0 && (is_device_ptr(pair_a) != dev_in || is_device_ptr(pair_b) != dev_in)))
+    return TG_EINVAL;
   const bool dev_out = n_pairs == 0 || is_device_ptr(scores);
   if (!dev_in && n_pairs > 0) {  // host pairs: range-checked here, before any launch
     for (int64_t p = 0; p < n_pairs; ++p)
@@ -1302,10 +1402,32 @@ tg_status tg_score_stream(tg_ctx* ctx, const int32_t* src, const int32_t* dst, c
   cudaStream_t st = (cudaStream_t)cuda_stream;
   CK(cudaSetDevice(ctx->device));
   Staged o;
-  TRY(stage_edges(ctx, src, dst, ts, n_edges, scores, st, o));
-  TRY(stream_edges(ctx, o.src, o.dst, o.ts, n_edges, batch, o.out, (long long*)batch_counters, st));
+  TRY(stage_edges(ctx, src, dst, ts, nullptr, n_edges, scores, st, o));
+  TRY(stream_edges(ctx, o.src, o.dst, o.ts, nullptr, n_edges, batch, o.out, (long long*)batch_counters, st));
   if (o.host_out) {  // device -> host read of the results (D2H)
     CK(cudaMemcpyAsync(scores, o.out, n_edges * 4, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+  }
+  return TG_OK;
+}
+
+tg_status tg_score_stream_neg(tg_ctx* ctx, const int32_t* src, const int32_t* dst, const uint32_t* ts,
+                              const int32_t* neg, int64_t n_edges, int32_t batch, float* scores,
+                              int64_t* batch_counters, void* cuda_stream) {
+  if (!ctx) return TG_EINVAL;
+  if (!ctx->loaded) return TG_ESTATE;
+  if (ctx->broken) return TG_ECUDA;
+  if (n_edges < 0 || batch < 1 || 3 * batch > ctx->cap[ctx->L] ||
+      (n_edges > 0 && (!src || !dst || !ts || !neg || !scores)))
+    return TG_EINVAL;
+  if (n_edges == 0) return TG_OK;
+  cudaStream_t st = (cudaStream_t)cuda_stream;
+  CK(cudaSetDevice(ctx->device));
+  Staged o;
+  TRY(stage_edges(ctx, src, dst, ts, neg, n_edges, scores, st, o));
+  TRY(stream_edges(ctx, o.src, o.dst, o.ts, o.neg, n_edges, batch, o.out, (long long*)batch_counters, st));
+  if (o.host_out) {  // device -> host read of the results (D2H)
+    CK(cudaMemcpyAsync(scores, o.out, 2 * n_edges * 4, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
   }
   return TG_OK;
@@ -1486,11 +1608,13 @@ void tg_free(tg_ctx* ctx) {
     fprintf(stderr, "libtg: index check mismatches %d (err bits %d)\n", e[1], e[0]);
   }
   for (void* p : ctx->owned) cudaFree(p);
+  for (void* p : ctx->owned_host) cudaFreeHost(p);
   for (cudaEvent_t e : ctx->ev_pool) cudaEventDestroy(e);
   for (cudaEvent_t e : {ctx->ev_front[0], ctx->ev_front[1], ctx->ev_back[0], ctx->ev_back[1], ctx->ev_in, ctx->ev_fend})
     if (e) cudaEventDestroy(e);
   if (ctx->fst) cudaStreamDestroy(ctx->fst);
   if (ctx->occ_h) cudaFreeHost(ctx->occ_h);
+  if (ctx->size_h) cudaFreeHost(ctx->size_h);
   if (ctx->stage) cudaFree(ctx->stage);
   delete ctx;
 }

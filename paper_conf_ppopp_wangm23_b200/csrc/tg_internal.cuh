@@ -131,8 +131,20 @@ struct CacheDev {
   // host-mapped report word: ((superbatch + 1) << 40) | occupied slots, written by
   // k_probe_pre, read by the host without synchronising (rebuild trigger bound)
   unsigned long long* occ_report;
+  unsigned long long* size_report;  // same format: live FIFO size at superbatch start
   long long report_sb;       // superbatch number of this launch (set per launch)
+  // superbatch-scoped lookup hash in global memory (L2-resident), grid-wide eviction-free
+  // CacheLookup pass (k_sbh_*): key -> min concatenated position j, then the ring slot of
+  // the key's first occurrence. T = sb_mask + 1 >= 2 x (S x cap) slots.
+  unsigned long long* sb_key;  // [T]
+  unsigned* sb_val;            // [T] min j
+  long long* sb_slot;          // [T] ring slot of the first occurrence
+  int* sb_h;                   // [S x cap] table slot of each unique-list entry
+  int* sb_blk;                 // [kSbhMaxBlocks] misses per scan block
+  unsigned long long sb_mask;
 };
+constexpr int kSbhItems = 8, kSbhThreads = 1024, kSbhChunk = kSbhItems * kSbhThreads;
+constexpr int kSbhMaxBlocks = 1024;  // S x cap <= 8.4M entries per cached level
 // Index maintenance: the index never deletes, so FIFO churn (small limits) fills it with
 // dead keys and absent-key probes lengthen; when more than half of the slots are occupied
 // the index is rebuilt from the live ring window (clear, then re-insert keys of positions
@@ -185,6 +197,7 @@ struct EdgeSrc {            // batch b of the superbatch = edges [e0 + b*B, +B) 
   const int32_t* src;
   const int32_t* dst;
   const uint32_t* ts;
+  const int32_t* neg;       // optional negative destinations (NEXT-3): targets src || dst || neg
   int64_t n_edges;
   int64_t e0;
   int B;

@@ -13,7 +13,7 @@ import numpy as np
 _PKG = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("TG_LIB") or os.path.join(_PKG, "libtg.so")
 
-TG_OPT_DEDUP, TG_OPT_CACHE, TG_OPT_TTABLE, TG_OPT_ALL = 1, 2, 4, 7
+TG_OPT_DEDUP, TG_OPT_CACHE, TG_OPT_TTABLE, TG_OPT_ALL, TG_OPT_HOST_CACHE = 1, 2, 4, 7, 8
 TG_PREC_FP32, TG_PREC_TF32X3, TG_PREC_BF16, TG_PREC_TF32, TG_PREC_F16X3 = 0, 1, 2, 3, 4
 TG_MAX_LAYERS = 4
 TG_CNT_PER_LAYER = 6
@@ -23,6 +23,7 @@ TG_NCOUNTERS = TG_CNT_TDIRECT + 1
 COUNTER_FIELDS = ("n", "unique", "lookups", "hits", "misses", "evicted")
 
 EXPORTS = ("tg_graph_load", "tg_model_load", "tg_embed_batch", "tg_score_edges", "tg_score_stream",
+           "tg_score_stream_neg",
            "tg_score_pairs", "tg_cache_reset", "tg_counters_read", "tg_dedup", "tg_sample", "tg_time_encode",
            "tg_kernel_launches", "tg_free", "tg_strerror", "tg_version", "tg_profile_enable",
            "tg_profile_read", "tg_gemm", "tg_superbatch")
@@ -64,6 +65,7 @@ def lib():
         L.tg_embed_batch.argtypes = [vp, vp, vp, i64, vp, vp]
         L.tg_score_edges.argtypes = [vp, vp, vp, vp, i64, vp, vp]
         L.tg_score_stream.argtypes = [vp, vp, vp, vp, i64, i32, vp, vp, vp]
+        L.tg_score_stream_neg.argtypes = [vp, vp, vp, vp, vp, i64, i32, vp, vp, vp]
         L.tg_score_pairs.argtypes = [vp, vp, vp, i64, vp, vp, i64, vp, vp]
         L.tg_cache_reset.argtypes = [vp, i64]
         L.tg_counters_read.argtypes = [vp, vp, i32]
@@ -174,6 +176,13 @@ class Context:
     def score_stream(self, src, dst, ts, batch, scores, batch_counters=None, stream=None):
         _check(lib().tg_score_stream(self.h, _ptr(src), _ptr(dst), _ptr(ts), int(src.shape[0]), int(batch),
                                      _ptr(scores), _ptr(batch_counters), _stream(stream)), "tg_score_stream")
+        return scores
+
+    def score_stream_neg(self, src, dst, ts, neg, batch, scores, batch_counters=None, stream=None):
+        """scores[:E] = positive (src, dst) pairs, scores[E:] = (src, neg) pairs (NEXT-3)."""
+        _check(lib().tg_score_stream_neg(self.h, _ptr(src), _ptr(dst), _ptr(ts), _ptr(neg), int(src.shape[0]),
+                                         int(batch), _ptr(scores), _ptr(batch_counters), _stream(stream)),
+               "tg_score_stream_neg")
         return scores
 
     def cache_reset(self, new_limit=-1):

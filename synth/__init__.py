@@ -7,5 +7,5 @@ workloads (Table 2) and BASELINE.json's configs.
 Both `oracle/` and the product path consume its outputs; it imports neither.
 """
 from .configs import CONFIGS, StreamConfig, ModelConfig, get_config  # noqa: F401
-from .streams import make_stream, Stream  # noqa: F401
+from .streams import make_stream, negatives, Stream  # noqa: F401
 from .params import make_params, param_count  # noqa: F401

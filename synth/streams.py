@@ -131,3 +131,12 @@ def make_stream(cfg, n_edges: int = None, with_features: bool = True) -> Stream:
 def batches(n_edges: int, batch: int):
     """Chronological batch boundaries [(lo, hi)], the last one partial (R13)."""
     return [(lo, min(lo + batch, n_edges)) for lo in range(0, n_edges, batch)]
+
+
+def negatives(s: Stream, seed: int = 0) -> np.ndarray:
+    """Seeded negative destinations for link-prediction evaluation (NEXT-3, the TGAT protocol
+    the paper's task follows): for every edge, a node drawn uniformly from the set of
+    destination nodes of the stream. An input of the evaluation, not part of the method."""
+    rng = np.random.Generator(np.random.PCG64(1_000_033 + seed))
+    pool = np.unique(s.dst)
+    return pool[rng.integers(0, pool.size, size=s.n_edges)].astype(np.int32)

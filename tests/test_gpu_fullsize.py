@@ -222,3 +222,74 @@ def test_batch_range_shards_equal_single_context(name, world, prec):
         ctx.close()
     assert np.array_equal(np.concatenate(parts), ref)
     assert tot is not None and tot.sum() > 0
+
+
+def _run_neg(ctx, s, neg, batch, E=None):
+    from paper_conf_ppopp_wangm23_b200 import TG_NCOUNTERS
+    E = s.n_edges if E is None else E
+    nb = (E + batch - 1) // batch
+    d = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    scores = torch.full((2 * E,), -1.0, dtype=torch.float32, device="cuda")
+    log = torch.zeros(nb * TG_NCOUNTERS, dtype=torch.int64, device="cuda")
+    ctx.score_stream_neg(d(s.src[:E]), d(s.dst[:E]), d(s.ts[:E].view(np.int32)), d(neg[:E]), batch, scores, log)
+    torch.cuda.synchronize()
+    sc = scores.cpu().numpy()
+    return sc[:E], sc[E:], log.cpu().numpy().reshape(nb, TG_NCOUNTERS)
+
+
+def _oracle_neg(o, s, neg, lo, hi):
+    B = hi - lo
+    t = s.ts[lo:hi]
+    H = o.embed(o.m.L, np.r_[s.src[lo:hi], s.dst[lo:hi], neg[lo:hi]], np.r_[t, t, t])
+    return o.score(H[:B], H[B:2 * B]), o.score(H[:B], H[2 * B:])
+
+
+@pytest.mark.parametrize("name,prec,E", [("config1", 1, None), ("config1", 2, None), ("reddit", 1, None)])
+def test_stream_negatives_parity_ap_auc(name, prec, E):
+    """NEXT-3 (TGAT [37]): link prediction with seeded negatives through the superbatched
+    stream path (tg_score_stream_neg): every batch's target list is src || dst || neg (3B targets,
+    one dedup). Positive and negative scores of stratified batches match the plain oracle (R17 /
+    R22), every batch's counters equal the Alg. 1/3 simulator fed the same 3B targets, scores are
+    bit-identical at S = 1 and the default S, and AP / AUC over the sampled batches equal the
+    oracle's (the random-weight model ranks near chance: this pins the evaluation path, not a
+    trained model)."""
+    from sklearn.metrics import average_precision_score, roc_auc_score
+    from synth import negatives
+    from oracle.tgopt import TGOptSim
+    from paper_conf_ppopp_wangm23_b200 import counters_dict
+    cfg, s, flat = setup(name)
+    mc = cfg.model
+    neg = negatives(s, seed=1)
+    ctx = make_ctx(s, flat, mc, precision=prec, max_targets=3 * mc.batch)
+    pos, ngs, log = _run_neg(ctx, s, neg, mc.batch)
+    assert ctx.superbatch() > 1
+    ctx.close()
+    o = make_oracle(s, flat, mc)
+    nb = log.shape[0]
+    picks = _picks(nb)
+    gp, gn, rp, rn = [], [], [], []
+    for b in picks:
+        lo, hi = b * mc.batch, min((b + 1) * mc.batch, s.n_edges)
+        p_ref, n_ref = _oracle_neg(o, s, neg, lo, hi)
+        for got, ref in ((pos[lo:hi], p_ref), (ngs[lo:hi], n_ref)):
+            ok, err, nbad = close(got, ref, *TOL[prec])
+            assert ok, (b, err, nbad)
+        gp.append(pos[lo:hi]); gn.append(ngs[lo:hi]); rp.append(p_ref); rn.append(n_ref)
+    y = np.r_[np.ones(sum(map(len, gp))), np.zeros(sum(map(len, gn)))]
+    g_all, r_all = np.r_[np.concatenate(gp), np.concatenate(gn)], np.r_[np.concatenate(rp), np.concatenate(rn)]
+    assert abs(average_precision_score(y, g_all) - average_precision_score(y, r_all)) <= 2e-3
+    assert abs(roc_auc_score(y, g_all) - roc_auc_score(y, r_all)) <= 2e-3
+    sim = TGOptSim(o, cache_limit=mc.cache_limit, time_window=mc.time_window, compute=False)
+    check = range(nb) if name == "config1" else range(0, nb, max(1, nb // 200))
+    for b in range(nb):
+        lo, hi = b * mc.batch, min((b + 1) * mc.batch, s.n_edges)
+        t = s.ts[lo:hi]
+        sim.reset_counters()
+        sim.embed(mc.n_layers, np.r_[s.src[lo:hi], s.dst[lo:hi], neg[lo:hi]], np.r_[t, t, t])
+        if b in check:
+            assert counters_dict(log[b], mc.n_layers) == sim.counters(), b
+    if name == "config1":
+        one = make_ctx(s, flat, mc, precision=prec, max_targets=3 * mc.batch, superbatch=1)
+        pos1, ngs1, _ = _run_neg(one, s, neg, mc.batch)
+        one.close()
+        assert np.array_equal(pos1, pos) and np.array_equal(ngs1, ngs)

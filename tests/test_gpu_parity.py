@@ -438,3 +438,33 @@ def test_f16x3_range_violation_is_loud():
     torch.cuda.synchronize()
     with pytest.raises(TGError):
         ctx.counters_raw()
+
+
+@pytest.mark.parametrize("name,limit,prec", [("config1", 2_000_000, 1), ("config1", 700, 1), ("tiny_bip", 25, 0)])
+def test_host_resident_cache_matches_device_cache(name, limit, prec):
+    """NEXT-2 (Table 5): with TG_OPT_HOST_CACHE the FIFO payload rings live in pinned
+    host memory (index in HBM). Storage location is semantic-preserving: every batch's counters
+    are identical to the device cache's, scores match the device-cache run and the oracle."""
+    from paper_conf_ppopp_wangm23_b200 import TG_NCOUNTERS, TG_OPT_ALL, TG_OPT_HOST_CACHE
+    cfg, s, flat = setup(name)
+    mc = cfg.model
+    o = make_oracle(s, flat, mc)
+    out = {}
+    for opts in (TG_OPT_ALL, TG_OPT_ALL | TG_OPT_HOST_CACHE):
+        ctx = make_ctx(s, flat, mc, precision=prec, opts=opts, cache_limit=limit)
+        nb = (s.n_edges + mc.batch - 1) // mc.batch
+        sc = torch.zeros(s.n_edges, dtype=torch.float32, device="cuda")
+        log = torch.zeros(nb * TG_NCOUNTERS, dtype=torch.int64, device="cuda")
+        ctx.score_stream(dev(s.src), dev(s.dst), dev(s.ts.view(np.int32)), mc.batch, sc, log)
+        torch.cuda.synchronize()
+        out[opts] = (sc.cpu().numpy(), log.cpu().numpy())
+        ctx.counters_raw()                      # no sticky device error
+        ctx.close()
+    (a, la), (b, lb) = out[TG_OPT_ALL], out[TG_OPT_ALL | TG_OPT_HOST_CACHE]
+    assert np.array_equal(la, lb)
+    assert np.allclose(a, b, rtol=1e-5, atol=1e-6)
+    for bi in (0, nb // 2, nb - 1):
+        lo, hi = bi * mc.batch, min((bi + 1) * mc.batch, s.n_edges)
+        _, ref = o.infer_batch(s.src[lo:hi], s.dst[lo:hi], s.ts[lo:hi])
+        ok, err, nbad = close(b[lo:hi], ref, *SCORE_TOL[prec])
+        assert ok, (bi, err, nbad)

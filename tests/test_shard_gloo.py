@@ -104,3 +104,19 @@ def test_gloo_world2_gathers_match_sequential_shards():
     for lo in range(0, s.n_edges, mc.batch):
         single.infer_batch(s.src[lo:lo + mc.batch], s.dst[lo:lo + mc.batch], s.ts[lo:lo + mc.batch])
     assert total[keys.index("l1_misses")] >= single.counters()["l1_misses"]
+
+
+def test_bench_spawns_one_rank_per_gpu():
+    """bench.py --gpus N without a torchrun environment re-executes itself through
+    torch.distributed.run with N local ranks (127.0.0.1); under torchrun WORLD_SIZE must
+    equal --gpus (--gpus used to be ignored)."""
+    import bench
+    cmd = bench.spawn_cmd(["--gpus", "4", "--steps", "2"], 4, 29555)
+    assert cmd[1:3] == ["-m", "torch.distributed.run"]
+    assert "--nproc-per-node=4" in cmd and "--master-addr=127.0.0.1" in cmd and "--master-port=29555" in cmd
+    assert cmd[-3:] == ["--gpus", "4", "--steps", "2"][-3:] and cmd[cmd.index("--master-port=29555") + 1].endswith("bench.py")
+    assert bench.check_world("0", 1) == 1 and bench.check_world("8", 8) == 8
+    with pytest.raises(SystemExit):
+        bench.check_world("2", 8)
+    with pytest.raises(SystemExit):
+        bench.check_world("0", 2)

@@ -11,7 +11,8 @@ import torch
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from synth import make_stream, make_params, get_config  # noqa: E402
-from paper_conf_ppopp_wangm23_b200 import Context, TG_PREC_FP32, TG_PREC_TF32X3, TG_PREC_BF16, TG_PREC_TF32  # noqa: E402
+from paper_conf_ppopp_wangm23_b200 import (Context, TG_PREC_FP32, TG_PREC_TF32X3, TG_PREC_BF16, TG_PREC_TF32,  # noqa: E402
+                                          TG_PREC_F16X3)
 
 ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="reddit")
@@ -23,7 +24,8 @@ cfg = get_config(a.config)
 mc = cfg.model
 s = make_stream(a.config, n_edges=a.edges)
 flat = make_params(mc.n_layers, mc.n_heads, s.d_n, s.d_e)
-prec = {"fp32": TG_PREC_FP32, "tf32x3": TG_PREC_TF32X3, "bf16": TG_PREC_BF16, "tf32": TG_PREC_TF32}[a.precision]
+prec = {"fp32": TG_PREC_FP32, "tf32x3": TG_PREC_TF32X3, "bf16": TG_PREC_BF16, "tf32": TG_PREC_TF32,
+        "f16x3": TG_PREC_F16X3}[a.precision]
 ctx = Context.from_stream(s).load_model(flat, n_layers=mc.n_layers, n_heads=mc.n_heads, n_neighbors=mc.n_neighbors,
                                         max_batch_targets=2 * mc.batch, cache_limit=mc.cache_limit,
                                         time_window=mc.time_window, precision=prec, superbatch=a.superbatch)
