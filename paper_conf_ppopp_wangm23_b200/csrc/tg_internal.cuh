@@ -27,7 +27,7 @@ namespace tg {
 constexpr unsigned long long kEmptyKey = 0xFFFFFFFFFFFFFFFFull;
 constexpr unsigned long long kLockedKey = 0xFFFFFFFFFFFFFFFEull;
 constexpr int kMaxK = 32;          // neighbours per target (warp lanes)
-constexpr int kMaxS = 64;          // batches per superbatch
+constexpr int kMaxS = 128;         // batches per superbatch
 constexpr int kDedupThreads = 1024;
 constexpr int kDedupIPT = 16;      // items per thread per CTA (ordered scan)
 constexpr int kDedupSlots = 16384; // smem hash slots per CTA (load <= ~0.6)
