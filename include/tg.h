@@ -106,14 +106,16 @@ typedef struct {
   int32_t time_window;        /* W of the precomputed Phi table (10,000)     */
   uint32_t opts;              /* TG_OPT_* bits                                        */
   int32_t precision;          /* TG_PREC_*                                            */
-  int32_t superbatch;         /* S: batches per launch sequence in tg_score_stream (0 = 32,
-                               * 1 = one batch at a time). Semantics per batch are unchanged:
-                               * dedup scope, cache lookups and FIFO inserts stay per batch
-                               * and in batch order, so outputs and counters do not depend on S.
-                               * S is lowered so that S x (per-batch capacity of each cached
-                               * level) fits the cache passes' DSMEM hash at a worst-case load
-                               * <= 0.9 (235,929 keys): batch 200, k = 20 runs S <= 28; batch
-                               * 2,000 runs S = 1. tg_superbatch() returns the S in use. */
+  int32_t superbatch;         /* S: batches per launch sequence in tg_score_stream (0 = 64,
+                               * 1 = one batch at a time, <= 128). Semantics per batch are
+                               * unchanged: dedup scope, cache lookups and FIFO inserts stay per
+                               * batch and in batch order, so outputs and counters do not depend
+                               * on S. Superbatches the host proves eviction-free (FIFO size bound
+                               * + S x capacity <= limit) run the grid-wide lookup pass with this S
+                               * (bounded by a ~40 GB workspace budget); superbatches that may
+                               * evict run the ordered pass with S_small, the largest S whose keys
+                               * fit its cluster DSMEM hash at a worst-case load <= 0.9 (batch 200,
+                               * k = 20: 28; batch 2,000: 1). tg_superbatch() returns S. */
 } tg_model_cfg;
 
 /* params: host float32 [n_params] in this order (row-major, Linear = [out x in]),

@@ -76,9 +76,13 @@ static inline void tc_plan(int prec, int BN, int ln, bool generic, int* stages, 
   const size_t st = (size_t)tc_planes(prec) * ((size_t)TC_BM * 128 + (size_t)BN * 128);
   const size_t budget = (tc_ctas_per_sm(prec) == 1 ? 205 * 1024 : 100 * 1024) - (ln ? TC_LN_BYTES : 0);
   int d = 0;  // 0: no room beside 2 stages -> the producers load synchronously
+  static const int d_env = [] {  // TG_GEMM_STG: cap on staging units (A/B experiments)
+    const char* e = getenv("TG_GEMM_STG");
+    return e ? atoi(e) : 4;
+  }();
   if (generic) {
     d = budget > 2 * st ? (int)((budget - 2 * st) / TC_STG_UNIT) : 0;
-    d = d > 4 ? 4 : d;
+    d = d > d_env ? d_env : d;
   }
   int s = (int)((budget - (size_t)d * TC_STG_UNIT) / st);
   if (s > TC_MAXSTAGES) s = TC_MAXSTAGES;

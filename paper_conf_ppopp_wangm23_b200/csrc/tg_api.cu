@@ -1140,7 +1140,11 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
       rows += (long long)ctx->lvs[0][l].c_cap * k;
     }
     const size_t bytes = (size_t)rows * ctx->dtp * sizeof(float);
-    ctx->phi_pre = 2 * bytes <= (16ull << 30) && rows < (1ll << 31);
+    static const bool phi_pre_env = [] {  // TG_PHI_PRE=0: Phi of dt >= W inside the attention (A/B)
+      const char* e = getenv("TG_PHI_PRE");
+      return !(e && e[0] == '0');
+    }();
+    ctx->phi_pre = phi_pre_env && 2 * bytes <= (16ull << 30) && rows < (1ll << 31);
     if (ctx->phi_pre)
       for (int set = 0; set < 2; ++set) {
         TRY(dalloc(ctx, &ctx->phi_buf[set], (size_t)rows * ctx->dtp));

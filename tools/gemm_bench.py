@@ -19,13 +19,14 @@ from paper_conf_ppopp_wangm23_b200 import Context  # noqa: E402
 ap = argparse.ArgumentParser()
 ap.add_argument("--m", type=int, default=6400)
 ap.add_argument("--reps", type=int, default=10)
+ap.add_argument("--precs", default="0,1,3,2,4")
 a = ap.parse_args()
 cfg = get_config("tiny")
 s = make_stream("tiny")
 ctx = Context.from_stream(s).load_model(make_params(2, 2, s.d_n, s.d_e), n_neighbors=3, max_batch_targets=16,
                                         cache_limit=100, time_window=10)
 shapes = [(1032, 172), (516, 1032), (172, 688), (172, 172)]
-for prec, name in [(0, "fp32"), (1, "tf32x3"), (3, "tf32"), (2, "bf16")]:
+for prec, name in [(p, {0: "fp32", 1: "tf32x3", 2: "bf16", 3: "tf32", 4: "f16x3"}[p]) for p in map(int, a.precs.split(","))]:
     for N, K in shapes:
         A = torch.randn(a.m, K, device="cuda")
         B = torch.randn(N, K, device="cuda") / K ** 0.5

@@ -19,7 +19,7 @@ sys.path.insert(0, ROOT)
 import numpy as np  # noqa: E402
 import torch  # noqa: E402
 from synth import make_stream, make_params, get_config  # noqa: E402
-from paper_conf_ppopp_wangm23_b200 import Context, TG_PREC_BF16, TG_PREC_TF32, TG_PREC_TF32X3  # noqa: E402
+from paper_conf_ppopp_wangm23_b200 import Context, TG_PREC_BF16, TG_PREC_TF32, TG_PREC_TF32X3, TG_PREC_F16X3  # noqa: E402
 from paper_conf_ppopp_wangm23_b200.tg import lib  # noqa: E402
 
 ap = argparse.ArgumentParser()
@@ -34,7 +34,7 @@ cfg = get_config("reddit")
 mc = cfg.model
 s = make_stream("reddit", n_edges=a.edges)
 flat = make_params(mc.n_layers, mc.n_heads, s.d_n, s.d_e)
-prec = {"bf16": TG_PREC_BF16, "tf32": TG_PREC_TF32, "tf32x3": TG_PREC_TF32X3}[a.precision]
+prec = {"bf16": TG_PREC_BF16, "tf32": TG_PREC_TF32, "tf32x3": TG_PREC_TF32X3, "f16x3": TG_PREC_F16X3}[a.precision]
 ctx = Context.from_stream(s).load_model(flat, n_layers=mc.n_layers, n_heads=mc.n_heads, n_neighbors=mc.n_neighbors,
                                         max_batch_targets=2 * mc.batch, cache_limit=mc.cache_limit,
                                         time_window=mc.time_window, precision=prec)

@@ -28,16 +28,19 @@ def main():
     peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
     hbm = peaks["hbm_gbs"]
     rows = []
-    gemm_names = ["G1", "G2", "G3", "G4"]
-    gi = 0
+    # GEMM role from its predecessor in the layer chain: G1 precedes the
+    # attention, G2 follows it, G3 follows the LayerNorm, G4 follows G3, score follows k_score_rows
+    prev_role = {"k_attn_g": "G2", "k_attn": "G2", "k_layernorm": "G3", "G3": "G4", "k_score_rows": "score"}
+    prev = ""
     for lid, d in sorted(summarise(a.rep).items(), key=lambda kv: int(kv[0])):
         name = re.sub(r"\(.*", "", d["kernel"]).replace("void ", "").replace("tg::", "").strip()
-        if name.startswith("k_gemm_tc") or name.startswith("k_gemm_simt"):
-            grid = d.get("grid", 0)
-            label = gemm_names[gi % 4] if grid == 148 else "score"
-            if grid == 148:
-                gi += 1
-            name = f"{name} {label}"
+        base = re.sub(r"<.*", "", name)
+        if base in ("k_gemm_tc", "k_gemm_simt"):
+            role = prev_role.get(prev, "G1")
+            name = f"{name} {role}"
+            prev = role
+        else:
+            prev = base
         dur = d.get("dur_us", 0.0)
         rb, wb = d.get("dram__bytes_read.sum", 0.0), d.get("dram__bytes_write.sum", 0.0)
         gbs = (rb + wb) / (dur * 1e-6) / 1e9 if dur else 0.0

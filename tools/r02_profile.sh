@@ -1,0 +1,7 @@
+# per-kernel evidence for profiles/: launch list of a whole pass + ncu --set full of one superbatch
+out=gpurun_out/$1; prec=${2:-tf32x3}; mkdir -p $out
+python -c "import __graft_entry__ as g; g.build()" > $out/build.log 2>&1 || { tail $out/build.log; exit 1; }
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $out/launches_$prec.csv python tools/profile_run.py --precision $prec > /dev/null 2>&1
+python tools/sb_launches.py $out/launches_$prec.csv > $out/sb_$prec.txt 2>&1; tail -25 $out/sb_$prec.txt
+timeout 1500 ncu --set full --clock-control none --import-source on -s 700 -c 40 -o $out/sb_full_$prec python tools/profile_run.py --precision $prec > $out/full_$prec.log 2>&1; echo "full rc=$?"
+python tools/kernel_table.py $out/sb_full_$prec.ncu-rep --out $out/kernels_$prec --tag $prec 2>&1 | tail -45; python tools/ncu_summary.py $out/sb_full_$prec.ncu-rep --json $out/sb_full_$prec.summary.json > /dev/null; gzip -f $out/launches_$prec.csv; rm -f $out/sb_full_$prec.ncu-rep
