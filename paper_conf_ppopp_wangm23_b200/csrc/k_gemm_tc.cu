@@ -38,8 +38,13 @@
 namespace tg {
 
 constexpr int TC_BM = 128;
-constexpr int TC_WARPS = 14;
-constexpr int TC_EPI_WARPS = 8;
+// warp roles: [0, 8) A producers, 8 TMA (B and dense A tiles), 9 MMA issuer, [10, 14)
+// epilogue (one per TMEM lane quadrant: warp w may only access lanes 32 (w % 4) .. + 31)
+constexpr int TC_PROD_WARPS = 8;
+constexpr int TC_EPI_WARPS = 4;
+constexpr int TC_EPI_HALVES = TC_EPI_WARPS / 4;  // epilogue warps per lane quadrant (column split)
+constexpr int TC_TMA_WARP = TC_PROD_WARPS, TC_MMA_WARP = TC_PROD_WARPS + 1, TC_EPI_WARP0 = TC_PROD_WARPS + 2;
+constexpr int TC_WARPS = TC_PROD_WARPS + 2 + TC_EPI_WARPS;
 constexpr int TC_THREADS = TC_WARPS * 32;
 constexpr int TC_MAXSTAGES = 8;
 // TMEM: two accumulator buffers of 256 columns (all 512 columns; one CTA per
@@ -72,9 +77,12 @@ constexpr int TC_LN_BYTES = (2 * 128 + 2 * TC_LN_MAXTN * 128) * 16 + 4 * 256 * 4
 // `stg` staging units of 16 KB (its cp.async look-ahead ring, up to 4 units) -- as many
 // staging units as fit beside 2 stages, then as many stages as fit beside those.
 constexpr int TC_STG_UNIT = TC_BM * 128;
+constexpr int TC_PTR_BYTES = 2 * TC_BM * 8;  // the producers' row-pointer table
+static inline bool tc_atmem(int prec) { return tc_planes(prec) == 2; }  // A operand in TMEM
 static inline void tc_plan(int prec, int BN, int ln, bool generic, int* stages, int* stg) {
-  const size_t st = (size_t)tc_planes(prec) * ((size_t)TC_BM * 128 + (size_t)BN * 128);
-  const size_t budget = (tc_ctas_per_sm(prec) == 1 ? 205 * 1024 : 100 * 1024) - (ln ? TC_LN_BYTES : 0);
+  const size_t st = (size_t)tc_planes(prec) * ((tc_atmem(prec) ? 0 : (size_t)TC_BM * 128) + (size_t)BN * 128);
+  const size_t budget = (tc_ctas_per_sm(prec) == 1 ? 205 * 1024 : 100 * 1024) - (ln ? TC_LN_BYTES : 0) -
+                        (generic ? TC_PTR_BYTES : 0);
   int d = 0;  // 0: no room beside 2 stages -> the producers load synchronously
   static const int d_env = [] {  // TG_GEMM_STG: cap on staging units (A/B experiments)
     const char* e = getenv("TG_GEMM_STG");
@@ -86,6 +94,11 @@ static inline void tc_plan(int prec, int BN, int ln, bool generic, int* stages, 
   }
   int s = (int)((budget - (size_t)d * TC_STG_UNIT) / st);
   if (s > TC_MAXSTAGES) s = TC_MAXSTAGES;
+  if (tc_atmem(prec)) {  // TMEM: one [big | small] accumulator + 64 columns of A per stage
+    const int acc = 2 * ((BN + 31) & ~31);
+    const int sa = (512 - acc) / 64;
+    if (s > sa) s = sa;
+  }
   *stages = s < 2 ? 2 : s;
   *stg = d;
 }
@@ -121,11 +134,13 @@ tg_status tc_prepare_weights(const float* W, int N, int K, int precision, TcWeig
   int ntn = (N > 256 && tc_acc_cols(precision) == 256) ? (N + 255) / 256 : (N + 127) / 128;
   // tf32x3 keeps a [big | small] accumulator pair per buffer: N tiles <= 128 keep the
   // epilogue double-buffered (4 x 128 TMEM columns); wider tiles run single-buffered
+  // fp32-level modes keep A in TMEM beside a [big | small] accumulator pair: wide N tiles are
+  // capped at 192 columns so that >= 2 A stages (64 columns each) fit in the 512 TMEM columns
   static const int x3_bn = [] {
     const char* e = getenv("TG_X3_BN");
-    return e ? atoi(e) : 256;
+    return e ? atoi(e) : 192;
   }();
-  if ((precision == TG_PREC_TF32X3 || precision == TG_PREC_F16X3) && x3_bn > 0 && x3_bn < 256)
+  if ((precision == TG_PREC_TF32X3 || precision == TG_PREC_F16X3) && x3_bn > 0 && x3_bn < 256 && N > 256)
     ntn = (N + x3_bn - 1) / x3_bn;
   int BN = (N + ntn - 1) / ntn;
   BN = (BN + 15) & ~15;
@@ -260,6 +275,36 @@ __device__ __forceinline__ void mma_issue(uint32_t tmem, uint64_t da, uint64_t d
   }
 }
 
+// A operand in tensor memory (M = 128 lanes = rows; kind::tf32: one element per 32-bit column,
+// kind::f16: two per column): the MMA reads only B from shared memory
+template <int PREC>
+__device__ __forceinline__ void mma_issue_ts(uint32_t tmem, uint32_t atmem, uint64_t db, uint32_t idesc, uint32_t acc) {
+  if (PREC == TG_PREC_F16X3) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n\t}\n" ::"r"(tmem),
+        "r"(atmem), "l"(db), "r"(idesc), "r"(acc));
+  } else {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::tf32 [%0], [%1], %2, %3, p;\n\t}\n" ::"r"(tmem),
+        "r"(atmem), "l"(db), "r"(idesc), "r"(acc));
+  }
+}
+__device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t (&v)[16]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};\n" ::"r"(
+          taddr),
+      "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]), "r"(v[8]), "r"(v[9]),
+      "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15])
+      : "memory");
+}
+__device__ __forceinline__ void tmem_st8(uint32_t taddr, const uint32_t (&v)[8]) {
+  asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};\n" ::"r"(taddr), "r"(v[0]),
+               "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7])
+               : "memory");
+}
+
 __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(smem_u32(bar)), "r"(count));
 }
@@ -345,6 +390,12 @@ __device__ __forceinline__ float rna_tf32(float x) {
   asm("cvt.rna.tf32.f32 %0, %1;\n" : "=r"(r) : "f"(x));
   return __uint_as_float(r);
 }
+// The same rounding (nearest, ties away from zero, on the 13 dropped mantissa bits) with two
+// full-rate integer ops instead of the conversion pipe -- the A producers' hot loop
+// (bit-identical to cvt.rna.tf32.f32 for finite x; a NaN may come out as Inf)
+__device__ __forceinline__ float rna_tf32_fast(float x) {
+  return __uint_as_float((__float_as_uint(x) + 0x1000u) & 0xffffe000u);
+}
 
 __device__ __forceinline__ float4 tc_load4(const GemmArgs& g, const float* r0, const float* r1, int col) {
   if (col >= g.K) return make_float4(0.f, 0.f, 0.f, 0.f);
@@ -382,6 +433,9 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
               const __grid_constant__ CUtensorMap tmA2, int a2_kb0, int a2_x0) {
   constexpr int EPC = (PREC == TG_PREC_BF16 || PREC == TG_PREC_F16X3) ? 64 : 32;
   constexpr int PLANES = (PREC == TG_PREC_TF32X3 || PREC == TG_PREC_F16X3) ? 2 : 1;
+  // fp32-level modes: the converted A operand goes to tensor memory (32 columns per plane and
+  // k-block: tf32 one element, f16 two per column), shared-memory stages hold only B
+  constexpr bool ATMEM = PLANES == 2;
   extern __shared__ __align__(1024) unsigned char smem_raw[];
   // 1024-byte alignment (128B swizzle atoms) by an integer offset from smem_raw, so
   // the compiler keeps the shared address space (LDS/STS, not generic LD/ST)
@@ -396,10 +450,12 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   const int BNc = (BN + 31) & ~31;
   const uint32_t buf_cols = PLANES == 2 ? 2u * BNc : (uint32_t)tc_acc_cols(PREC);
   const uint32_t small_off = PLANES == 2 ? (uint32_t)BNc : 0u;
-  const uint32_t nbuf = (PLANES == 2 && 4 * BNc > 512) ? 1u : 2u;
+  const uint32_t nbuf = (ATMEM || 4 * BNc > 512) ? 1u : 2u;
   const uint32_t a_plane = TC_BM * 128;
   const uint32_t b_plane = (uint32_t)BN * 128;
-  const uint32_t stage_bytes = PLANES * (a_plane + b_plane);
+  const uint32_t a_bytes = ATMEM ? 0u : PLANES * a_plane;  // A bytes at the head of a smem stage
+  const uint32_t stage_bytes = a_bytes + PLANES * b_plane;
+  const uint32_t a_tcol0 = nbuf * buf_cols;  // ATMEM: A stage s at TMEM column a_tcol0 + 64 s
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + stages * stage_bytes);
   uint64_t* empty = full + TC_MAXSTAGES;
   uint64_t* tfull = empty + TC_MAXSTAGES;   // [2]
@@ -423,9 +479,13 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   }
 #endif
   const int nkb = w.nkb;
+  // the generic fp32 A producer (all TC_PROD_WARPS warps) unless A arrives by TMA, streams raw
+  // (one-pass tf32) or as a dense bf16 activation (128 threads, warps 0-3)
+  const bool generic = !a_tma && PREC != TG_PREC_TF32 && !(PREC == TG_PREC_BF16 && g.a_h);
   if (tid == 0) {
     for (int s = 0; s < stages; ++s) {
-      mbar_init(&full[s], a_tma ? 1 : TC_BM + 1);  // (128 A rows +) the TMA producer's expect_tx
+      // arrivals: the A producer threads (256 generic, 128 streamed) + the TMA warp's expect_tx
+      mbar_init(&full[s], a_tma ? 1 : (generic ? TC_PROD_WARPS * 32 : TC_BM) + 1);
       mbar_init(&empty[s], 1);         // MMA commit
     }
     for (int a = 0; a < 2; ++a) {
@@ -456,9 +516,9 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   const int ntiles = tiles_m * w.ntn;  // CTAs past ntiles run no tile and fall through to the end
   if (tid == 0) TCT(2, clock64());
 
-  if (warp < 4 && a_tma) {
+  if (warp < TC_PROD_WARPS && (a_tma || (!generic && warp >= 4))) {
     // A arrives by TMA (issued by warp 4 with B): nothing to produce here
-  } else if (warp < 4 && PREC == TG_PREC_TF32) {
+  } else if (warp < TC_PROD_WARPS && PREC == TG_PREC_TF32) {
     // ===================== A producers, streamed: raw fp32 rows go straight into
     // the swizzled operand with 16-byte cp.async (zero-fill past K / M); the
     // tensor core reads them as tf32. Completion is tracked by the full barrier
@@ -492,7 +552,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];\n" ::"r"(smem_u32(&full[s])) : "memory");
       }
     }
-  } else if (warp < 4 && PREC == TG_PREC_BF16 && g.a_h) {
+  } else if (warp < TC_PROD_WARPS && PREC == TG_PREC_BF16 && g.a_h) {
     // ===================== A producers, streamed bf16: the activation was
     // written in bf16 by the producing kernel (attention, LayerNorm, FFN1), so
     // its rows go straight into the swizzled operand (64 elements = 128 B per
@@ -518,25 +578,31 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];\n" ::"r"(smem_u32(&full[s])) : "memory");
       }
     }
-  } else if (warp < 4) {
+  } else if (warp < TC_PROD_WARPS) {
     // ===================== A producers (fp32 rows: gathered through row pointers or dense),
-    // converted on the fly. Loads run ahead through a per-thread cp.async staging ring of
-    // `stg` units (a unit = 32 fp32 = 128 B of the thread's own row; UPK units per k-block),
-    // so up to stg x 16 KB per CTA are in flight without holding registers: the producers
-    // are bound by L2 latency otherwise (one k-block of register prefetch measured ~1.4 us
-    // per k-block at ~35% tensor-pipe activity). Each thread reads back only what it
-    // copied itself (cp.async.wait_group), so no cross-thread synchronisation is needed.
+    // converted on the fly by the 256 threads of warps 0-7: thread p converts half the
+    // columns (fp32 chunks 4 (p / 128) .. + 3 of each 32-float unit) of row p % 128. Loads
+    // run ahead through a cp.async staging ring of `stg` units (a unit = 32 fp32 = 128 B of
+    // each of the tile's 128 rows, 16 KB; UPK units per k-block), up to 64 KB per CTA in
+    // flight without holding registers; the copies are coalesced (each warp instruction
+    // moves 8 rows x 64 contiguous bytes). Named barrier 2 (the 256 producer threads) orders
+    // the copies and the reads of a slot. The producers are instruction-latency bound (one
+    // converting warp per scheduler measured ~1.2 us per 16 KB unit), hence 8 warps.
     constexpr int UPK = EPC / 32;
+    constexpr int NPT = TC_PROD_WARPS * 32;
+    const int prow = tid & (TC_BM - 1), ph = tid >> 7;  // row, column half
     unsigned char* sring = smem + stages * stage_bytes + TC_BAR_BYTES + TC_EPI_BYTES + (g.ln ? TC_LN_BYTES : 0);
+    const float** sptr = reinterpret_cast<const float**>(sring + (size_t)stg * TC_STG_UNIT);  // [2][128]
     const int D = stg;
     const int upt = nkb * UPK;  // units per tile
+    auto pbar = [] { asm volatile("bar.sync 2, %0;\n" ::"n"(NPT) : "memory"); };
     // issue cursor: tile it_t (this CTA's sequence), unit it_u within the tile
     int it_t = blockIdx.x, it_u = 0;
     const float* ir0 = nullptr;
     const float* ir1 = nullptr;
     bool irv = false;
     auto rows_of = [&](int tt) {
-      const int row = (tt / w.ntn) * TC_BM + tid;
+      const int row = (tt / w.ntn) * TC_BM + prow;
       irv = tt < ntiles && row < M;
       ir0 = ir1 = nullptr;
       if (irv) {
@@ -544,61 +610,117 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         if (g.K0 < g.K) ir1 = g.a_rows1 ? g.a_rows1[row] : g.a_base1 + (size_t)row * g.lda1;
       }
     };
-    rows_of(it_t);
+    auto publish = [&](int tt) {  // the tile's row pointers -> shared table (threads 0..127)
+      if (ph == 0) rows_of(tt);
+      pbar();                     // every thread is done issuing from the previous table
+      if (ph == 0) {
+        sptr[prow] = irv ? ir0 : nullptr;
+        sptr[TC_BM + prow] = ir1;
+      }
+      pbar();
+    };
     const void* dummy = w.hi;  // valid global address for zero-byte (zero-fill) copies
     auto issue = [&](int slot) {
       if (it_t < ntiles) {
-        const uint32_t dst = smem_u32(sring + (size_t)slot * (TC_BM * 128) + tid * 128);
-        const int col0 = it_u * 32;
+        unsigned char* base = sring + (size_t)slot * TC_STG_UNIT;
+        const int q = lane & 3;
 #pragma unroll
-        for (int c = 0; c < 8; ++c) {
-          const int col = col0 + 4 * c;
-          const bool ok = irv && col < g.K;
-          const void* src = !ok ? dummy : (const void*)(col < g.K0 ? ir0 + col : ir1 + (col - g.K0));
-          asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(dst + ((c ^ (tid & 7)) << 4)),
-                       "l"(src), "r"(ok ? 16 : 0)
-                       : "memory");
+        for (int it = 0; it < TC_BM / (TC_PROD_WARPS * 8); ++it) {
+          const int r = warp * (TC_BM / TC_PROD_WARPS) + it * 8 + (lane >> 2);
+          const float* p0 = sptr[r];
+          const float* p1 = sptr[TC_BM + r];
+#pragma unroll
+          for (int hh = 0; hh < 2; ++hh) {
+            const int c = q + 4 * hh;
+            const int col = it_u * 32 + 4 * c;
+            const bool ok = p0 && col < g.K;
+            const void* src = !ok ? dummy : (const void*)(col < g.K0 ? p0 + col : p1 + (col - g.K0));
+            asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(
+                             smem_u32(base + r * 128 + ((c ^ (r & 7)) << 4))),
+                         "l"(src), "r"(ok ? 16 : 0)
+                         : "memory");
+          }
         }
         if (++it_u == upt) {
           it_u = 0;
           it_t += gridDim.x;
-          rows_of(it_t);
+          if (it_t < ntiles) publish(it_t);
         }
       }
       asm volatile("cp.async.commit_group;\n" ::: "memory");  // (empty past the last tile)
     };
-    for (int i = 0; i < D; ++i) issue(i);
+    if (D > 0) {
+      if (it_t < ntiles) publish(it_t);
+      for (int i = 0; i < D; ++i) issue(i);
+    }
     uint32_t gk = 0, gu = 0;
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
       if (D == 0) rows_of(t);  // no room for staging (widest N tiles): blocking loads
       for (int kb = 0; kb < nkb; ++kb, ++gk) {
         const int s = gk % stages;
         mbar_wait(&empty[s], ((gk / stages) & 1) ^ 1);
+        if (ATMEM) asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
         unsigned char* sA = smem + s * stage_bytes;
         bool big = false;
 #pragma unroll
         for (int h = 0; h < UPK; ++h, ++gu) {
-          // unit gu is the oldest of the D outstanding groups
-          float4 x[8];
+          float4 x[4];  // fp32 chunks 4 ph .. 4 ph + 3 of this unit of row prow
           const int slot = D > 0 ? (int)(gu % (uint32_t)D) : 0;
           if (D == 0) {
 #pragma unroll
-            for (int c = 0; c < 8; ++c)
-              x[c] = irv ? tc_load4(g, ir0, ir1, (kb * UPK + h) * 32 + 4 * c) : make_float4(0.f, 0.f, 0.f, 0.f);
+            for (int i = 0; i < 4; ++i)
+              x[i] = irv ? tc_load4(g, ir0, ir1, (kb * UPK + h) * 32 + 4 * (4 * ph + i))
+                         : make_float4(0.f, 0.f, 0.f, 0.f);
           } else {
             if (D == 1) asm volatile("cp.async.wait_group 0;\n" ::: "memory");
             else if (D == 2) asm volatile("cp.async.wait_group 1;\n" ::: "memory");
             else if (D == 3) asm volatile("cp.async.wait_group 2;\n" ::: "memory");
             else asm volatile("cp.async.wait_group 3;\n" ::: "memory");
-            const unsigned char* src = sring + (size_t)slot * (TC_BM * 128) + tid * 128;
+            pbar();  // every producer's copies of this unit have landed
+            const unsigned char* src = sring + (size_t)slot * TC_STG_UNIT + prow * 128;
 #pragma unroll
-            for (int c = 0; c < 8; ++c) x[c] = *reinterpret_cast<const float4*>(src + ((c ^ (tid & 7)) << 4));
+            for (int i = 0; i < 4; ++i)
+              x[i] = *reinterpret_cast<const float4*>(src + (((4 * ph + i) ^ (prow & 7)) << 4));
+            pbar();  // every producer has read the slot: it may be refilled
+            issue(slot);  // unit gu + D
           }
-          if (PREC == TG_PREC_F16X3) {
+          if (ATMEM) {
+            // columns of this unit: tf32 32 elements = 32 columns (thread half ph: 16);
+            // f16 32 elements = 16 columns (thread half ph: 8); lanes = rows (warp quadrant)
+            const uint32_t tq = tmem + ((uint32_t)((warp & 3) * 32) << 16) + a_tcol0 + 64u * (uint32_t)s;
+            if (PREC == TG_PREC_F16X3) {
+              uint32_t hv[8], lv[8];
 #pragma unroll
-            for (int j = 0; j < 4; ++j) {
-              const float xs[8] = {x[2 * j].x, x[2 * j].y, x[2 * j].z, x[2 * j].w,
-                                   x[2 * j + 1].x, x[2 * j + 1].y, x[2 * j + 1].z, x[2 * j + 1].w};
+              for (int e = 0; e < 8; ++e) {
+                const float x0 = (&x[e >> 1].x)[2 * (e & 1)], x1 = (&x[e >> 1].x)[2 * (e & 1) + 1];
+                const __half2 hh = __floats2half2_rn(x0, x1);
+                const float2 hf = __half22float2(hh);
+                const __half2 ll = __floats2half2_rn(x0 - hf.x, x1 - hf.y);
+                big |= !(fabsf(x0) < 65504.f) | !(fabsf(x1) < 65504.f);
+                hv[e] = *reinterpret_cast<const uint32_t*>(&hh);
+                lv[e] = *reinterpret_cast<const uint32_t*>(&ll);
+              }
+              const uint32_t col = (uint32_t)(h * 16 + ph * 8);
+              tmem_st8(tq + col, hv);
+              tmem_st8(tq + 32u + col, lv);
+            } else {
+              uint32_t hv[16], lv[16];
+#pragma unroll
+              for (int e = 0; e < 16; ++e) {
+                const float xv = (&x[e >> 2].x)[e & 3];
+                const float hi = rna_tf32_fast(xv);
+                hv[e] = __float_as_uint(hi);
+                lv[e] = __float_as_uint(rna_tf32_fast(xv - hi));
+              }
+              const uint32_t col = (uint32_t)(ph * 16);
+              tmem_st16(tq + col, hv);
+              tmem_st16(tq + 32u + col, lv);
+            }
+          } else if (PREC == TG_PREC_F16X3) {
+#pragma unroll
+            for (int jj = 0; jj < 2; ++jj) {  // fp16 chunk j = 2 ph + jj <- fp32 chunks 2j, 2j + 1
+              const float xs[8] = {x[2 * jj].x, x[2 * jj].y, x[2 * jj].z, x[2 * jj].w,
+                                   x[2 * jj + 1].x, x[2 * jj + 1].y, x[2 * jj + 1].z, x[2 * jj + 1].w};
               uint32_t hv[4], lv[4];
 #pragma unroll
               for (int e = 0; e < 4; ++e) {
@@ -609,14 +731,14 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
                 hv[e] = *reinterpret_cast<const uint32_t*>(&hh);
                 lv[e] = *reinterpret_cast<const uint32_t*>(&ll);
               }
-              const int c = h * 4 + j;
-              *reinterpret_cast<uint4*>(sA + sw128(tid, c)) = make_uint4(hv[0], hv[1], hv[2], hv[3]);
-              *reinterpret_cast<uint4*>(sA + a_plane + sw128(tid, c)) = make_uint4(lv[0], lv[1], lv[2], lv[3]);
+              const int c = h * 4 + 2 * ph + jj;
+              *reinterpret_cast<uint4*>(sA + sw128(prow, c)) = make_uint4(hv[0], hv[1], hv[2], hv[3]);
+              *reinterpret_cast<uint4*>(sA + a_plane + sw128(prow, c)) = make_uint4(lv[0], lv[1], lv[2], lv[3]);
             }
           } else if (PREC == TG_PREC_BF16) {
 #pragma unroll
-            for (int j = 0; j < 4; ++j) {
-              const float4 x0 = x[2 * j], x1 = x[2 * j + 1];
+            for (int jj = 0; jj < 2; ++jj) {
+              const float4 x0 = x[2 * jj], x1 = x[2 * jj + 1];
               __nv_bfloat162 p0 = __floats2bfloat162_rn(x0.x, x0.y), p1 = __floats2bfloat162_rn(x0.z, x0.w);
               __nv_bfloat162 p2 = __floats2bfloat162_rn(x1.x, x1.y), p3 = __floats2bfloat162_rn(x1.z, x1.w);
               uint4 u;
@@ -624,36 +746,41 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
               u.y = *reinterpret_cast<uint32_t*>(&p1);
               u.z = *reinterpret_cast<uint32_t*>(&p2);
               u.w = *reinterpret_cast<uint32_t*>(&p3);
-              *reinterpret_cast<uint4*>(sA + sw128(tid, h * 4 + j)) = u;
+              *reinterpret_cast<uint4*>(sA + sw128(prow, h * 4 + 2 * ph + jj)) = u;
             }
           } else {
 #pragma unroll
-            for (int c = 0; c < 8; ++c) {
-              const float4 xv = x[c];
+            for (int i = 0; i < 4; ++i) {
+              const int c = 4 * ph + i;
+              const float4 xv = x[i];
               float4 hi, lo;
-              hi.x = rna_tf32(xv.x);
-              hi.y = rna_tf32(xv.y);
-              hi.z = rna_tf32(xv.z);
-              hi.w = rna_tf32(xv.w);
-              *reinterpret_cast<float4*>(sA + sw128(tid, c)) = hi;
+              hi.x = rna_tf32_fast(xv.x);
+              hi.y = rna_tf32_fast(xv.y);
+              hi.z = rna_tf32_fast(xv.z);
+              hi.w = rna_tf32_fast(xv.w);
+              *reinterpret_cast<float4*>(sA + sw128(prow, c)) = hi;
               if (PLANES == 2) {
-                lo.x = rna_tf32(xv.x - hi.x);
-                lo.y = rna_tf32(xv.y - hi.y);
-                lo.z = rna_tf32(xv.z - hi.z);
-                lo.w = rna_tf32(xv.w - hi.w);
-                *reinterpret_cast<float4*>(sA + a_plane + sw128(tid, c)) = lo;
+                lo.x = rna_tf32_fast(xv.x - hi.x);
+                lo.y = rna_tf32_fast(xv.y - hi.y);
+                lo.z = rna_tf32_fast(xv.z - hi.z);
+                lo.w = rna_tf32_fast(xv.w - hi.w);
+                *reinterpret_cast<float4*>(sA + a_plane + sw128(prow, c)) = lo;
               }
             }
           }
-          if (D > 0) issue(slot);  // refill the slot just consumed: unit gu + D
         }
         if (PREC == TG_PREC_F16X3 && big && g.err) atomicOr(g.err, kErrF16Range);
-        asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");  // generic -> async proxy
+        if (ATMEM) {
+          asm volatile("tcgen05.wait::st.sync.aligned;\n" ::: "memory");
+          asm volatile("tcgen05.fence::before_thread_sync;\n" ::: "memory");
+        } else {
+          asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");  // generic -> async proxy
+        }
         mbar_arrive(&full[s]);
       }
     }
     asm volatile("cp.async.wait_group 0;\n" ::: "memory");
-  } else if (warp == 4) {
+  } else if (warp == TC_TMA_WARP) {
     // ===================== B producer (TMA bulk copies of weight tile images)
     if (lane == 0) {
       uint32_t gk = 0;
@@ -662,7 +789,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         for (int kb = 0; kb < nkb; ++kb, ++gk) {
           const int s = gk % stages;
           mbar_wait(&empty[s], ((gk / stages) & 1) ^ 1);
-          unsigned char* sB = smem + s * stage_bytes + PLANES * a_plane;
+          unsigned char* sB = smem + s * stage_bytes + a_bytes;
           const unsigned char* src =
               reinterpret_cast<const unsigned char*>(w.hi) + ((size_t)tn * nkb + kb) * PLANES * b_plane;
           if (gk == 0) TCT(4, clock64());
@@ -681,7 +808,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         }
       }
     }
-  } else if (warp == 5) {
+  } else if (warp == TC_MMA_WARP) {
     // ===================== MMA issuer
     if (lane == 0) {
       const uint32_t idesc = umma_idesc(PREC, BN);
@@ -698,10 +825,17 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");  // cp.async A -> tensor core
           asm volatile("tcgen05.fence::after_thread_sync;\n");
           const uint32_t aH = smem_u32(smem + s * stage_bytes);
-          const uint32_t bH = aH + PLANES * a_plane;
+          const uint32_t bH = aH + a_bytes;
+          const uint32_t aT = tmem + a_tcol0 + 64u * (uint32_t)s;  // ATMEM: A planes at aT, aT + 32
 #pragma unroll
           for (int kk = 0; kk < 4; ++kk) {  // 4 MMAs of 32 bytes of K per 128B k-block
             const uint32_t acc0 = (kb > 0 || kk > 0) ? 1u : 0u;
+            if (ATMEM) {  // 8 TMEM columns of A per MMA; correction terms into `small`
+              mma_issue_ts<PREC>(dtm, aT + kk * 8, umma_desc(bH + kk * 32), idesc, acc0);
+              mma_issue_ts<PREC>(dtm + small_off, aT + kk * 8, umma_desc(bH + b_plane + kk * 32), idesc, acc0);
+              mma_issue_ts<PREC>(dtm + small_off, aT + 32 + kk * 8, umma_desc(bH + kk * 32), idesc, 1u);
+              continue;
+            }
             mma_issue<PREC>(dtm, umma_desc(aH + kk * 32), umma_desc(bH + kk * 32), idesc, acc0);
             if (PLANES == 2) {
               mma_issue<PREC>(dtm + small_off, umma_desc(aH + kk * 32), umma_desc(bH + b_plane + kk * 32), idesc,
@@ -730,7 +864,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     // arrive); pass 2 re-reads the accumulator, normalises with the merged statistics
     // (fixed tile order) and stores the bf16 LN(y) block of the merge-FFN input (Eq. 7).
     const int quad = warp & 3;
-    const int ew = warp - 6;
+    const int ew = warp - TC_EPI_WARP0;
     const int half = ew >> 2;
     float* stg = reinterpret_cast<float*>(smem + stages * stage_bytes + TC_BAR_BYTES) + ew * (32 * TC_STG_LD);
     float4* lnh = reinterpret_cast<float4*>(smem + stages * stage_bytes + TC_BAR_BYTES + TC_EPI_BYTES);  // [2][128]
@@ -744,7 +878,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     const int ntn = w.ntn;
     {  // this CTA's column tile is fixed (grid is a multiple of ntn)
       const int nb0 = (int)(blockIdx.x % ntn) * BN;
-      for (int i = tid - 6 * 32; i < BN; i += TC_EPI_WARPS * 32) {
+      for (int i = tid - TC_EPI_WARP0 * 32; i < BN; i += TC_EPI_WARPS * 32) {
         const int c = nb0 + i;
         const bool in = c < g.N;
         s_bias[i] = in ? g.bias[c] : 0.f;
@@ -766,7 +900,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       const uint32_t tacc = tmem + acc * buf_cols + ((uint32_t)(quad * 32) << 16);
       // ---- pass 1: row statistics of this thread's column chunks
       float sn = 0.f, sm = 0.f, sM = 0.f;
-      for (int c0 = 16 * half; c0 < BN; c0 += 32) {
+      for (int c0 = 16 * half; c0 < BN; c0 += 16 * TC_EPI_HALVES) {
         uint32_t v[16];
         tmem_ld16(tacc + (uint32_t)c0, v);
         asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
@@ -792,8 +926,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       lnh[half * TC_BM + rloc] = make_float4(sn, sm, sM, 0.f);
       asm volatile("bar.sync 1, %0;\n" ::"n"(TC_EPI_WARPS * 32) : "memory");
       if (half == 0) {
-        const float4 o = lnh[TC_BM + rloc];
-        chan_merge(sn, sm, sM, o.x, o.y, o.z);
+        if (TC_EPI_HALVES == 2) {
+          const float4 o = lnh[TC_BM + rloc];
+          chan_merge(sn, sm, sM, o.x, o.y, o.z);
+        }
         const float4 st4 = make_float4(sn, sm, sM, 0.f);
         const uint32_t slot = smem_u32(lnx + (par * TC_LN_MAXTN + tn) * TC_BM + rloc);
         for (int r = 0; r < ntn; ++r) st_cluster_v4(mapa_u32(slot, (uint32_t)r), st4);
@@ -809,11 +945,11 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       const float rstd = rsqrtf(M2 / fmaxf(n, 1.f) + 1e-5f);
       // ---- pass 2: normalise, transpose through shared memory, coalesced bf16 stores
       bool released = false;
-      for (int c0 = 16 * half; c0 < BN; c0 += 32) {
+      for (int c0 = 16 * half; c0 < BN; c0 += 16 * TC_EPI_HALVES) {
         uint32_t v[16];
         tmem_ld16(tacc + (uint32_t)c0, v);
         asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
-        if (c0 + 32 >= BN) {  // this warp's last chunk: hand the accumulator back
+        if (c0 + 16 * TC_EPI_HALVES >= BN) {  // this warp's last chunk: hand the accumulator back
           asm volatile("tcgen05.fence::before_thread_sync;\n");
           mbar_arrive(&tempty[acc]);
           released = true;
@@ -859,8 +995,8 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     // aligned, conflict-free STS.128) and written back with lanes = 4 columns x
     // 8 rows: float4 bias/ReLU and 64-byte coalesced row segments.
     const int quad = warp & 3;
-    const int ew = warp - 6;               // 0..7
-    const int half = ew >> 2;              // which alternate chunk
+    const int ew = warp - TC_EPI_WARP0;    // 0 .. TC_EPI_WARPS - 1
+    const int half = ew >> 2;              // which alternate chunk (with 8 epilogue warps)
     float* stg = reinterpret_cast<float*>(smem + stages * stage_bytes + TC_BAR_BYTES) + ew * (32 * TC_STG_LD);
     const int rq = lane >> 2, cq = lane & 3;  // read-back: row rq + 8i, float4 column cq
     uint32_t tc = 0;
@@ -877,10 +1013,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         if (g.c_h) hrow = g.c_h + (size_t)er * g.ldc_h;
       }
       mbar_wait(&tfull[acc], (tc / nbuf) & 1);
-      if (tc == 0 && warp == 6 && lane == 0) TCT(5, clock64());
+      if (tc == 0 && warp == TC_EPI_WARP0 && lane == 0) TCT(5, clock64());
       asm volatile("tcgen05.fence::after_thread_sync;\n");
       bool released = false;
-      for (int c0 = 16 * half; c0 < BN; c0 += 32) {
+      for (int c0 = 16 * half; c0 < BN; c0 += 16 * TC_EPI_HALVES) {
         uint32_t v[16];
         const uint32_t tq = tmem + acc * buf_cols + ((uint32_t)(quad * 32) << 16) + (uint32_t)c0;
         tmem_ld16(tq, v);
@@ -893,7 +1029,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         } else {
           asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
         }
-        if (c0 + 32 >= BN) {  // this warp's last chunk: hand the accumulator back
+        if (c0 + 16 * TC_EPI_HALVES >= BN) {  // this warp's last chunk: hand the accumulator back
           asm volatile("tcgen05.fence::before_thread_sync;\n");
           mbar_arrive(&tempty[acc]);
           released = true;
@@ -953,14 +1089,14 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         asm volatile("tcgen05.fence::before_thread_sync;\n");
         mbar_arrive(&tempty[acc]);
       }
-      if (tc == 0 && warp == 6 && lane == 0) TCT(6, clock64());
+      if (tc == 0 && warp == TC_EPI_WARP0 && lane == 0) TCT(6, clock64());
     }
   }
-  if (lane == 0 && warp >= 4 && warp <= 6) TCT(56 + warp, clock64());  // role done (before the barrier)
+  if (lane == 0 && warp >= TC_TMA_WARP && warp <= TC_EPI_WARP0) TCT(60 + warp - TC_TMA_WARP, clock64());  // role done (before the barrier)
   asm volatile("tcgen05.fence::before_thread_sync;\n");
   __syncthreads();
   if (tid == 0) TCT(7, clock64());
-  if (tid == 6 * 32) TCT(55, clock64());
+  if (tid == TC_EPI_WARP0 * 32) TCT(55, clock64());
   asm volatile("tcgen05.fence::after_thread_sync;\n");
   if (g.ln) {  // no CTA leaves while a peer may still address its shared memory
     asm volatile("barrier.cluster.arrive.release.aligned;\n" ::: "memory");
@@ -971,8 +1107,9 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
 
 static size_t tc_smem(int prec, int BN, int stages, int stg, int ln = 0) {
   const size_t planes = tc_planes(prec);
-  size_t s = 1024 + (size_t)stages * planes * ((size_t)TC_BM * 128 + (size_t)BN * 128) + TC_BAR_BYTES + TC_EPI_BYTES +
-             (ln ? TC_LN_BYTES : 0) + (size_t)stg * TC_STG_UNIT;
+  size_t s = 1024 + (size_t)stages * planes * ((tc_atmem(prec) ? 0 : (size_t)TC_BM * 128) + (size_t)BN * 128) +
+             TC_BAR_BYTES + TC_EPI_BYTES +
+             (ln ? TC_LN_BYTES : 0) + (size_t)stg * TC_STG_UNIT + (stg ? TC_PTR_BYTES : 0);
   // tf32x3: one CTA per SM (it allocates all 512 TMEM columns; a second
   // co-resident CTA would block in tcgen05.alloc until the first one exits).
   const size_t one_per_sm = 120 * 1024;

@@ -1,0 +1,4 @@
+python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
+timeout 300 python -m pytest tests/test_gpu_parity.py -q -x -k "gemm or embed_parity" 2>&1 | tail -2
+for nk in "516 1032" "172 688"; do set -- $nk; echo "== tf32x3 N=$1 K=$2"; python tools/gemm_trace.py --n $1 --k $2 --precision tf32x3 --edges 60000 2>&1 | grep -E "landed|mma_commit"; done
+python tools/gemm_bench.py --m 25000 --precs 1 --reps 10 2>&1 | grep -v "^$"
