@@ -110,12 +110,10 @@ typedef struct {
                                * 1 = one batch at a time, <= 128). Semantics per batch are
                                * unchanged: dedup scope, cache lookups and FIFO inserts stay per
                                * batch and in batch order, so outputs and counters do not depend
-                               * on S. Superbatches the host proves eviction-free (FIFO size bound
-                               * + S x capacity <= limit) run the grid-wide lookup pass with this S
-                               * (bounded by a ~40 GB workspace budget); superbatches that may
-                               * evict run the ordered pass with S_small, the largest S whose keys
-                               * fit its cluster DSMEM hash at a worst-case load <= 0.9 (batch 200,
-                               * k = 20: 28; batch 2,000: 1). tg_superbatch() returns S. */
+                               * on S. Both cache passes (grid-wide eviction-free pass, ordered
+                               * pass) keep their superbatch hash in global memory, so S is bounded
+                               * only by a ~40 GB budget for the S-proportional workspaces.
+                               * tg_superbatch() returns the S in use. */
 } tg_model_cfg;
 
 /* params: host float32 [n_params] in this order (row-major, Linear = [out x in]),

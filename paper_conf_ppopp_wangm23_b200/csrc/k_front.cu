@@ -450,9 +450,6 @@ __global__ void k_probe_pre(LevelDev lv, int S, CacheDev c) { pdl_enter();
   if (blockIdx.x == 0 && threadIdx.x == 0 && c.occ_report) {  // one 64-bit store: consistent pair
     const unsigned long long occ = (unsigned long long)c.state[3] & ((1ull << 40) - 1);
     *(volatile unsigned long long*)c.occ_report = ((unsigned long long)(c.report_sb + 1) << 40) | occ;
-    if (c.size_report)  // live size at superbatch start (host bound for the eviction-free schedule)
-      *(volatile unsigned long long*)c.size_report =
-          ((unsigned long long)(c.report_sb + 1) << 40) | ((unsigned long long)c.state[1] & ((1ull << 40) - 1));
     __threadfence_system();
   }
   if (c.sb_key) {  // clear the superbatch-scoped hash of the grid-wide pass (k_sbh_*)
@@ -490,9 +487,11 @@ constexpr int kSeqSlots = kSeqSlotsPerCTA;
 
 __global__ void __launch_bounds__(kSeqThreads, 1)
 k_probe_seq(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err) { pdl_enter();
-  extern __shared__ __align__(16) unsigned char smem[];
-  unsigned long long* skey = reinterpret_cast<unsigned long long*>(smem);
-  int* sq = reinterpret_cast<int*>(skey + kSeqSlots);  // key -> q of its latest miss in this SB
+  // key -> q of its latest miss in this superbatch: the superbatch hash in global memory
+  // (L2-resident, cleared by k_probe_pre), so any S fits (r1 kept it in DSMEM, capping S)
+  unsigned long long* skey = c.sb_key;
+  unsigned* sq = c.sb_val;
+  __shared__ int s_pre[kMaxS + 1];
   __shared__ int s_warp[32];
   __shared__ int s_total;
   __shared__ long long s_head, s_size;
@@ -501,14 +500,8 @@ k_probe_seq(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err)
   const unsigned CL = cluster.num_blocks();
   const unsigned rank = cluster.block_rank();
   const int tid = threadIdx.x;
+  const int NT = sbh_pre(lv, S, s_pre);
   if (c.state[5] == 1) return;  // the eviction-free parallel pass handled this superbatch
-  // the host runs superbatches that may evict with S small enough for this DSMEM hash
-  // (tg_model_load: S_small); a larger one would overflow it -- report, never mis-count
-  if ((long long)S * lv.cap * 10 > (long long)CL * kSeqSlots * 9) {
-    if (rank == 0 && tid == 0) atomicOr(err, kErrIndexFull);
-    return;
-  }
-  for (int s = tid; s < kSeqSlots; s += blockDim.x) skey[s] = kEmptyKey;
   if (rank == 0 && tid == 0) {
     s_head = __ldcg(c.state + 0);
     s_size = __ldcg(c.state + 1);
@@ -517,7 +510,7 @@ k_probe_seq(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err)
   }
   const long long limit = __ldcg(c.state + 2);
   const long long head0 = __ldcg(c.state + 0);
-  const unsigned long long tmask = (unsigned long long)CL * kSeqSlots - 1ull;
+  const unsigned long long tmask = sbh_mask(c, NT);
   cluster.sync();
   for (int b = 0; b < S; ++b) {
     const long long head = *cluster.map_shared_rank(&s_head, 0);
@@ -542,11 +535,11 @@ k_probe_seq(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err)
         long long p = -1;
         unsigned long long h = mix64(key) & tmask;
         for (unsigned long long pr = 0; pr <= tmask; ++pr) {
-          const unsigned long long k0 = *(cluster.map_shared_rank(skey, (unsigned)(h / kSeqSlots)) + (h % kSeqSlots));
+          const unsigned long long k0 = __ldcg(skey + h);
           if (k0 == kEmptyKey) break;
           if (k0 == key) {
             sbslot[j] = (unsigned)h;
-            p = head0 + *(cluster.map_shared_rank(sq, (unsigned)(h / kSeqSlots)) + (h % kSeqSlots));
+            p = head0 + __ldcg(sq + h);
             break;
           }
           h = (h + 1) & tmask;
@@ -587,16 +580,16 @@ k_probe_seq(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err)
         const unsigned long long key = tkey(node, t);
         if (sbslot[j] != 0xFFFFFFFFu) {  // evicted and missed again inside this SB
           const unsigned h = sbslot[j];
-          int* qp = cluster.map_shared_rank(sq, h / kSeqSlots) + (h % kSeqSlots);
-          lv.sup[*qp] = 1;
-          *qp = q;
+          unsigned* qp = sq + h;
+          lv.sup[__ldcg(qp)] = 1;
+          *qp = (unsigned)q;
         } else {
           unsigned long long h = mix64(key) & tmask;
           for (unsigned long long pr = 0; pr <= tmask; ++pr) {
-            unsigned long long* kp = cluster.map_shared_rank(skey, (unsigned)(h / kSeqSlots)) + (h % kSeqSlots);
+            unsigned long long* kp = skey + h;
             const unsigned long long old = atomicCAS(kp, kEmptyKey, key);
             if (old == kEmptyKey || old == key) {
-              *(cluster.map_shared_rank(sq, (unsigned)(h / kSeqSlots)) + (h % kSeqSlots)) = q;
+              sq[h] = (unsigned)q;
               break;
             }
             h = (h + 1) & tmask;
@@ -998,16 +991,14 @@ int launch_probe(LevelDev lv, int S, const CacheDev* cache, long long* cnt, int 
   int blocks = (S * lv.cap + 255) / 256;
   if (blocks > 148 * 8) blocks = 148 * 8;
   launch_k(k_probe_pre, dim3(blocks), dim3(256), 0, st, lv, S, c);
-  const size_t smem = (size_t)kSeqSlots * (sizeof(unsigned long long) + sizeof(int));
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(k_probe_seq, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     cudaFuncSetAttribute(k_probe_seq, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
     attr = true;
   }
-  // cluster large enough for every key of the superbatch to be an in-SB miss (load <= 0.6)
+  // the ordered pass walks one batch at a time: enough CTAs for <= 4 keys per thread
   int cl = 1;
-  while (cl < kSeqCL && (long long)cl * kSeqSlots * 6 / 10 < (long long)S * lv.cap) cl <<= 1;
+  while (cl < kSeqCL && (long long)cl * kSeqThreads * 4 < (long long)lv.cap) cl <<= 1;
   // eviction-free superbatches: grid-wide pass (k_sbh_*); otherwise the ordered pass
   const int nj = S * lv.cap;
   int gb = (nj + 255) / 256;
@@ -1017,8 +1008,7 @@ int launch_probe(LevelDev lv, int S, const CacheDev* cache, long long* cnt, int 
   launch_k(k_sbh_count, dim3(nblk), dim3(kSbhThreads), 0, st, lv, S, c);
   launch_k(k_sbh_assign, dim3(nblk), dim3(kSbhThreads), 0, st, lv, S, c);
   launch_k(k_sbh_finish, dim3(gb), dim3(256), 0, st, lv, S, c, cnt, layer, nblk);
-  if (cl > kSeqCL) cl = kSeqCL;
-  launch_k_cluster(k_probe_seq, dim3(cl), dim3(kSeqThreads), smem, st, cl, lv, S, c, cnt, layer, err);
+  launch_k_cluster(k_probe_seq, dim3(cl), dim3(kSeqThreads), 0, st, cl, lv, S, c, cnt, layer, err);
   int ib = (S * lv.cap + 255) / 256;
   if (ib > 148 * 4) ib = 148 * 4;
   launch_k(k_probe_ins, dim3(ib), dim3(256), 0, st, lv, c, err);

@@ -91,8 +91,9 @@ static inline void tc_plan(int prec, int BN, int ln, bool generic, int* stages, 
   if (generic) {
     d = budget > 2 * st ? (int)((budget - 2 * st) / TC_STG_UNIT) : 0;
     d = d > d_env ? d_env : d;
+    if (d_env < 0) d = -1;  // TG_GEMM_STG=-1: register prefetch, no staging ring
   }
-  int s = (int)((budget - (size_t)d * TC_STG_UNIT) / st);
+  int s = (int)((budget - (size_t)(d > 0 ? d : 0) * TC_STG_UNIT) / st);
   if (s > TC_MAXSTAGES) s = TC_MAXSTAGES;
   if (tc_atmem(prec)) {  // TMEM: one [big | small] accumulator + 64 columns of A per stage
     const int acc = 2 * ((BN + 31) & ~31);
@@ -402,6 +403,11 @@ __device__ __forceinline__ float4 tc_load4(const GemmArgs& g, const float* r0, c
   const float* p = col < g.K0 ? r0 + col : r1 + (col - g.K0);
   return *reinterpret_cast<const float4*>(p);
 }
+__device__ __forceinline__ float4 tc_ldg4(const GemmArgs& g, const float* r0, const float* r1, int col) {
+  if (col >= g.K) return make_float4(0.f, 0.f, 0.f, 0.f);
+  const float* p = col < g.K0 ? r0 + col : r1 + (col - g.K0);
+  return __ldg(reinterpret_cast<const float4*>(p));  // A is read-only for the whole launch
+}
 
 #ifdef TG_TC_TRACE
 // Debug build only (build.py TG_TRACE=1 -> libtg_trace.so): clock64 stamps of the
@@ -592,10 +598,44 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     constexpr int NPT = TC_PROD_WARPS * 32;
     const int prow = tid & (TC_BM - 1), ph = tid >> 7;  // row, column half
     unsigned char* sring = smem + stages * stage_bytes + TC_BAR_BYTES + TC_EPI_BYTES + (g.ln ? TC_LN_BYTES : 0);
-    const float** sptr = reinterpret_cast<const float**>(sring + (size_t)stg * TC_STG_UNIT);  // [2][128]
-    const int D = stg;
+    const float** sptr = reinterpret_cast<const float**>(sring + (size_t)(stg > 0 ? stg : 0) * TC_STG_UNIT);  // [2][128]
+    // stg < 0: no staging ring -- each thread prefetches its own row half two units ahead
+    // in registers (no shared-memory round trip, no producer barriers)
+    const bool regpf = stg < 0;
+    const int D = regpf ? 0 : stg;
     const int upt = nkb * UPK;  // units per tile
     auto pbar = [] { asm volatile("bar.sync 2, %0;\n" ::"n"(NPT) : "memory"); };
+    float4 pf0[4], pf1[4];
+    int pt = blockIdx.x, pu = 0;
+    const float* pr0 = nullptr;
+    const float* pr1 = nullptr;
+    bool prv = false;
+    auto prow_of = [&](int tt) {
+      const int row = (tt / w.ntn) * TC_BM + prow;
+      prv = tt < ntiles && row < M;
+      pr0 = pr1 = nullptr;
+      if (prv) {
+        pr0 = g.a_rows0 ? g.a_rows0[row] : g.a_base0 + (size_t)row * g.lda0;
+        if (g.K0 < g.K) pr1 = g.a_rows1 ? g.a_rows1[row] : g.a_base1 + (size_t)row * g.lda1;
+      }
+    };
+    auto fetch = [&](float4 (&d)[4]) {
+      if (pt < ntiles) {
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+          d[i] = prv ? tc_ldg4(g, pr0, pr1, pu * 32 + 4 * (4 * ph + i)) : make_float4(0.f, 0.f, 0.f, 0.f);
+        if (++pu == upt) {
+          pu = 0;
+          pt += gridDim.x;
+          prow_of(pt);
+        }
+      }
+    };
+    if (regpf) {
+      prow_of(pt);
+      fetch(pf0);
+      fetch(pf1);
+    }
     // issue cursor: tile it_t (this CTA's sequence), unit it_u within the tile
     int it_t = blockIdx.x, it_u = 0;
     const float* ir0 = nullptr;
@@ -649,13 +689,13 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       }
       asm volatile("cp.async.commit_group;\n" ::: "memory");  // (empty past the last tile)
     };
-    if (D > 0) {
+    if (D > 0) {  // (regpf: D = 0)
       if (it_t < ntiles) publish(it_t);
       for (int i = 0; i < D; ++i) issue(i);
     }
     uint32_t gk = 0, gu = 0;
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
-      if (D == 0) rows_of(t);  // no room for staging (widest N tiles): blocking loads
+      if (D == 0 && !regpf) rows_of(t);  // no room for staging (widest N tiles): blocking loads
       for (int kb = 0; kb < nkb; ++kb, ++gk) {
         const int s = gk % stages;
         mbar_wait(&empty[s], ((gk / stages) & 1) ^ 1);
@@ -666,7 +706,14 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         for (int h = 0; h < UPK; ++h, ++gu) {
           float4 x[4];  // fp32 chunks 4 ph .. 4 ph + 3 of this unit of row prow
           const int slot = D > 0 ? (int)(gu % (uint32_t)D) : 0;
-          if (D == 0) {
+          if (regpf) {
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+              x[i] = pf0[i];
+              pf0[i] = pf1[i];
+            }
+            fetch(pf1);  // unit gu + 2
+          } else if (D == 0) {
 #pragma unroll
             for (int i = 0; i < 4; ++i)
               x[i] = irv ? tc_load4(g, ir0, ir1, (kb * UPK + h) * 32 + 4 * (4 * ph + i))
@@ -1109,7 +1156,7 @@ static size_t tc_smem(int prec, int BN, int stages, int stg, int ln = 0) {
   const size_t planes = tc_planes(prec);
   size_t s = 1024 + (size_t)stages * planes * ((tc_atmem(prec) ? 0 : (size_t)TC_BM * 128) + (size_t)BN * 128) +
              TC_BAR_BYTES + TC_EPI_BYTES +
-             (ln ? TC_LN_BYTES : 0) + (size_t)stg * TC_STG_UNIT + (stg ? TC_PTR_BYTES : 0);
+             (ln ? TC_LN_BYTES : 0) + (size_t)(stg > 0 ? stg : 0) * TC_STG_UNIT + (stg > 0 ? TC_PTR_BYTES : 0);
   // tf32x3: one CTA per SM (it allocates all 512 TMEM columns; a second
   // co-resident CTA would block in tcgen05.alloc until the first one exits).
   const size_t one_per_sm = 120 * 1024;

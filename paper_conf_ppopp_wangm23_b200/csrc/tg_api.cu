@@ -49,9 +49,6 @@ struct tg_ctx {
   bool loaded = false;
   tg_model_cfg cfg{};
   int L = 0, H = 0, k = 0, d_n = 0, d_e = 0, d_t = 0, dnp = 0, dep = 0, dtp = 0, Dp = 0, W = 0, S = 1;
-  // superbatch sizes: S (workspaces; superbatches the host can prove eviction-free) and
-  // S_small (superbatches that may evict: the ordered pass's DSMEM hash bounds it)
-  int S_small = 1;
   LayerW lw[TG_MAX_LAYERS];
   float *omega = nullptr, *phi = nullptr, *table = nullptr;
   float *Wa1 = nullptr, *ba1 = nullptr, *Wa2 = nullptr;
@@ -75,9 +72,6 @@ struct tg_ctx {
   int64_t limit0 = 0;
   long long idx_bound[TG_MAX_LAYERS + 1]{};  // host upper bound on occupied index slots (rebuild trigger)
   unsigned long long* occ_h = nullptr;       // host-mapped [TG_MAX_LAYERS + 1] occupancy reports
-  unsigned long long* size_h = nullptr;      // host-mapped [TG_MAX_LAYERS + 1] live-size reports
-  long long extra_keys = 0;                  // layer-L targets that need not be edge endpoints
-  long long ins_bound[TG_MAX_LAYERS + 1]{};  // sum of S x cap over superbatches since the reset
   long long sb_count = 0;                    // superbatches issued since the last cache reset
   long long targets_issued = 0;              // layer-L targets issued since the last cache reset
   // compute workspace
@@ -469,10 +463,6 @@ tg_status run_front(tg_ctx* ctx, int S, bool edge_mode, const EdgeSrc& es, int n
   long long* cnt = ctx->cnt_sb;
   ctx->targets_issued += edge_mode ? (es.neg ? 3 : 2) * std::min<int64_t>((int64_t)S * es.B, es.n_edges - es.e0)
                                    : (long long)S * n_max_top;
-  // keys outside the 2E + 1 edge-endpoint universe: negatives, arbitrary embed targets
-  ctx->extra_keys += edge_mode ? (es.neg ? std::min<int64_t>((int64_t)S * es.B, es.n_edges - es.e0) : 0)
-                               : (long long)S * n_max_top;
-  for (int l = 1; l < L; ++l) ctx->ins_bound[l] += (long long)S * ctx->cap[l];
   // ---- top-down (Alg. 1 l.5-12): dedup, lookup/compaction, sampling
   {
     Prof pf(ctx, TG_ST_DEDUP, st);
@@ -517,7 +507,6 @@ tg_status run_front(tg_ctx* ctx, int S, bool edge_mode, const EdgeSrc& es, int n
           if (b < ctx->idx_bound[l - 1]) ctx->idx_bound[l - 1] = b;
         }
         cd.occ_report = ctx->occ_h ? ctx->occ_h + (l - 1) : nullptr;
-        cd.size_report = ctx->size_h ? ctx->size_h + (l - 1) : nullptr;
         cd.report_sb = ctx->sb_count;
         if (ctx->idx_bound[l - 1] * kIndexRebuildDen > slots * kIndexRebuildNum) {
           Prof pf(ctx, TG_ST_LOOKUP, st);
@@ -574,28 +563,6 @@ tg_status run_front(tg_ctx* ctx, int S, bool edge_mode, const EdgeSrc& es, int n
   return TG_OK;
 }
 
-// Can the next superbatch of S batches be proven eviction-free on the host, without a
-// device sync (then it may use the large S: the grid-wide lookup pass has no S bound)?
-// Upper bounds on the live FIFO size of each cached level at its start: the key universe
-// (with dedup every live item is a distinct key, and every cached key is an edge endpoint
-// <i, t_e>, <0, 0> or an extra target), the inserts issued since the reset, and
-// the latest device report (k_probe_pre) plus the inserts issued after it.
-bool sb_eviction_free(tg_ctx* ctx, int S) {
-  if (!(ctx->cfg.opts & TG_OPT_CACHE)) return true;
-  const long long limit = ctx->cfg.cache_limit;
-  for (int l = 1; l < ctx->L; ++l) {
-    const long long per_sb = (long long)ctx->S * ctx->cap[l];
-    long long b = ctx->ins_bound[l];
-    if (ctx->cfg.opts & TG_OPT_DEDUP) b = std::min(b, 2 * ctx->g.E + 1 + ctx->extra_keys);
-    const unsigned long long rep = ctx->size_h ? *(volatile unsigned long long*)&ctx->size_h[l] : 0ull;
-    const long long sb_obs = (long long)(rep >> 40) - 1;
-    if (sb_obs >= 0 && sb_obs <= ctx->sb_count)
-      b = std::min(b, (long long)(rep & ((1ull << 40) - 1)) + (ctx->sb_count - sb_obs) * per_sb);
-    if (b + (long long)S * ctx->cap[l] > limit) return false;
-  }
-  return true;
-}
-
 // Bottom-up half (Alg. 1 l.13-18): M and FFN, layer by layer over all S batches.
 tg_status run_back(tg_ctx* ctx, cudaStream_t st) {
   for (int l = 1; l <= ctx->L; ++l) TRY(run_layer(ctx, l, st));
@@ -627,7 +594,7 @@ tg_status stream_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, cons
   CK(cudaStreamWaitEvent(ctx->fst, ctx->ev_in, 0));
   int64_t sb = 0;
   for (int64_t b0 = 0, S = 0; b0 < nb; b0 += S, ++sb) {
-    S = std::min<int64_t>(sb_eviction_free(ctx, ctx->S) ? ctx->S : ctx->S_small, nb - b0);
+    S = std::min<int64_t>(ctx->S, nb - b0);
     const int set = (int)(sb & 1);
     EdgeSrc es{src, dst, ts, neg, n_edges, b0 * batch, batch};
     const int per_edge = neg ? 3 : 2;  // targets per edge: src || dst (|| neg, NEXT-3)
@@ -828,16 +795,9 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     if (cap[l] > 16 * 10000) return TG_EINVAL;                   // dedup cluster bound
     if (cap[l] > kSeqCLMax * 1024 * kProbeIPT) return TG_EINVAL; // ordered cache pass bound
   }
-  // Superbatches that may evict run the ordered cache pass, whose DSMEM hash must hold
-  // every key of the superbatch's cached level at a worst-case load <= 0.9 (cap assumes
-  // every target and neighbour distinct): S_small (batch 200 / k = 20: 28; batch 2,000: 1).
-  // Superbatches the host proves eviction-free run the grid-wide pass (global-memory
-  // hash) and use S, bounded by the grid-wide pass and a ~40 GB workspace budget.
-  int S_small = S;
-  for (int l = 1; l < L; ++l) {
-    const int64_t fit = (int64_t)kSeqCLMax * kSeqSlotsPerCTA * 9 / 10 / cap[l];
-    if (fit < S_small) S_small = fit < 1 ? 1 : (int)fit;
-  }
+  // Both cache passes keep their superbatch hash in global memory (r1: DSMEM, which capped
+  // S at 28 for batch 200 / k = 20 and at 1 for batch 2,000): S is bounded only by the
+  // grid-wide pass's block count and a ~40 GB budget for the S-proportional workspaces.
   {
     const int64_t HDp_ = (int64_t)H * (round4(d_n) + round4(d_e) + round4(d_t)), Dp_ = HDp_ / H;
     auto ws = [&](int64_t s) {  // device bytes that grow with S (both level sets)
@@ -849,13 +809,12 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
       }
       return b + mx * 4 * (2 * HDp_ + 2 * Dp_ + round4(d_n)) + mx * 2 * (HDp_ + Dp_ + 2 * round4(d_n));
     };
-    while (S > S_small && (ws(S) > (40ll << 30) || (int64_t)cap[1] * S > (int64_t)kSbhMaxBlocks * kSbhChunk)) --S;
+    while (S > 1 && (ws(S) > (40ll << 30) || (int64_t)cap[1] * S > (int64_t)kSbhMaxBlocks * kSbhChunk)) --S;
   }
   if ((int64_t)cap[1] * S > ((int64_t)1 << 26)) return TG_EINVAL;
   if (cudaSetDevice(ctx->device) != cudaSuccess) return TG_ECUDA;
   ctx->cfg = *cfg;
   ctx->S = S;
-  ctx->S_small = S_small;
   ctx->L = L;
   ctx->H = H;
   ctx->k = k;
@@ -1186,8 +1145,6 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
   if (!ctx->occ_h) {
     CK(cudaHostAlloc(&ctx->occ_h, (TG_MAX_LAYERS + 1) * sizeof(unsigned long long), cudaHostAllocMapped));
     memset(ctx->occ_h, 0, (TG_MAX_LAYERS + 1) * sizeof(unsigned long long));
-    CK(cudaHostAlloc(&ctx->size_h, (TG_MAX_LAYERS + 1) * sizeof(unsigned long long), cudaHostAllocMapped));
-    memset(ctx->size_h, 0, (TG_MAX_LAYERS + 1) * sizeof(unsigned long long));
   }
   CK(cudaDeviceSynchronize());
   ctx->loaded = true;
@@ -1209,12 +1166,9 @@ tg_status tg_cache_reset(tg_ctx* ctx, int64_t new_limit) {
     CK(cudaMemcpy(cd.state, st, sizeof(st), cudaMemcpyHostToDevice));
     ctx->idx_bound[l] = 0;
     if (ctx->occ_h) ctx->occ_h[l] = 0;
-    if (ctx->size_h) ctx->size_h[l] = 0;
-    ctx->ins_bound[l] = 0;
   }
   ctx->sb_count = 0;
   ctx->targets_issued = 0;
-  ctx->extra_keys = 0;
   CK(cudaMemset(ctx->cnt_total, 0, TG_NCOUNTERS * sizeof(long long)));
   CK(cudaMemset(ctx->cnt_sb, 0, (size_t)kMaxS * TG_NCOUNTERS * sizeof(long long)));
   CK(cudaMemset(ctx->err, 0, 2 * sizeof(int)));
@@ -1618,7 +1572,6 @@ void tg_free(tg_ctx* ctx) {
     if (e) cudaEventDestroy(e);
   if (ctx->fst) cudaStreamDestroy(ctx->fst);
   if (ctx->occ_h) cudaFreeHost(ctx->occ_h);
-  if (ctx->size_h) cudaFreeHost(ctx->size_h);
   if (ctx->stage) cudaFree(ctx->stage);
   delete ctx;
 }

@@ -131,7 +131,6 @@ struct CacheDev {
   // host-mapped report word: ((superbatch + 1) << 40) | occupied slots, written by
   // k_probe_pre, read by the host without synchronising (rebuild trigger bound)
   unsigned long long* occ_report;
-  unsigned long long* size_report;  // same format: live FIFO size at superbatch start
   long long report_sb;       // superbatch number of this launch (set per launch)
   // superbatch-scoped lookup hash in global memory (L2-resident), grid-wide eviction-free
   // CacheLookup pass (k_sbh_*): key -> min concatenated position j, then the ring slot of
