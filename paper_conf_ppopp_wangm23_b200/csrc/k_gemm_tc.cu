@@ -56,6 +56,20 @@ __host__ __device__ inline int tc_epc(int prec) {  // elements per 128 B
   return (prec == TG_PREC_BF16 || prec == TG_PREC_F16X3) ? 64 : 32;
 }
 __host__ __device__ inline int tc_planes(int prec) { return (prec == TG_PREC_TF32X3 || prec == TG_PREC_F16X3) ? 2 : 1; }
+// TMEM plan of the fp32-level modes (A in TMEM): accumulator buffers of [big | small]
+// (2 x round32(BN) columns) -- two (the epilogue drains one while the MMA fills the other)
+// when they leave room for >= 2 A stages of 64 columns, else one; returns the A stages that fit
+#ifndef TG_X3_NBUF_MAX
+#define TG_X3_NBUF_MAX 2
+#endif
+__host__ __device__ inline int tc_tmem_nbuf(int BN) {
+  const int buf = 2 * ((BN + 31) & ~31);
+  return (TG_X3_NBUF_MAX > 1 && 2 * buf + 2 * 64 <= 512) ? 2 : 1;
+}
+__host__ __device__ inline int tc_tmem_astages(int BN) {
+  const int buf = 2 * ((BN + 31) & ~31);
+  return (512 - tc_tmem_nbuf(BN) * buf) / 64;
+}
 
 // offset of 16-byte chunk c of row r inside a 128B-swizzled K-major tile
 __host__ __device__ inline unsigned sw128(int r, int c) {
@@ -95,9 +109,8 @@ static inline void tc_plan(int prec, int BN, int ln, bool generic, int* stages, 
   }
   int s = (int)((budget - (size_t)(d > 0 ? d : 0) * TC_STG_UNIT) / st);
   if (s > TC_MAXSTAGES) s = TC_MAXSTAGES;
-  if (tc_atmem(prec)) {  // TMEM: one [big | small] accumulator + 64 columns of A per stage
-    const int acc = 2 * ((BN + 31) & ~31);
-    const int sa = (512 - acc) / 64;
+  if (tc_atmem(prec)) {  // TMEM: [big | small] accumulator buffer(s) + 64 columns of A per stage
+    const int sa = tc_tmem_astages(BN);
     if (s > sa) s = sa;
   }
   *stages = s < 2 ? 2 : s;
@@ -456,7 +469,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   const int BNc = (BN + 31) & ~31;
   const uint32_t buf_cols = PLANES == 2 ? 2u * BNc : (uint32_t)tc_acc_cols(PREC);
   const uint32_t small_off = PLANES == 2 ? (uint32_t)BNc : 0u;
-  const uint32_t nbuf = (ATMEM || 4 * BNc > 512) ? 1u : 2u;
+  const uint32_t nbuf = ATMEM ? (uint32_t)tc_tmem_nbuf(BN) : (4 * BNc > 512 ? 1u : 2u);
   const uint32_t a_plane = TC_BM * 128;
   const uint32_t b_plane = (uint32_t)BN * 128;
   const uint32_t a_bytes = ATMEM ? 0u : PLANES * a_plane;  // A bytes at the head of a smem stage
