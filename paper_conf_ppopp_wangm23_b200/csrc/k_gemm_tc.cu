@@ -64,16 +64,25 @@ __host__ __device__ inline int tc_planes(int prec) { return (prec == TG_PREC_TF3
 #endif
 __host__ __device__ inline int tc_tmem_nbuf(int BN) {
   const int buf = 2 * ((BN + 31) & ~31);
-  return (TG_X3_NBUF_MAX > 1 && 2 * buf + 2 * 64 <= 512) ? 2 : 1;
+  return (TG_X3_NBUF_MAX > 1 && 2 * buf + 4 * 32 <= 512) ? 2 : 1;
 }
-__host__ __device__ inline int tc_tmem_astages(int BN) {
+__host__ __device__ inline int tc_tmem_astages(int BN) {  // A stages of 32 columns (64-byte k-blocks)
   const int buf = 2 * ((BN + 31) & ~31);
-  return (512 - tc_tmem_nbuf(BN) * buf) / 64;
+  return (512 - tc_tmem_nbuf(BN) * buf) / 32;
 }
 
 // offset of 16-byte chunk c of row r inside a 128B-swizzled K-major tile
 __host__ __device__ inline unsigned sw128(int r, int c) {
   return (unsigned)((r >> 3) * 1024 + (r & 7) * 128 + ((c ^ (r & 7)) << 4));
+}
+// ... inside a 64B-swizzled K-major tile (8-row atoms of 512 B; chunk c in [0, 4))
+__host__ __device__ inline unsigned sw64(int r, int c) {
+  return (unsigned)((r >> 3) * 512 + (r & 7) * 64 + ((c ^ ((r >> 1) & 3)) << 4));
+}
+// The fp32-level modes (A in TMEM) stage B in 64-byte k-blocks (tf32: 16, f16: 32 elements):
+// twice the pipeline stages in the same TMEM / shared memory as 128-byte k-blocks
+__host__ __device__ inline int tc_kb_bytes(int prec) {
+  return (prec == TG_PREC_TF32X3 || prec == TG_PREC_F16X3) ? 64 : 128;
 }
 
 // shared memory after the stages: barriers, then a 32 x 16 fp32 transpose
@@ -94,7 +103,7 @@ constexpr int TC_STG_UNIT = TC_BM * 128;
 constexpr int TC_PTR_BYTES = 2 * TC_BM * 8;  // the producers' row-pointer table
 static inline bool tc_atmem(int prec) { return tc_planes(prec) == 2; }  // A operand in TMEM
 static inline void tc_plan(int prec, int BN, int ln, bool generic, int* stages, int* stg) {
-  const size_t st = (size_t)tc_planes(prec) * ((tc_atmem(prec) ? 0 : (size_t)TC_BM * 128) + (size_t)BN * 128);
+  const size_t st = (size_t)tc_planes(prec) * ((tc_atmem(prec) ? 0 : (size_t)TC_BM * 128) + (size_t)BN * tc_kb_bytes(prec));
   const size_t budget = (tc_ctas_per_sm(prec) == 1 ? 205 * 1024 : 100 * 1024) - (ln ? TC_LN_BYTES : 0) -
                         (generic ? TC_PTR_BYTES : 0);
   int d = 0;  // 0: no room beside 2 stages -> the producers load synchronously
@@ -158,10 +167,11 @@ tg_status tc_prepare_weights(const float* W, int N, int K, int precision, TcWeig
     ntn = (N + x3_bn - 1) / x3_bn;
   int BN = (N + ntn - 1) / ntn;
   BN = (BN + 15) & ~15;
-  const int epc = tc_epc(precision);
+  const int kbb = tc_kb_bytes(precision);          // bytes of K per k-block row
+  const int epc = tc_epc(precision) * kbb / 128;   // elements per k-block row
   const int nkb = (K + epc - 1) / epc;
   const int planes = tc_planes(precision);
-  const size_t plane_bytes = (size_t)BN * 128;
+  const size_t plane_bytes = (size_t)BN * kbb;
   const size_t total = (size_t)ntn * nkb * planes * plane_bytes;
   std::vector<float> w((size_t)N * K);
   if (cudaMemcpy(w.data(), W, w.size() * 4, cudaMemcpyDeviceToHost) != cudaSuccess) return TG_ECUDA;
@@ -189,8 +199,8 @@ tg_status tc_prepare_weights(const float* W, int N, int K, int precision, TcWeig
       unsigned char* base = img.data() + ((size_t)tn * nkb + kb) * planes * plane_bytes;
       for (int r = 0; r < BN; ++r) {
         const int n = tn * BN + r;
-        for (int c = 0; c < 8; ++c) {
-          unsigned char* dst0 = base + sw128(r, c);
+        for (int c = 0; c < kbb / 16; ++c) {
+          unsigned char* dst0 = base + (kbb == 64 ? sw64(r, c) : sw128(r, c));
           if (precision == TG_PREC_F16X3) {
             uint16_t vh[8], vl[8];
             for (int e = 0; e < 8; ++e) {
@@ -260,6 +270,17 @@ __device__ __forceinline__ uint64_t umma_desc(uint32_t saddr) {
   d |= (uint64_t)(1024 >> 4) << 32;
   d |= (uint64_t)1 << 46;
   d |= (uint64_t)2 << 61;
+  return d;
+}
+
+__device__ __forceinline__ uint64_t umma_desc64(uint32_t saddr) {
+  // K-major, SWIZZLE_64B: SBO = 512 B between 8-row groups, layout type 4
+  uint64_t d = 0;
+  d |= (uint64_t)((saddr >> 4) & 0x3FFF);
+  d |= (uint64_t)1 << 16;
+  d |= (uint64_t)(512 >> 4) << 32;
+  d |= (uint64_t)1 << 46;
+  d |= (uint64_t)4 << 61;
   return d;
 }
 
@@ -471,10 +492,11 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   const uint32_t small_off = PLANES == 2 ? (uint32_t)BNc : 0u;
   const uint32_t nbuf = ATMEM ? (uint32_t)tc_tmem_nbuf(BN) : (4 * BNc > 512 ? 1u : 2u);
   const uint32_t a_plane = TC_BM * 128;
-  const uint32_t b_plane = (uint32_t)BN * 128;
+  const uint32_t b_plane = (uint32_t)BN * (ATMEM ? 64 : 128);
   const uint32_t a_bytes = ATMEM ? 0u : PLANES * a_plane;  // A bytes at the head of a smem stage
   const uint32_t stage_bytes = a_bytes + PLANES * b_plane;
-  const uint32_t a_tcol0 = nbuf * buf_cols;  // ATMEM: A stage s at TMEM column a_tcol0 + 64 s
+  // ATMEM: A stage s at TMEM columns a_tcol0 + 32 s: [hi 16 | lo 16] per 64-byte k-block
+  const uint32_t a_tcol0 = nbuf * buf_cols;
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + stages * stage_bytes);
   uint64_t* empty = full + TC_MAXSTAGES;
   uint64_t* tfull = empty + TC_MAXSTAGES;   // [2]
@@ -504,7 +526,8 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   if (tid == 0) {
     for (int s = 0; s < stages; ++s) {
       // arrivals: the A producer threads (256 generic, 128 streamed) + the TMA warp's expect_tx
-      mbar_init(&full[s], a_tma ? 1 : (generic ? TC_PROD_WARPS * 32 : TC_BM) + 1);
+      // (ATMEM tf32x3: each 64-byte k-block is produced by one half of the producers)
+      mbar_init(&full[s], a_tma ? 1 : ((generic && !(ATMEM && PREC == TG_PREC_TF32X3)) ? TC_PROD_WARPS * 32 : TC_BM) + 1);
       mbar_init(&empty[s], 1);         // MMA commit
     }
     for (int a = 0; a < 2; ++a) {
@@ -616,7 +639,9 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     // in registers (no shared-memory round trip, no producer barriers)
     const bool regpf = stg < 0;
     const int D = regpf ? 0 : stg;
-    const int upt = nkb * UPK;  // units per tile
+    // units (32 fp32 of each row) per tile; ATMEM k-blocks are 64 B (tf32 16, f16 32 elements)
+    constexpr int EPK = PREC == TG_PREC_F16X3 ? 32 : 16;
+    const int upt = ATMEM ? (nkb * EPK + 31) / 32 : nkb * UPK;
     auto pbar = [] { asm volatile("bar.sync 2, %0;\n" ::"n"(NPT) : "memory"); };
     float4 pf0[4], pf1[4];
     int pt = blockIdx.x, pu = 0;
@@ -707,14 +732,105 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       for (int i = 0; i < D; ++i) issue(i);
     }
     uint32_t gk = 0, gu = 0;
-    for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    if (ATMEM) {
+      // unit u of a tile feeds k-blocks 2u (thread half 0) and 2u + 1 (half 1) in tf32x3 --
+      // the two halves fill different stages concurrently -- or k-block u (both halves,
+      // 8 TMEM columns each) in f16x3
+      const uint32_t lanes = (uint32_t)((warp & 3) * 32) << 16;
+      int tseq = 0;
+      for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++tseq) {
+        if (D == 0) rows_of(t);
+        for (int u = 0; u < upt; ++u, ++gu) {
+#ifdef TG_TC_TRACE
+          const bool tr5 = tg_tct_nk[2] == 5 && tseq == 0 && tid == 0 && u < 8;
+#define TR5(i) do { if (tr5) TCT(8 + 6 * u + (i), clock64()); } while (0)
+#else
+#define TR5(i) do { } while (0)
+#endif
+          TR5(0);
+          float4 x[4];  // fp32 chunks 4 ph .. 4 ph + 3 of unit u of row prow
+          const int slot = D > 0 ? (int)(gu % (uint32_t)D) : 0;
+          if (D <= 0) {
+#pragma unroll
+            for (int i = 0; i < 4; ++i)
+              x[i] = irv ? tc_load4(g, ir0, ir1, u * 32 + 4 * (4 * ph + i)) : make_float4(0.f, 0.f, 0.f, 0.f);
+          } else {
+            if (D == 1) asm volatile("cp.async.wait_group 0;\n" ::: "memory");
+            else if (D == 2) asm volatile("cp.async.wait_group 1;\n" ::: "memory");
+            else if (D == 3) asm volatile("cp.async.wait_group 2;\n" ::: "memory");
+            else asm volatile("cp.async.wait_group 3;\n" ::: "memory");
+            pbar();  // every producer's copies of this unit have landed
+            TR5(1);
+            const unsigned char* src = sring + (size_t)slot * TC_STG_UNIT + prow * 128;
+#pragma unroll
+            for (int i = 0; i < 4; ++i)
+              x[i] = *reinterpret_cast<const float4*>(src + (((4 * ph + i) ^ (prow & 7)) << 4));
+            pbar();  // every producer has read the slot: it may be refilled
+            TR5(2);
+            issue(slot);  // unit gu + D
+          }
+          const int kbq = EPK == 16 ? 2 * u + ph : u;
+          if (kbq >= nkb) continue;
+          const uint32_t g2 = (uint32_t)tseq * (uint32_t)nkb + (uint32_t)kbq;
+          const int s = (int)(g2 % (uint32_t)stages);
+          TR5(3);
+          mbar_wait(&empty[s], ((g2 / (uint32_t)stages) & 1) ^ 1);
+          asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
+          TR5(4);
+          const uint32_t tq = tmem + lanes + a_tcol0 + 32u * (uint32_t)s;
+          if (PREC == TG_PREC_F16X3) {
+            uint32_t hv[8], lv[8];
+            bool big = false;
+#pragma unroll
+            for (int e = 0; e < 8; ++e) {
+              const float x0 = (&x[e >> 1].x)[2 * (e & 1)], x1 = (&x[e >> 1].x)[2 * (e & 1) + 1];
+              const __half2 hh = __floats2half2_rn(x0, x1);
+              const float2 hf = __half22float2(hh);
+              const __half2 ll = __floats2half2_rn(x0 - hf.x, x1 - hf.y);
+              big |= !(fabsf(x0) < 65504.f) | !(fabsf(x1) < 65504.f);
+              hv[e] = *reinterpret_cast<const uint32_t*>(&hh);
+              lv[e] = *reinterpret_cast<const uint32_t*>(&ll);
+            }
+            if (big && g.err) atomicOr(g.err, kErrF16Range);
+            tmem_st8(tq + 8u * (uint32_t)ph, hv);
+            tmem_st8(tq + 16u + 8u * (uint32_t)ph, lv);
+          } else {
+            uint32_t hv[16], lv[16];
+#pragma unroll
+            for (int e = 0; e < 16; ++e) {
+              const float xv = (&x[e >> 2].x)[e & 3];
+              const float hi = rna_tf32_fast(xv);
+              hv[e] = __float_as_uint(hi);
+              lv[e] = __float_as_uint(rna_tf32_fast(xv - hi));
+            }
+            tmem_st16(tq, hv);
+            tmem_st16(tq + 16u, lv);
+          }
+          asm volatile("tcgen05.wait::st.sync.aligned;\n" ::: "memory");
+          asm volatile("tcgen05.fence::before_thread_sync;\n" ::: "memory");
+          TR5(5);
+          mbar_arrive(&full[s]);
+        }
+#undef TR5
+      }
+    }
+    for (int t = blockIdx.x; t < (ATMEM ? 0 : ntiles); t += gridDim.x) {
       if (D == 0 && !regpf) rows_of(t);  // no room for staging (widest N tiles): blocking loads
       for (int kb = 0; kb < nkb; ++kb, ++gk) {
         const int s = gk % stages;
         mbar_wait(&empty[s], ((gk / stages) & 1) ^ 1);
-        if (ATMEM) asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
+#ifdef TG_TC_TRACE
+        if (t == (int)blockIdx.x && tid == 0 && tg_tct_nk[2] == 1) TCT(8 + kb, clock64());
+        if (t == (int)blockIdx.x && tid == 0 && tg_tct_nk[2] == 3 && kb < 16) TCT(24 + kb, clock64());
+#endif
         unsigned char* sA = smem + s * stage_bytes;
         bool big = false;
+#ifdef TG_TC_TRACE
+        if (tg_tct_nk[2] == 4) {  // debug: MMA/TMA-bound cadence (producer does no work; results invalid)
+          mbar_arrive(&full[s]);
+          continue;
+        }
+#endif
 #pragma unroll
         for (int h = 0; h < UPK; ++h, ++gu) {
           float4 x[4];  // fp32 chunks 4 ph .. 4 ph + 3 of this unit of row prow
@@ -744,39 +860,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
             pbar();  // every producer has read the slot: it may be refilled
             issue(slot);  // unit gu + D
           }
-          if (ATMEM) {
-            // columns of this unit: tf32 32 elements = 32 columns (thread half ph: 16);
-            // f16 32 elements = 16 columns (thread half ph: 8); lanes = rows (warp quadrant)
-            const uint32_t tq = tmem + ((uint32_t)((warp & 3) * 32) << 16) + a_tcol0 + 64u * (uint32_t)s;
-            if (PREC == TG_PREC_F16X3) {
-              uint32_t hv[8], lv[8];
-#pragma unroll
-              for (int e = 0; e < 8; ++e) {
-                const float x0 = (&x[e >> 1].x)[2 * (e & 1)], x1 = (&x[e >> 1].x)[2 * (e & 1) + 1];
-                const __half2 hh = __floats2half2_rn(x0, x1);
-                const float2 hf = __half22float2(hh);
-                const __half2 ll = __floats2half2_rn(x0 - hf.x, x1 - hf.y);
-                big |= !(fabsf(x0) < 65504.f) | !(fabsf(x1) < 65504.f);
-                hv[e] = *reinterpret_cast<const uint32_t*>(&hh);
-                lv[e] = *reinterpret_cast<const uint32_t*>(&ll);
-              }
-              const uint32_t col = (uint32_t)(h * 16 + ph * 8);
-              tmem_st8(tq + col, hv);
-              tmem_st8(tq + 32u + col, lv);
-            } else {
-              uint32_t hv[16], lv[16];
-#pragma unroll
-              for (int e = 0; e < 16; ++e) {
-                const float xv = (&x[e >> 2].x)[e & 3];
-                const float hi = rna_tf32_fast(xv);
-                hv[e] = __float_as_uint(hi);
-                lv[e] = __float_as_uint(rna_tf32_fast(xv - hi));
-              }
-              const uint32_t col = (uint32_t)(ph * 16);
-              tmem_st16(tq + col, hv);
-              tmem_st16(tq + 32u + col, lv);
-            }
-          } else if (PREC == TG_PREC_F16X3) {
+          if (PREC == TG_PREC_F16X3) {
 #pragma unroll
             for (int jj = 0; jj < 2; ++jj) {  // fp16 chunk j = 2 ph + jj <- fp32 chunks 2j, 2j + 1
               const float xs[8] = {x[2 * jj].x, x[2 * jj].y, x[2 * jj].z, x[2 * jj].w,
@@ -830,12 +914,11 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           }
         }
         if (PREC == TG_PREC_F16X3 && big && g.err) atomicOr(g.err, kErrF16Range);
-        if (ATMEM) {
-          asm volatile("tcgen05.wait::st.sync.aligned;\n" ::: "memory");
-          asm volatile("tcgen05.fence::before_thread_sync;\n" ::: "memory");
-        } else {
-          asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");  // generic -> async proxy
-        }
+        asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");  // generic -> async proxy
+#ifdef TG_TC_TRACE
+        if (t == (int)blockIdx.x && tid == 0 && tg_tct_nk[2] == 2) TCT(8 + kb, clock64());
+        if (t == (int)blockIdx.x && tid == 0 && tg_tct_nk[2] == 3 && kb < 16) TCT(40 + kb, clock64());
+#endif
         mbar_arrive(&full[s]);
       }
     }
@@ -881,19 +964,25 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         for (int kb = 0; kb < nkb; ++kb, ++gk) {
           const int s = gk % stages;
           mbar_wait(&full[s], (gk / stages) & 1);
-          if (tc == 0) TCT(8 + kb, clock64());
+#ifdef TG_TC_TRACE
+          if (tc == 0 && (tg_tct_nk[2] == 0 || tg_tct_nk[2] == 4)) TCT(8 + kb, clock64());
+          if (tc == 0 && tg_tct_nk[2] == 3 && kb < 16) TCT(8 + kb, clock64());
+#endif
           asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");  // cp.async A -> tensor core
           asm volatile("tcgen05.fence::after_thread_sync;\n");
           const uint32_t aH = smem_u32(smem + s * stage_bytes);
           const uint32_t bH = aH + a_bytes;
-          const uint32_t aT = tmem + a_tcol0 + 64u * (uint32_t)s;  // ATMEM: A planes at aT, aT + 32
+          const uint32_t aT = tmem + a_tcol0 + 32u * (uint32_t)s;  // ATMEM: A planes at aT, aT + 16
 #pragma unroll
           for (int kk = 0; kk < 4; ++kk) {  // 4 MMAs of 32 bytes of K per 128B k-block
             const uint32_t acc0 = (kb > 0 || kk > 0) ? 1u : 0u;
-            if (ATMEM) {  // 8 TMEM columns of A per MMA; correction terms into `small`
-              mma_issue_ts<PREC>(dtm, aT + kk * 8, umma_desc(bH + kk * 32), idesc, acc0);
-              mma_issue_ts<PREC>(dtm + small_off, aT + kk * 8, umma_desc(bH + b_plane + kk * 32), idesc, acc0);
-              mma_issue_ts<PREC>(dtm + small_off, aT + 32 + kk * 8, umma_desc(bH + kk * 32), idesc, 1u);
+            if (ATMEM) {  // 64-byte k-block: 2 MMAs of 32 bytes of K, 8 TMEM columns of A each;
+              // B 64B-swizzled; correction products into `small`
+              if (kk < 2) {
+                mma_issue_ts<PREC>(dtm, aT + kk * 8, umma_desc64(bH + kk * 32), idesc, acc0);
+                mma_issue_ts<PREC>(dtm + small_off, aT + kk * 8, umma_desc64(bH + b_plane + kk * 32), idesc, acc0);
+                mma_issue_ts<PREC>(dtm + small_off, aT + 16 + kk * 8, umma_desc64(bH + kk * 32), idesc, 1u);
+              }
               continue;
             }
             mma_issue<PREC>(dtm, umma_desc(aH + kk * 32), umma_desc(bH + kk * 32), idesc, acc0);
@@ -1167,7 +1256,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
 
 static size_t tc_smem(int prec, int BN, int stages, int stg, int ln = 0) {
   const size_t planes = tc_planes(prec);
-  size_t s = 1024 + (size_t)stages * planes * ((tc_atmem(prec) ? 0 : (size_t)TC_BM * 128) + (size_t)BN * 128) +
+  size_t s = 1024 + (size_t)stages * planes * ((tc_atmem(prec) ? 0 : (size_t)TC_BM * 128) + (size_t)BN * tc_kb_bytes(prec)) +
              TC_BAR_BYTES + TC_EPI_BYTES +
              (ln ? TC_LN_BYTES : 0) + (size_t)(stg > 0 ? stg : 0) * TC_STG_UNIT + (stg > 0 ? TC_PTR_BYTES : 0);
   // tf32x3: one CTA per SM (it allocates all 512 TMEM columns; a second
@@ -1222,7 +1311,11 @@ void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaSt
   tc_plan(precision, w.BN, ln, generic, &stages, &stg);
   const size_t smem = tc_smem(precision, w.BN, stages, stg, ln);
   const int tiles = ((g.m_max + TC_BM - 1) / TC_BM) * w.ntn;
-  int slots = 148 * tc_ctas_per_sm(precision);
+  static const int grid_cap = [] {  // TG_GEMM_GRID: cap on persistent CTAs (experiments)
+    const char* e = getenv("TG_GEMM_GRID");
+    return e ? atoi(e) : 148;
+  }();
+  int slots = grid_cap * tc_ctas_per_sm(precision);
   if (ln) slots = slots / w.ntn * w.ntn;  // whole clusters; a cluster walks the M tiles in lockstep
   int grid = tiles < slots ? tiles : slots;
   if (grid < 1) grid = 1;

@@ -61,7 +61,15 @@ for i, nm in names.items():
     if v.size:
         print(f"{nm:11s} median {us(np.median(v)):7.2f} us  min {us(v.min()):7.2f}  max {us(v.max()):7.2f}")
 print(f"M {T[0, 63]}")
-kb = [i for i in range(8, 55) if (T[:, i] != 0).any()]
+if a.mode == 3:  # one run: MMA landing (8+kb), producer empty release (24+kb), producer arrive (40+kb)
+    for nm, base in (("mma_full", 8), ("prod_empty", 24), ("prod_arrive", 40)):
+        med = [us(np.median(rel[:, base + i])) for i in range(16) if (T[:, base + i] != 0).all()]
+        print(f"{nm:12s}", " ".join(f"{x:.2f}" for x in med))
+if a.mode == 5:  # producer phases per unit: [start, staged, read+issue, converted, empty ok, stored]
+    for u in range(8):
+        v = [us(np.median(rel[:, 8 + 6 * u + i])) for i in range(6)]
+        print(f"unit {u}: " + " ".join(f"{x:7.2f}" for x in v) + "   d: " + " ".join(f"{v[i+1]-v[i]:5.2f}" for i in range(5)))
+kb = [i for i in range(8, 55) if (T[:, i] != 0).any()] if a.mode not in (3, 5) else []
 if kb:
     med = [us(np.median(rel[:, i])) for i in kb]
     print("k-block landed (median us):", " ".join(f"{x:.2f}" for x in med))
