@@ -100,12 +100,12 @@ constexpr int TC_LN_BYTES = (2 * 128 + 2 * TC_LN_MAXTN * 128) * 16 + 4 * 256 * 4
 // `stg` staging units of 16 KB (its cp.async look-ahead ring, up to 4 units) -- as many
 // staging units as fit beside 2 stages, then as many stages as fit beside those.
 constexpr int TC_STG_UNIT = TC_BM * 128;
-constexpr int TC_PTR_BYTES = 2 * TC_BM * 8;  // the producers' row-pointer table
+constexpr int TC_PTR_BYTES = 2 * TC_BM * 8 + 64;  // the producers' row-pointer table + staging mbarriers
 static inline bool tc_atmem(int prec) { return tc_planes(prec) == 2; }  // A operand in TMEM
 static inline void tc_plan(int prec, int BN, int ln, bool generic, int* stages, int* stg) {
   const size_t st = (size_t)tc_planes(prec) * ((tc_atmem(prec) ? 0 : (size_t)TC_BM * 128) + (size_t)BN * tc_kb_bytes(prec));
   const size_t budget = (tc_ctas_per_sm(prec) == 1 ? 205 * 1024 : 100 * 1024) - (ln ? TC_LN_BYTES : 0) -
-                        (generic ? TC_PTR_BYTES : 0);
+                        (generic ? TC_PTR_BYTES + 1024 : 0);
   int d = 0;  // 0: no room beside 2 stages -> the producers load synchronously
   static const int d_env = [] {  // TG_GEMM_STG: cap on staging units (A/B experiments)
     const char* e = getenv("TG_GEMM_STG");
@@ -522,12 +522,16 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   const int nkb = w.nkb;
   // the generic fp32 A producer (all TC_PROD_WARPS warps) unless A arrives by TMA, streams raw
   // (one-pass tf32) or as a dense bf16 activation (128 threads, warps 0-3)
-  const bool generic = !a_tma && PREC != TG_PREC_TF32 && !(PREC == TG_PREC_BF16 && g.a_h);
+  // a_tma == 2 (fp32-level modes, dense fp32 A): the producers' staging ring is filled by TMA
+  // 2D tile loads (box 32 fp32 x 128 rows, 128B swizzle = the ring's layout) instead of
+  // per-thread cp.async copies
+  const bool stage_tma = ATMEM && a_tma == 2;
+  const bool generic = (!a_tma || stage_tma) && PREC != TG_PREC_TF32 && !(PREC == TG_PREC_BF16 && g.a_h);
   if (tid == 0) {
     for (int s = 0; s < stages; ++s) {
       // arrivals: the A producer threads (256 generic, 128 streamed) + the TMA warp's expect_tx
       // (ATMEM tf32x3: each 64-byte k-block is produced by one half of the producers)
-      mbar_init(&full[s], a_tma ? 1 : ((generic && !(ATMEM && PREC == TG_PREC_TF32X3)) ? TC_PROD_WARPS * 32 : TC_BM) + 1);
+      mbar_init(&full[s], (a_tma && !stage_tma) ? 1 : ((generic && !(ATMEM && PREC == TG_PREC_TF32X3)) ? TC_PROD_WARPS * 32 : TC_BM) + 1);
       mbar_init(&empty[s], 1);         // MMA commit
     }
     for (int a = 0; a < 2; ++a) {
@@ -558,7 +562,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   const int ntiles = tiles_m * w.ntn;  // CTAs past ntiles run no tile and fall through to the end
   if (tid == 0) TCT(2, clock64());
 
-  if (warp < TC_PROD_WARPS && (a_tma || (!generic && warp >= 4))) {
+  if (warp < TC_PROD_WARPS && ((a_tma && !stage_tma) || (!generic && warp >= 4))) {
     // A arrives by TMA (issued by warp 4 with B): nothing to produce here
   } else if (warp < TC_PROD_WARPS && PREC == TG_PREC_TF32) {
     // ===================== A producers, streamed: raw fp32 rows go straight into
@@ -633,8 +637,11 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     constexpr int UPK = EPC / 32;
     constexpr int NPT = TC_PROD_WARPS * 32;
     const int prow = tid & (TC_BM - 1), ph = tid >> 7;  // row, column half
-    unsigned char* sring = smem + stages * stage_bytes + TC_BAR_BYTES + TC_EPI_BYTES + (g.ln ? TC_LN_BYTES : 0);
+    // staging ring at a 1024-byte boundary: TMA's 128-byte swizzle is a function of the address
+    unsigned char* sring =
+        smem + ((stages * stage_bytes + TC_BAR_BYTES + TC_EPI_BYTES + (g.ln ? TC_LN_BYTES : 0) + 1023u) & ~1023u);
     const float** sptr = reinterpret_cast<const float**>(sring + (size_t)(stg > 0 ? stg : 0) * TC_STG_UNIT);  // [2][128]
+    uint64_t* sbar = reinterpret_cast<uint64_t*>(sptr + 2 * TC_BM);  // [4] staging slots (stage_tma)
     // stg < 0: no staging ring -- each thread prefetches its own row half two units ahead
     // in registers (no shared-memory round trip, no producer barriers)
     const bool regpf = stg < 0;
@@ -699,6 +706,28 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     };
     const void* dummy = w.hi;  // valid global address for zero-byte (zero-fill) copies
     auto issue = [&](int slot) {
+      if (stage_tma) {  // one thread: TMA tile (32 fp32 x 128 rows) of dense A into the slot
+        if (it_t < ntiles) {
+          if (tid == 0) {
+            // the producers' generic reads of this slot (ordered by named barrier 2) before the
+            // async-proxy (TMA) write that refills it
+            asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
+            const uint32_t bar = smem_u32(&sbar[slot]);
+            asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(bar), "r"(TC_STG_UNIT)
+                         : "memory");
+            asm volatile(
+                "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], "
+                "[%4];\n" ::"r"(smem_u32(sring + (size_t)slot * TC_STG_UNIT)),
+                "l"(reinterpret_cast<uint64_t>(&tmA)), "r"(it_u * 32), "r"((it_t / w.ntn) * TC_BM), "r"(bar)
+                : "memory");
+          }
+          if (++it_u == upt) {
+            it_u = 0;
+            it_t += gridDim.x;
+          }
+        }
+        return;
+      }
       if (it_t < ntiles) {
         unsigned char* base = sring + (size_t)slot * TC_STG_UNIT;
         const int q = lane & 3;
@@ -727,7 +756,14 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       }
       asm volatile("cp.async.commit_group;\n" ::: "memory");  // (empty past the last tile)
     };
-    if (D > 0) {  // (regpf: D = 0)
+    if (stage_tma) {
+      if (tid == 0) {
+        for (int i = 0; i < D; ++i) mbar_init(&sbar[i], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+      }
+      pbar();
+      for (int i = 0; i < D; ++i) issue(i);
+    } else if (D > 0) {  // (regpf: D = 0)
       if (it_t < ntiles) publish(it_t);
       for (int i = 0; i < D; ++i) issue(i);
     }
@@ -755,11 +791,15 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
             for (int i = 0; i < 4; ++i)
               x[i] = irv ? tc_load4(g, ir0, ir1, u * 32 + 4 * (4 * ph + i)) : make_float4(0.f, 0.f, 0.f, 0.f);
           } else {
-            if (D == 1) asm volatile("cp.async.wait_group 0;\n" ::: "memory");
-            else if (D == 2) asm volatile("cp.async.wait_group 1;\n" ::: "memory");
-            else if (D == 3) asm volatile("cp.async.wait_group 2;\n" ::: "memory");
-            else asm volatile("cp.async.wait_group 3;\n" ::: "memory");
-            pbar();  // every producer's copies of this unit have landed
+            if (stage_tma) {
+              mbar_wait(&sbar[slot], (gu / (uint32_t)D) & 1);  // the unit's TMA tile has landed
+            } else {
+              if (D == 1) asm volatile("cp.async.wait_group 0;\n" ::: "memory");
+              else if (D == 2) asm volatile("cp.async.wait_group 1;\n" ::: "memory");
+              else if (D == 3) asm volatile("cp.async.wait_group 2;\n" ::: "memory");
+              else asm volatile("cp.async.wait_group 3;\n" ::: "memory");
+              pbar();  // every producer's copies of this unit have landed
+            }
             TR5(1);
             const unsigned char* src = sring + (size_t)slot * TC_STG_UNIT + prow * 128;
 #pragma unroll
@@ -936,8 +976,8 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           const unsigned char* src =
               reinterpret_cast<const unsigned char*>(w.hi) + ((size_t)tn * nkb + kb) * PLANES * b_plane;
           if (gk == 0) TCT(4, clock64());
-          mbar_expect_tx(&full[s], PLANES * b_plane + (a_tma ? a_plane : 0u));
-          if (a_tma) {  // A tile [128 rows x 128 B] of the dense activation, 128B-swizzled by TMA
+          mbar_expect_tx(&full[s], PLANES * b_plane + ((a_tma && !stage_tma) ? a_plane : 0u));
+          if (a_tma && !stage_tma) {  // A tile [128 rows x 128 B] of the dense activation, 128B-swizzled by TMA
             // k-blocks >= a2_kb0 come from a second activation (columns a2_x0 + ...)
             const bool second = kb >= a2_kb0;
             const int x = second ? a2_x0 + (kb - a2_kb0) * EPC : kb * EPC, y = (t / w.ntn) * TC_BM;
@@ -1258,7 +1298,7 @@ static size_t tc_smem(int prec, int BN, int stages, int stg, int ln = 0) {
   const size_t planes = tc_planes(prec);
   size_t s = 1024 + (size_t)stages * planes * ((tc_atmem(prec) ? 0 : (size_t)TC_BM * 128) + (size_t)BN * tc_kb_bytes(prec)) +
              TC_BAR_BYTES + TC_EPI_BYTES +
-             (ln ? TC_LN_BYTES : 0) + (size_t)(stg > 0 ? stg : 0) * TC_STG_UNIT + (stg > 0 ? TC_PTR_BYTES : 0);
+             (ln ? TC_LN_BYTES : 0) + (size_t)(stg > 0 ? stg : 0) * TC_STG_UNIT + (stg > 0 ? TC_PTR_BYTES + 1024 : 0);
   // tf32x3: one CTA per SM (it allocates all 512 TMEM columns; a second
   // co-resident CTA would block in tcgen05.alloc until the first one exits).
   const size_t one_per_sm = 120 * 1024;
@@ -1299,16 +1339,18 @@ void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaSt
                     const TcTensorA* ta2, int a2_kb0, int a2_x0) {
   static const CUtensorMap zero_map{};
   const CUtensorMap& tm = (ta && ta->valid) ? ta->map : zero_map;
-  const int a_tma = (ta && ta->valid) ? 1 : 0;
+  int a_tma = (ta && ta->valid) ? 1 : 0;
+  if (a_tma && tc_atmem(precision)) a_tma = 2;  // fp32-level modes: the map feeds the producers' staging ring
   const bool two = a_tma && ta2 && ta2->valid;
   const CUtensorMap& tm2 = two ? ta2->map : zero_map;
   if (!two) a2_kb0 = 1 << 30;
   const int ln = g.ln ? 1 : 0;
   // the generic fp32 A producer (cp.async staging) runs unless A comes by TMA, as raw fp32
   // (one-pass tf32) or as a dense bf16 activation
-  const bool generic = !a_tma && precision != TG_PREC_TF32 && !(precision == TG_PREC_BF16 && g.a_h);
+  const bool generic = (!a_tma || a_tma == 2) && precision != TG_PREC_TF32 && !(precision == TG_PREC_BF16 && g.a_h);
   int stages = 2, stg = 0;
   tc_plan(precision, w.BN, ln, generic, &stages, &stg);
+  if (a_tma == 2 && stg <= 0) a_tma = 0;  // no staging ring: per-thread loads
   const size_t smem = tc_smem(precision, w.BN, stages, stg, ln);
   const int tiles = ((g.m_max + TC_BM - 1) / TC_BM) * w.ntn;
   static const int grid_cap = [] {  // TG_GEMM_GRID: cap on persistent CTAs (experiments)
@@ -1369,7 +1411,7 @@ void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaSt
       cudaFuncSetAttribute(k_gemm_tc<TG_PREC_F16X3>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       set = smem;
     }
-    launch_k(k_gemm_tc<TG_PREC_F16X3>, dim3(grid), dim3(TC_THREADS), smem, st, g, w, stages, stg, tm, 0, tm2,
+    launch_k(k_gemm_tc<TG_PREC_F16X3>, dim3(grid), dim3(TC_THREADS), smem, st, g, w, stages, stg, tm, a_tma, tm2,
              1 << 30, 0);
   } else {
     static size_t set = 0;
@@ -1377,7 +1419,7 @@ void launch_gemm_tc(const GemmArgs& g, const TcWeights& w, int precision, cudaSt
       cudaFuncSetAttribute(k_gemm_tc<TG_PREC_TF32X3>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       set = smem;
     }
-    launch_k(k_gemm_tc<TG_PREC_TF32X3>, dim3(grid), dim3(TC_THREADS), smem, st, g, w, stages, stg, tm, 0, tm2,
+    launch_k(k_gemm_tc<TG_PREC_TF32X3>, dim3(grid), dim3(TC_THREADS), smem, st, g, w, stages, stg, tm, a_tma, tm2,
              1 << 30, 0);
   }
 }

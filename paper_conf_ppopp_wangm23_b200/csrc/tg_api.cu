@@ -82,6 +82,7 @@ struct tg_ctx {
   int ld_ch = 0, ld_rh = 0, ld_z = 0;
   int dpa = 0;  // BF16 merge-FFN input row [LN(y) (Dp) | 0 | h at dpa = round8(Dp) (16-byte aligned) | 0]
   TcTensorA ta_c, ta_rh, ta_z;  // TMA tensor maps of the bf16 activations (dense GEMM A operands)
+  TcTensorA ta_c32, ta_z32;     // fp32-level modes: fp32 c and z, feeding the GEMM producers' staging
   AttnMaps am[2][TG_MAX_LAYERS + 1]{};  // per set and level l: TMA row-gather maps (h rows, E rows, Phi rows)
   int cur_set = 0;
   // Phi rows per set: [table (W rows) | direct rows of level 1 | level 2 | ...] (k_phi_rows, front stream)
@@ -268,6 +269,7 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   a.nb_hidx = lv.nb_hidx;
   a.phi_row0 = ctx->phi_pre ? ctx->phi_row0[l] : -1;
   const bool bfa = ctx->cfg.precision == TG_PREC_BF16;  // bf16 activations between the GEMMs
+  const bool x3 = ctx->cfg.precision == TG_PREC_TF32X3 || ctx->cfg.precision == TG_PREC_F16X3;
   // TG_LN_FUSE=1: LayerNorm in G2's epilogue (thread-block clusters, DSMEM statistics);
   // measured slower end to end than G2 + k_layernorm, so off by default
   static const bool ln_fuse_env = [] {
@@ -379,7 +381,7 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   {
     Prof pf(ctx, TG_ST_PROJ_V, st);
     if (fuse) launch_gemm_tc(g2, w.tcFa, ctx->cfg.precision, st, &ctx->ta_c, &ctx->ta_rh, w.fa_kb0, ctx->dpa);
-    else if (tc) launch_gemm_tc(g2, w.tcF, ctx->cfg.precision, st, bfa ? &ctx->ta_c : nullptr);
+    else if (tc) launch_gemm_tc(g2, w.tcF, ctx->cfg.precision, st, bfa ? &ctx->ta_c : (x3 ? &ctx->ta_c32 : nullptr));
     else launch_gemm_simt(g2, st);
   }
   TRY(launched(ctx));
@@ -437,7 +439,7 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   }
   {
     Prof pf(ctx, TG_ST_FFN2, st);
-    if (tc) launch_gemm_tc(g4, w.tcW2, ctx->cfg.precision, st, bfa ? &ctx->ta_z : nullptr);
+    if (tc) launch_gemm_tc(g4, w.tcW2, ctx->cfg.precision, st, bfa ? &ctx->ta_z : (x3 ? &ctx->ta_z32 : nullptr));
     else launch_gemm_simt(g4, st);
   }
   return launched(ctx);
@@ -1089,6 +1091,10 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     TRY(tc_make_tensor_a(ctx->rh_h, 2, ctx->ld_rh, maxC, &ctx->ta_rh));
     TRY(tc_make_tensor_a(ctx->z_h, 2, ctx->ld_z, maxC, &ctx->ta_z));
   }
+  if (cfg->precision == TG_PREC_TF32X3 || cfg->precision == TG_PREC_F16X3) {
+    TRY(tc_make_tensor_a(ctx->c, 4, HDp, maxC, &ctx->ta_c32));
+    TRY(tc_make_tensor_a(ctx->z, 4, dnp, maxC, &ctx->ta_z32));
+  }
   // Phi rows of dt >= W computed ahead on the front stream into a per-set buffer that follows a
   // copy of the table, so the attention gathers every Phi row from one tensor (dense row index
   // W + q*k + m per level; skipped when the buffers would exceed 16 GB: in-kernel Phi instead)
@@ -1545,7 +1551,8 @@ tg_status tg_gemm(tg_ctx* ctx, int32_t precision, int32_t M, int32_t N, int32_t 
       w = &ctx->gemm_cache.back().w;
     }
     TcTensorA ta;  // dense fp32 A via TMA in the one-pass tf32 mode
-    if (precision == TG_PREC_TF32 && M > 0) TRY(tc_make_tensor_a(A, 4, K, M, &ta));
+    if ((precision == TG_PREC_TF32 || precision == TG_PREC_TF32X3 || precision == TG_PREC_F16X3) && M > 0)
+      TRY(tc_make_tensor_a(A, 4, K, M, &ta));  // tf32: the MMA's A; fp32-level: the producers' staging
     launch_gemm_tc(g, *w, precision, st, ta.valid ? &ta : nullptr);
   }
   cudaError_t e = cudaGetLastError();
