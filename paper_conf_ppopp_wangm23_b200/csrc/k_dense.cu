@@ -98,7 +98,8 @@ void launch_gemm_simt(const GemmArgs& g, cudaStream_t st) {
 // mean and biased variance over the D valid columns, eps 1e-5. Warp per row;
 // per-column parameters (gamma, beta, valid weight, Phi(0) block of q) are
 // staged in shared memory once per CTA; the grid is one resident wave that
-// strides over the rows. Outputs: fp32 r [M x Dp] and/or the bf16 merge-FFN
+// strides over the rows. Outputs: fp32 r [M x (Dp + dnp)] = [LN(y) | h^(l-1)] (the
+// dense A operand of the merge FFN, Eq. 7) and/or the bf16 merge-FFN
 // input row rh = [LN(y) (Dp) | 0 | h^(l-1) at rh_off (16-byte aligned) | 0] (Eq. 7).
 constexpr int kLnMaxD4 = 256;  // Dp <= 1024 (checked at model load)
 __global__ void __launch_bounds__(256, 4)
@@ -106,6 +107,7 @@ __global__ void __launch_bounds__(256, 4)
                 const float* __restrict__ gamma, const float* __restrict__ beta, const int* __restrict__ m_dev,
                 const float* const* __restrict__ hs_rows, const float* __restrict__ phi0,
                 unsigned short* __restrict__ rh, int ldrh, int rh_off) {
+  const int ldr = Dp + dnp;
   __shared__ float4 s_g[kLnMaxD4], s_b[kLnMaxD4], s_w[kLnMaxD4], s_q[kLnMaxD4];
   const int D4 = Dp >> 2;
   const int s1 = dnp, s2 = dnp + dep;
@@ -169,7 +171,7 @@ __global__ void __launch_bounds__(256, 4)
         const float4 g = s_g[q], b = s_b[q];  // zero on padded columns -> output 0 there
         const float4 o4 = make_float4(fmaf((v[j].x - mu) * rstd, g.x, b.x), fmaf((v[j].y - mu) * rstd, g.y, b.y),
                                       fmaf((v[j].z - mu) * rstd, g.z, b.z), fmaf((v[j].w - mu) * rstd, g.w, b.w));
-        if (r) reinterpret_cast<float4*>(r + (size_t)row * Dp)[q] = o4;
+        if (r) reinterpret_cast<float4*>(r + (size_t)row * ldr)[q] = o4;
         if (rh) {
           __nv_bfloat162 lo = __floats2bfloat162_rn(o4.x, o4.y), hi = __floats2bfloat162_rn(o4.z, o4.w);
           uint2 pk;
@@ -179,6 +181,8 @@ __global__ void __launch_bounds__(256, 4)
         }
       }
     }
+    if (r)  // h^(l-1) after LN(y): the merge FFN's [LN(y) | h] row is dense
+      for (int q = lane; q < nh4; q += 32) reinterpret_cast<float4*>(r + (size_t)row * ldr + Dp)[q] = hr[q];
     if (rh) {  // [Dp, ldrh): zeros, h^(l-1) at rh_off, zeros
       const int q0 = (rh_off - Dp) >> 2;
       for (int q = lane; 4 * q < ldrh - Dp; q += 32) {

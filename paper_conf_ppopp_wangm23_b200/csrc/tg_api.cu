@@ -82,7 +82,7 @@ struct tg_ctx {
   int ld_ch = 0, ld_rh = 0, ld_z = 0;
   int dpa = 0;  // BF16 merge-FFN input row [LN(y) (Dp) | 0 | h at dpa = round8(Dp) (16-byte aligned) | 0]
   TcTensorA ta_c, ta_rh, ta_z;  // TMA tensor maps of the bf16 activations (dense GEMM A operands)
-  TcTensorA ta_c32, ta_z32;     // fp32-level modes: fp32 c and z, feeding the GEMM producers' staging
+  TcTensorA ta_c32, ta_z32, ta_r32;  // fp32-level modes: fp32 c, z and [LN | h], feeding the GEMM staging
   AttnMaps am[2][TG_MAX_LAYERS + 1]{};  // per set and level l: TMA row-gather maps (h rows, E rows, Phi rows)
   int cur_set = 0;
   // Phi rows per set: [table (W rows) | direct rows of level 1 | level 2 | ...] (k_phi_rows, front stream)
@@ -392,14 +392,12 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
                      bfa ? ctx->rh_h : nullptr, ctx->ld_rh, ctx->dpa, st);
     TRY(launched(ctx));
   }
-  // G3: z = ReLU(W1 [r || h^(l-1)] + b1)  (Eq. 7)
+  // G3: z = ReLU(W1 [r || h^(l-1)] + b1)  (Eq. 7); the LayerNorm wrote the dense row [r | h]
   GemmArgs g3{};
   g3.err = ctx->err;
   g3.a_base0 = ctx->r;
-  g3.lda0 = ctx->Dp;
-  g3.K0 = ctx->Dp;
-  g3.a_rows1 = lv.hs_row;
-  g3.K = ctx->Dp + ctx->dnp;
+  g3.lda0 = ctx->Dp + ctx->dnp;
+  g3.K0 = g3.K = ctx->Dp + ctx->dnp;
   g3.B = w.W1;
   g3.N = ctx->dnp;
   g3.bias = w.b1;
@@ -417,7 +415,7 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   }
   {
     Prof pf(ctx, TG_ST_FFN1, st);
-    if (tc) launch_gemm_tc(g3, w.tcW1, ctx->cfg.precision, st, bfa ? &ctx->ta_rh : nullptr);
+    if (tc) launch_gemm_tc(g3, w.tcW1, ctx->cfg.precision, st, bfa ? &ctx->ta_rh : (x3 ? &ctx->ta_r32 : nullptr));
     else launch_gemm_simt(g3, st);
   }
   TRY(launched(ctx));
@@ -1076,7 +1074,7 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
   TRY(dalloc(ctx, &ctx->u, (size_t)maxC * HDp));
   TRY(dalloc(ctx, &ctx->c, (size_t)maxC * HDp));
   TRY(dalloc(ctx, &ctx->y, (size_t)maxC * Dp));
-  TRY(dalloc(ctx, &ctx->r, (size_t)maxC * Dp));
+  TRY(dalloc(ctx, &ctx->r, (size_t)maxC * (Dp + dnp)));  // [LN(y) | h^(l-1)] rows (G3's A)
   TRY(dalloc(ctx, &ctx->z, (size_t)maxC * dnp));
   TRY(dalloc(ctx, &ctx->HL, (size_t)S * cap[L] * dnp));
   if (cfg->precision == TG_PREC_BF16) {
@@ -1094,6 +1092,7 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
   if (cfg->precision == TG_PREC_TF32X3 || cfg->precision == TG_PREC_F16X3) {
     TRY(tc_make_tensor_a(ctx->c, 4, HDp, maxC, &ctx->ta_c32));
     TRY(tc_make_tensor_a(ctx->z, 4, dnp, maxC, &ctx->ta_z32));
+    TRY(tc_make_tensor_a(ctx->r, 4, Dp + dnp, maxC, &ctx->ta_r32));
   }
   // Phi rows of dt >= W computed ahead on the front stream into a per-set buffer that follows a
   // copy of the table, so the attention gathers every Phi row from one tensor (dense row index

@@ -327,7 +327,7 @@ void launch_gemm_simt(const GemmArgs& g, cudaStream_t st);
 
 // LayerNorm over the true (unpadded) columns of each row (R1: eps 1e-5, biased var)
 // of y + q, with the attention residual q = [h^(l-1) || 0 || Phi(0)] (Eq. 4)
-// added on load (y = F c + b_fc comes from G2). r (fp32 [M x Dp]) and/or rh
+// added on load (y = F c + b_fc comes from G2). r (fp32 [M x (Dp + dnp)] = [LN | h]) and/or rh
 // (bf16 [M x ldrh] = [LN(y+q) | h^(l-1) | 0-pad], the A operand of the merge
 // FFN) are written when non-null.
 void launch_layernorm(const float* y, float* r, int Dp, int dn, int dnp, int de, int dep, int dt,
