@@ -268,6 +268,7 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   a.nc_max = mmax;
   a.nb_hidx = lv.nb_hidx;
   a.phi_row0 = ctx->phi_pre ? ctx->phi_row0[l] : -1;
+  a.trows = ctx->phi_pre ? ctx->phi_buf[ctx->cur_set] : ctx->table;
   const bool bfa = ctx->cfg.precision == TG_PREC_BF16;  // bf16 activations between the GEMMs
   const bool x3 = ctx->cfg.precision == TG_PREC_TF32X3 || ctx->cfg.precision == TG_PREC_F16X3;
   // TG_LN_FUSE=1: LayerNorm in G2's epilogue (thread-block clusters, DSMEM statistics);

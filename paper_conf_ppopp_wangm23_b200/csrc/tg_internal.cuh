@@ -256,6 +256,7 @@ struct AttnArgs {
   int ldc_h;
   const int32_t* nb_hidx;  // row indices of nb_row in maps.h (gather path)
   long long phi_row0;      // >= 0: Phi rows of dt >= W precomputed at rows phi_row0 + p*k + m of maps.t
+  const float* trows;      // base of the maps.t rows (table, or table + precomputed rows)
   // if rh_h: the target's own h^(l-1) row (hs_row[p], dnp floats) is also written as bf16 to
   // rh_h[p][rh_off : rh_off+dnp] (rh_off 16-byte aligned, >= Dp) and zeros to the rest of
   // [Dp, ld_rh): the h block of the merge-FFN input [LN(y) | h] (Eq. 7), read by G2 (residual

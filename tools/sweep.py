@@ -3,7 +3,7 @@
 The paper's own variants: Fig. 6's ablation (memoization -> + dedup -> + time-encoding
 precompute) and Table 4's cache-limit sweep {1e4, 1e5, 1e6, 3e6} (P:L450-466,
 plus the 2e6 default of P:L380). Each row is cold-cache chronological passes over a whole
-stream through tg_score_stream (the bench's launch configuration: bf16 GEMM operands,
+stream through tg_score_stream (the bench launch configuration: tf32x3 GEMMs,
 default superbatch), device-timed with CUDA events, L2 flushed before each pass; edges/s is the
 median of --passes passes. Outputs do not depend on the toggles (bit-exact invariance is a
 GPU test), so only speed and the counters move.
@@ -76,7 +76,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--configs", nargs="+", default=["reddit", "lastfm"])
     ap.add_argument("--passes", type=int, default=3)
-    ap.add_argument("--precision", type=int, default=2)  # TG_PREC_BF16
+    ap.add_argument("--precision", type=int, default=1)  # TG_PREC_TF32X3 (the bench headline)
     ap.add_argument("--out", default=None)
     ap.add_argument("--model", default=None, help="L,k override, e.g. 3,8 (NEXT-4: L = 3, k = 8)")
     args = ap.parse_args()
