@@ -435,11 +435,8 @@ __device__ __forceinline__ int sbh_batch(const int* s_pre, int S, int j) {  // l
 }
 __device__ __forceinline__ unsigned long long sbh_mask(const CacheDev& c, int NT) {
   unsigned long long T = 1024;
-  while (T < 2ull * (unsigned long long)NT && T <= c.sb_mask) T <<= 1;
+  while (T < 4ull * (unsigned long long)NT && T <= c.sb_mask) T <<= 1;  // both passes' keys: load <= 1/2
   return (T > c.sb_mask + 1 ? c.sb_mask + 1 : T) - 1;
-}
-__device__ __forceinline__ bool sbh_evfree(const CacheDev& c, int NT) {
-  return __ldcg(c.state + 1) + NT <= __ldcg(c.state + 2);
 }
 
 __global__ void k_probe_pre(LevelDev lv, int S, CacheDev c) { pdl_enter();
@@ -483,6 +480,9 @@ __global__ void k_probe_pre(LevelDev lv, int S, CacheDev c) { pdl_enter();
 
 constexpr int kSeqCL = kSeqCLMax;
 constexpr int kSeqThreads = 1024;
+// k_probe_seq runs after an abandoned grid-wide attempt whose keys still occupy the superbatch
+// table: its own entries carry bit 63 (node ids < 2^31 leave it clear in Hash(n, t))
+constexpr unsigned long long kSeqTag = 1ull << 63;
 constexpr int kSeqSlots = kSeqSlotsPerCTA;
 
 __global__ void __launch_bounds__(kSeqThreads, 1)
@@ -531,7 +531,7 @@ k_probe_seq(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err)
       sbslot[j] = 0xFFFFFFFFu;
       const int i = tbeg + j;
       if (j < ipt && i < cend) {
-        const unsigned long long key = tkey(lv.u_node[seg + i], lv.u_ts[seg + i]);
+        const unsigned long long key = tkey(lv.u_node[seg + i], lv.u_ts[seg + i]) | kSeqTag;
         long long p = -1;
         unsigned long long h = mix64(key) & tmask;
         for (unsigned long long pr = 0; pr <= tmask; ++pr) {
@@ -577,7 +577,7 @@ k_probe_seq(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err)
         lv.c_ts[q] = t;
         lv.sup[q] = 0;
         lv.slot[seg + i] = (head + rr) % c.rcap;  // == (head0 + q) % rcap
-        const unsigned long long key = tkey(node, t);
+        const unsigned long long key = tkey(node, t) | kSeqTag;
         if (sbslot[j] != 0xFFFFFFFFu) {  // evicted and missed again inside this SB
           const unsigned h = sbslot[j];
           unsigned* qp = sq + h;
@@ -642,9 +642,10 @@ k_probe_seq(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int* err)
 __global__ void k_sbh_insert(LevelDev lv, int S, CacheDev c, int* err) { pdl_enter();
   __shared__ int s_pre[kMaxS + 1];
   const int NT = sbh_pre(lv, S, s_pre);
-  const bool ef = sbh_evfree(c, NT);
-  if (blockIdx.x == 0 && threadIdx.x == 0) c.state[5] = ef ? 1 : 0;
-  if (!ef) return;
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    c.state[5] = 1;          // grid-wide pass attempted (k_sbh_finish may hand over to k_probe_seq)
+    c.state[6] = LLONG_MAX;  // min index position of the superbatch's first-occurrence hits
+  }
   const unsigned long long tmask = sbh_mask(c, NT);
   for (int j = blockIdx.x * blockDim.x + threadIdx.x; j < NT; j += gridDim.x * blockDim.x) {
     const int b = sbh_batch(s_pre, S, j);
@@ -749,7 +750,9 @@ __global__ void __launch_bounds__(kSbhThreads) k_sbh_assign(LevelDev lv, int S, 
       sl = (head0 + q) % c.rcap;
       ++q;
     } else {
-      sl = __ldcg(lv.p0 + idx) % c.rcap;
+      const long long p = __ldcg(lv.p0 + idx);
+      atomicMin(reinterpret_cast<long long*>(c.state + 6), p);
+      sl = p % c.rcap;
     }
     lv.slot[idx] = sl;
     c.sb_slot[c.sb_h[idx]] = sl;
@@ -768,12 +771,22 @@ __global__ void k_sbh_finish(LevelDev lv, int S, CacheDev c, long long* cnt, int
     if (!sbh_first(lv, c, idx, j)) lv.slot[idx] = __ldcg(c.sb_slot + c.sb_h[idx]);
   }
   if (blockIdx.x != 0) return;
+  __shared__ int s_ok;
   if (threadIdx.x == 0) {
     int M = 0;
     for (int q = 0; q < nblk; ++q) M += __ldcg(c.sb_blk + q);
     s_M = M;
+    // The closed form is the sequential outcome iff nothing it counts as a hit leaves the FIFO
+    // window before its batch: every first-occurrence hit's position must still be live after
+    // the superbatch's last store, and no in-superbatch miss may be evicted (M <= limit).
+    // Otherwise the ordered pass (k_probe_seq) redoes the superbatch batch by batch.
+    const long long head0 = c.state[0], size0 = c.state[1], limit = c.state[2];
+    const long long live_lo_end = head0 + M - (size0 + M < limit ? size0 + M : limit);
+    s_ok = (M <= limit && __ldcg(c.state + 6) >= live_lo_end) ? 1 : 0;
+    if (!s_ok) c.state[5] = 0;
   }
   __syncthreads();
+  if (!s_ok) return;
   const int M = s_M;
   if (threadIdx.x < S) {
     // misses of batch b = misses with j in [pre[b], pre[b+1]): bounds in the compute list
@@ -798,11 +811,19 @@ __global__ void k_sbh_finish(LevelDev lv, int S, CacheDev c, long long* cnt, int
   }
   __syncthreads();
   if (threadIdx.x == 0) {
-    const long long head0 = c.state[0], size0 = c.state[1];
+    const long long head0 = c.state[0], size0 = c.state[1], limit = c.state[2];
+    long long size = size0;
+    for (int b = 0; b < S; ++b) {  // FIFO sizes and evictions batch by batch (R11, R19)
+      const long long m = lv.n_c[b];
+      const long long nsz = size + m < limit ? size + m : limit;
+      const long long ev_total = size + m - nsz;
+      cnt_add(cnt, b, layer * TG_CNT_PER_LAYER + 5, ev_total < size ? ev_total : size);
+      size = nsz;
+    }
     *lv.n_c_total = M;
     c.state[4] = head0;
     c.state[0] = head0 + M;
-    c.state[1] = size0 + M;
+    c.state[1] = size;
   }
 }
 

@@ -806,7 +806,7 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
       for (int l = 1; l <= L; ++l) {
         b += 2 * s * cap[l] * (72 + 24 * (int64_t)k);
         mx = std::max<int64_t>(mx, s * cap[l]);
-        if (l < L) b += s * cap[l] * 4 * 20 + s * cap[l] * 4;  // grid-wide lookup table (2x pow2) + slots
+        if (l < L) b += s * cap[l] * 8 * 20 + s * cap[l] * 4;  // superbatch lookup table (4x pow2) + slots
       }
       return b + mx * 4 * (2 * HDp_ + 2 * Dp_ + round4(d_n)) + mx * 2 * (HDp_ + Dp_ + 2 * round4(d_n));
     };
@@ -1059,7 +1059,7 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     TRY(dalloc(ctx, &cd.rkey, (size_t)rcap));
     {  // grid-wide eviction-free lookup pass: superbatch-scoped hash, >= 2x its entries
       unsigned long long T = 1024;
-      while (T < 2ull * (unsigned long long)S * cap[l]) T <<= 1;
+      while (T < 4ull * (unsigned long long)S * cap[l]) T <<= 1;  // grid-wide + ordered pass keys
       TRY(dalloc(ctx, &cd.sb_key, T));
       TRY(dalloc(ctx, &cd.sb_val, T));
       TRY(dalloc(ctx, &cd.sb_slot, T));

@@ -126,7 +126,8 @@ struct CacheDev {
   float* ring;               // [rcap x ldn]
   long long rcap;
   long long* state;          // device [8]: head, size, limit, occupied index slots, head at SB start,
-                             // eviction-free flag, -, slots filled by an index rebuild
+                             // grid-wide pass valid (1) / ordered pass (0), min position of the
+                             // superbatch's first-occurrence hits, slots filled by an index rebuild
   unsigned long long* rkey;  // [rcap] key stored at each ring slot (index rebuild)
   // host-mapped report word: ((superbatch + 1) << 40) | occupied slots, written by
   // k_probe_pre, read by the host without synchronising (rebuild trigger bound)
