@@ -49,6 +49,12 @@ struct tg_ctx {
   bool loaded = false;
   tg_model_cfg cfg{};
   int L = 0, H = 0, k = 0, d_n = 0, d_e = 0, d_t = 0, dnp = 0, dep = 0, dtp = 0, Dp = 0, W = 0, S = 1;
+  // Wt: rows of the device Phi table. The paper's window W fixes which dt count as
+  // served by the precomputed table (the t_table / t_direct counters, the ablation); the table
+  // itself extends to Wt = min(max t + 1, 4M) rows (same bits as the direct path, R5), so the
+  // kernels gather Phi(dt) for every dt < Wt instead of recomputing it
+  int Wt = 0;
+  uint32_t max_ts = 0;
   LayerW lw[TG_MAX_LAYERS];
   float *omega = nullptr, *phi = nullptr, *table = nullptr;
   float *Wa1 = nullptr, *ba1 = nullptr, *Wa2 = nullptr;
@@ -255,7 +261,7 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   a.omega = ctx->omega;
   a.phi = ctx->phi;
   a.table = ctx->table;
-  a.W = ctx->W;
+  a.W = ctx->Wt;
   a.use_table = (ctx->cfg.opts & TG_OPT_TTABLE) ? 1 : 0;
   a.dnp = ctx->dnp;
   a.dep = ctx->dep;
@@ -551,7 +557,7 @@ tg_status run_front(tg_ctx* ctx, int S, bool edge_mode, const EdgeSrc& es, int n
     pa.phi = ctx->phi;
     pa.L = L;
     pa.k = k;
-    pa.W = ctx->W;
+    pa.W = ctx->Wt;
     pa.use_table = use_table;
     pa.d_t = ctx->d_t;
     pa.dtp = ctx->dtp;
@@ -754,6 +760,7 @@ tg_status tg_graph_load(int device, const tg_graph_desc* gd, tg_ctx** out) {
   g.d_n = gd->d_n;
   g.d_e = gd->d_e;
   g.ldn = ldn;
+  for (int64_t i = 0; i < E; ++i) ctx->max_ts = std::max(ctx->max_ts, gd->ts[i]);
   g.lde = lde;
   TRYF(dalloc(ctx, &ctx->err, 2));  // [0] sticky error bits, [1] debug index-check mismatches
   cudaMemset(ctx->err, 0, 2 * sizeof(int));
@@ -838,7 +845,15 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     if (!(std::fabs((double)om[c]) * 4294967296.0 + std::fabs((double)ph[c]) < 1e15)) return TG_EINVAL;
   TRY(dalloc(ctx, &ctx->omega, d_t));
   TRY(dalloc(ctx, &ctx->phi, d_t));
-  const int Wrows = std::max(ctx->W, 1);
+  {
+    static const int wt_env = [] {  // TG_PHI_TABLE=0: table of the paper's window only (A/B)
+      const char* e = getenv("TG_PHI_TABLE");
+      return e ? atoi(e) : 1;
+    }();
+    const long long want = (long long)ctx->max_ts + 1;
+    ctx->Wt = (ctx->W > 0 && wt_env) ? (int)std::min<long long>(std::max<long long>(want, ctx->W), 1ll << 22) : ctx->W;
+  }
+  const int Wrows = std::max(ctx->Wt, 1);
   TRY(dalloc(ctx, &ctx->table, (size_t)Wrows * ctx->dtp));
   CK(cudaMemcpy(ctx->omega, om, d_t * 4, cudaMemcpyHostToDevice));
   CK(cudaMemcpy(ctx->phi, ph, d_t * 4, cudaMemcpyHostToDevice));
