@@ -1190,6 +1190,24 @@ __global__ void k_resolve(ResolveArgs a, int* err) { pdl_enter();
   }
 }
 
+__global__ void k_gather_hs(ResolveArgs a, int l0) { pdl_enter();
+  const int l = blockIdx.y + l0;
+  const LevelDev& lv = a.lv[l];
+  if (!lv.hs_dense) return;
+  const int n = *lv.n_c_total;
+  const int lane = threadIdx.x & 31;
+  const int nq = a.ldn >> 2;
+  for (int q = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; q < n; q += (gridDim.x * blockDim.x) >> 5) {
+    const float4* src = reinterpret_cast<const float4*>(lv.hs_row[q]);
+    float4* dst = reinterpret_cast<float4*>(lv.hs_dense + (size_t)q * a.ldn);
+    for (int c = lane; c < nq; c += 32) dst[c] = src[c];
+  }
+}
+
+void launch_gather_hs(const ResolveArgs& a, int l0, int l1, cudaStream_t st) {
+  launch_k(k_gather_hs, dim3(dim3(148 * 2, l1 - l0 + 1)), dim3(256), 0, st, a, l0);
+}
+
 void launch_resolve(const ResolveArgs& a, int* err, cudaStream_t st) {
   long long mx = (long long)a.c_cap_max * (a.k + 1);
   int bx = (int)((mx + 255) / 256);

@@ -89,6 +89,7 @@ struct tg_ctx {
   int dpa = 0;  // BF16 merge-FFN input row [LN(y) (Dp) | 0 | h at dpa = round8(Dp) (16-byte aligned) | 0]
   TcTensorA ta_c, ta_rh, ta_z;  // TMA tensor maps of the bf16 activations (dense GEMM A operands)
   TcTensorA ta_c32, ta_z32, ta_r32;  // fp32-level modes: fp32 c, z and [LN | h], feeding the GEMM staging
+  TcTensorA ta_hs[2][TG_MAX_LAYERS + 1];  // fp32-level modes: dense h^(l-1) rows of each set / level (G1)
   AttnMaps am[2][TG_MAX_LAYERS + 1]{};  // per set and level l: TMA row-gather maps (h rows, E rows, Phi rows)
   int cur_set = 0;
   // Phi rows per set: [table (W rows) | direct rows of level 1 | level 2 | ...] (k_phi_rows, front stream)
@@ -230,9 +231,15 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   const bool tc = ctx->cfg.precision != TG_PREC_FP32;
   const int* m_dev = lv.n_c_total;
   // G1: u = P h^(l-1) + bu  (target-side K projection with W_q and 1/sqrt(d_k) folded)
+  // level 1: the node-feature rows were gathered densely on the front stream (TMA-fed A);
+  // levels >= 2 read layer l-1 embeddings of this superbatch through their row pointers
+  // (densifying them here on the layer stream measured no faster: 9.31 vs 9.35 M edges/s)
+  const bool dense_hs = lv.hs_dense && l == 1;
   GemmArgs g1{};
   g1.err = ctx->err;
-  g1.a_rows0 = lv.hs_row;
+  g1.a_rows0 = dense_hs ? nullptr : lv.hs_row;
+  g1.a_base0 = dense_hs ? lv.hs_dense : nullptr;
+  g1.lda0 = ctx->dnp;
   g1.K0 = g1.K = ctx->dnp;
   g1.B = w.P;
   g1.N = HDp;
@@ -243,7 +250,7 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   g1.m_max = mmax;
   {
     Prof pf(ctx, TG_ST_PROJ_K, st);
-    if (tc) launch_gemm_tc(g1, w.tcP, ctx->cfg.precision, st);
+    if (tc) launch_gemm_tc(g1, w.tcP, ctx->cfg.precision, st, dense_hs ? &ctx->ta_hs[ctx->cur_set][l] : nullptr);
     else launch_gemm_simt(g1, st);
   }
   TRY(launched(ctx));
@@ -546,6 +553,11 @@ tg_status run_front(tg_ctx* ctx, int S, bool edge_mode, const EdgeSrc& es, int n
     launch_resolve(ra, ctx->err, st);
   }
   TRY(launched(ctx));
+  if (ctx->lv[1].hs_dense) {  // fp32-level modes: G1's A rows of level 1 (node features) made dense
+    Prof pf(ctx, TG_ST_RESOLVE, st);
+    launch_gather_hs(ra, 1, 1, st);
+    TRY(launched(ctx));
+  }
   if (ctx->phi_pre && ctx->am[ctx->cur_set][1].valid) {  // TimeEncode of the dt >= W rows (Eq. 8)
     PhiRowsArgs pa{};
     for (int l = 0; l <= L; ++l) {
@@ -1039,6 +1051,8 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     TRY(dalloc(ctx, &v.nb_ts, n * k));
     TRY(dalloc(ctx, &v.nb_eid, n * k));
     TRY(dalloc(ctx, &v.hs_row, n));
+    if ((cfg->precision == TG_PREC_TF32X3 || cfg->precision == TG_PREC_F16X3) && l == 1)
+      TRY(dalloc(ctx, &v.hs_dense, n * round4(d_n)));
     TRY(dalloc(ctx, &v.nb_row, n * k));
     TRY(dalloc(ctx, &v.nb_hidx, n * k));
     TRY(dalloc(ctx, &v.dst_row, n));
@@ -1109,6 +1123,8 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     TRY(tc_make_tensor_a(ctx->c, 4, HDp, maxC, &ctx->ta_c32));
     TRY(tc_make_tensor_a(ctx->z, 4, dnp, maxC, &ctx->ta_z32));
     TRY(tc_make_tensor_a(ctx->r, 4, Dp + dnp, maxC, &ctx->ta_r32));
+    for (int set = 0; set < 2; ++set)
+      TRY(tc_make_tensor_a(ctx->lvs[set][1].hs_dense, 4, dnp, ctx->lvs[set][1].c_cap, &ctx->ta_hs[set][1]));
   }
   // Phi rows of dt >= W computed ahead on the front stream into a per-set buffer that follows a
   // copy of the table, so the attention gathers every Phi row from one tensor (dense row index

@@ -182,6 +182,7 @@ struct LevelDev {
   int32_t* nb_eid;
   // row addresses resolved for the layer-l compute
   const float** hs_row;      // [c_cap]     h^(l-1) of the target
+  float* hs_dense;           // [c_cap x ldn] the same rows gathered densely (G1's A; may be null)
   const float** nb_row;      // [c_cap * k] h^(l-1) of each neighbour
   int32_t* nb_hidx;          // [c_cap * k] its row in the level's h tensor (X at l = 1, else ring l-1)
   float** dst_row;           // [c_cap]     where h^(l) goes (ring slot or H_L)
@@ -229,6 +230,11 @@ struct ResolveArgs {
   int c_cap_max;
 };
 void launch_resolve(const ResolveArgs& a, int* err, cudaStream_t st);
+// hs_dense[q] = *hs_row[q] for every computed target of levels l0..l1 (warp per row), so the
+// key projection G1 reads a dense A operand (TMA tiles) instead of gathering rows. Level 1
+// reads node features (front stream); level l >= 2 reads layer l-1 embeddings of the same
+// superbatch, so it runs on the layer stream after layer l-1
+void launch_gather_hs(const ResolveArgs& a, int l0, int l1, cudaStream_t st);
 
 // Phi table [W x dtp] built on device with the same function as the direct path.
 void launch_time_table(const float* omega, const float* phi, int d_t, int dtp, int W, float* table,
