@@ -511,8 +511,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="reddit")
     ap.add_argument("--precision", default="tf32x3", choices=["tf32x3", "f16x3", "bf16", "fp32", "tf32"])
-    ap.add_argument("--second-precision", default="bf16",
-                    help="also measure this precision into the same line ('none' to skip)")
+    ap.add_argument("--second-precision", default="bf16,f16x3",
+                    help="also measure these precisions (comma list) into the same line ('none' to skip)")
     ap.add_argument("--scaling", default="strong", choices=["strong", "weak"])
     ap.add_argument("--superbatch", type=int, default=0)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
@@ -558,8 +558,8 @@ def main():
     else:
         shard = (0, (s.n_edges + B - 1) // B, 0, s.n_edges)
 
-    precs = [args.precision] + ([args.second_precision] if args.second_precision not in ("none", args.precision)
-                                else [])
+    precs = [args.precision] + [p for p in args.second_precision.split(",")
+                                if p and p not in ("none", args.precision)]
     res = {}
     for p in precs:
         res[p] = measure(args, p, s, flat, mc, {}, shard, world, rank, local, dist, args.steps, args.warmup,

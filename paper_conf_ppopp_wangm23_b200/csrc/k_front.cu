@@ -733,6 +733,7 @@ __global__ void __launch_bounds__(kSbhThreads) k_sbh_assign(LevelDev lv, int S, 
   int tot;
   const int excl = block_excl_scan(m, s_warp, tot);  // (syncs: s_off visible)
   int q = s_off + excl;
+  long long pmin = LLONG_MAX;  // min index position of this thread's first-occurrence hits
 #pragma unroll
   for (int e = 0; e < kSbhItems; ++e) {
     if (!(first & (1u << e))) continue;
@@ -751,12 +752,19 @@ __global__ void __launch_bounds__(kSbhThreads) k_sbh_assign(LevelDev lv, int S, 
       ++q;
     } else {
       const long long p = __ldcg(lv.p0 + idx);
-      atomicMin(reinterpret_cast<long long*>(c.state + 6), p);
+      pmin = p < pmin ? p : pmin;
       sl = p % c.rcap;
     }
     lv.slot[idx] = sl;
     c.sb_slot[c.sb_h[idx]] = sl;
   }
+  // one atomic per warp (a single hot address otherwise serialises the whole grid)
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const long long other = __shfl_xor_sync(0xffffffffu, pmin, o);
+    pmin = other < pmin ? other : pmin;
+  }
+  if ((threadIdx.x & 31) == 0 && pmin != LLONG_MAX) atomicMin(reinterpret_cast<long long*>(c.state + 6), pmin);
 }
 
 __global__ void k_sbh_finish(LevelDev lv, int S, CacheDev c, long long* cnt, int layer, int nblk) { pdl_enter();
