@@ -44,7 +44,9 @@ constexpr int TC_PROD_WARPS = 8;
 constexpr int TC_EPI_WARPS = 4;
 constexpr int TC_EPI_HALVES = TC_EPI_WARPS / 4;  // epilogue warps per lane quadrant (column split)
 constexpr int TC_TMA_WARP = TC_PROD_WARPS, TC_MMA_WARP = TC_PROD_WARPS + 1, TC_EPI_WARP0 = TC_PROD_WARPS + 2;
-constexpr int TC_WARPS = TC_PROD_WARPS + 2 + TC_EPI_WARPS;
+// + one staging warp: refills the fp32-level producers' staging ring by TMA (stage_tma)
+constexpr int TC_STG_WARP = TC_EPI_WARP0 + TC_EPI_WARPS;
+constexpr int TC_WARPS = TC_PROD_WARPS + 2 + TC_EPI_WARPS + 1;
 constexpr int TC_THREADS = TC_WARPS * 32;
 constexpr int TC_MAXSTAGES = 8;
 // TMEM: two accumulator buffers of 256 columns (all 512 columns; one CTA per
@@ -89,7 +91,9 @@ __host__ __device__ inline int tc_kb_bytes(int prec) {
 // buffer per epilogue warp
 constexpr int TC_BAR_BYTES = 256;
 constexpr int TC_STG_LD = 20;  // floats per staged row (16 columns + pad)
-constexpr int TC_EPI_BYTES = TC_EPI_WARPS * 32 * TC_STG_LD * 4;
+// + per-tile bias / column-scale staging, double-buffered by tile parity: [2][bias 256 | scale 256]
+constexpr int TC_EPI_XPOSE_BYTES = TC_EPI_WARPS * 32 * TC_STG_LD * 4;
+constexpr int TC_EPI_BYTES = TC_EPI_XPOSE_BYTES + 2 * 2 * 256 * 4;
 
 // fused-LayerNorm epilogue (g.ln): per-row partial statistics of the two
 // column halves [2][128] and the cluster exchange buffers [2 parities][4 N tiles][128]
@@ -100,7 +104,7 @@ constexpr int TC_LN_BYTES = (2 * 128 + 2 * TC_LN_MAXTN * 128) * 16 + 4 * 256 * 4
 // `stg` staging units of 16 KB (its cp.async look-ahead ring, up to 4 units) -- as many
 // staging units as fit beside 2 stages, then as many stages as fit beside those.
 constexpr int TC_STG_UNIT = TC_BM * 128;
-constexpr int TC_PTR_BYTES = 2 * TC_BM * 8 + 64;  // the producers' row-pointer table + staging mbarriers
+constexpr int TC_PTR_BYTES = 2 * TC_BM * 8 + 64;  // the producers' row-pointer table + staging mbarriers [2][4]
 static inline bool tc_atmem(int prec) { return tc_planes(prec) == 2; }  // A operand in TMEM
 static inline void tc_plan(int prec, int BN, int ln, bool generic, int* stages, int* stg) {
   const size_t st = (size_t)tc_planes(prec) * ((tc_atmem(prec) ? 0 : (size_t)TC_BM * 128) + (size_t)BN * tc_kb_bytes(prec));
@@ -467,6 +471,17 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t* v) {
       : "r"(taddr));
 }
 
+// staging ring of the generic A producers: after stages, barriers, epilogue buffers [, LN], at a
+// 1024-byte boundary (TMA's 128-byte swizzle is a function of the address); then the row-pointer
+// table [2][128] and the staging mbarriers [landed 4 | read 4]
+__device__ __forceinline__ unsigned char* tc_stage_ring(unsigned char* smem, uint32_t stage_total, int ln) {
+  return smem + ((stage_total + TC_BAR_BYTES + TC_EPI_BYTES + (ln ? TC_LN_BYTES : 0) + 1023u) & ~1023u);
+}
+__device__ __forceinline__ uint64_t* tc_stage_bars(unsigned char* smem, uint32_t stage_total, int ln, int stg) {
+  return reinterpret_cast<uint64_t*>(tc_stage_ring(smem, stage_total, ln) + (size_t)(stg > 0 ? stg : 0) * TC_STG_UNIT +
+                                     2 * TC_BM * sizeof(float*));
+}
+
 template <int PREC>
 __global__ void __launch_bounds__(TC_THREADS, 1)
     k_gemm_tc(GemmArgs g, TcWeights w, int stages, int stg, const __grid_constant__ CUtensorMap tmA, int a_tma,
@@ -533,6 +548,13 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       // (ATMEM tf32x3: each 64-byte k-block is produced by one half of the producers)
       mbar_init(&full[s], (a_tma && !stage_tma) ? 1 : ((generic && !(ATMEM && PREC == TG_PREC_TF32X3)) ? TC_PROD_WARPS * 32 : TC_BM) + 1);
       mbar_init(&empty[s], 1);         // MMA commit
+    }
+    if (stage_tma) {  // staging ring (ATMEM, dense A by TMA): landed (tx) / read by the 8 producer warps
+      uint64_t* sb = tc_stage_bars(smem, stages * stage_bytes, g.ln, stg);
+      for (int i = 0; i < stg; ++i) {
+        mbar_init(&sb[i], 1);
+        mbar_init(&sb[4 + i], TC_PROD_WARPS);
+      }
     }
     for (int a = 0; a < 2; ++a) {
       mbar_init(&tfull[a], 1);     // MMA commit after the tile's last k-block
@@ -638,10 +660,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     constexpr int NPT = TC_PROD_WARPS * 32;
     const int prow = tid & (TC_BM - 1), ph = tid >> 7;  // row, column half
     // staging ring at a 1024-byte boundary: TMA's 128-byte swizzle is a function of the address
-    unsigned char* sring =
-        smem + ((stages * stage_bytes + TC_BAR_BYTES + TC_EPI_BYTES + (g.ln ? TC_LN_BYTES : 0) + 1023u) & ~1023u);
+    unsigned char* sring = tc_stage_ring(smem, stages * stage_bytes, g.ln);
     const float** sptr = reinterpret_cast<const float**>(sring + (size_t)(stg > 0 ? stg : 0) * TC_STG_UNIT);  // [2][128]
-    uint64_t* sbar = reinterpret_cast<uint64_t*>(sptr + 2 * TC_BM);  // [4] staging slots (stage_tma)
+    uint64_t* sbar = reinterpret_cast<uint64_t*>(sptr + 2 * TC_BM);  // [4] staging slots landed (stage_tma)
+    uint64_t* sempty = sbar + 4;  // [4] staging slots read by every producer warp (stage_tma)
     // stg < 0: no staging ring -- each thread prefetches its own row half two units ahead
     // in registers (no shared-memory round trip, no producer barriers)
     const bool regpf = stg < 0;
@@ -757,12 +779,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       asm volatile("cp.async.commit_group;\n" ::: "memory");  // (empty past the last tile)
     };
     if (stage_tma) {
-      if (tid == 0) {
-        for (int i = 0; i < D; ++i) mbar_init(&sbar[i], 1);
-        asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
-      }
-      pbar();
-      for (int i = 0; i < D; ++i) issue(i);
+      // the staging warp (TC_STG_WARP) fills the ring; its barriers were initialised with the others
     } else if (D > 0) {  // (regpf: D = 0)
       if (it_t < ntiles) publish(it_t);
       for (int i = 0; i < D; ++i) issue(i);
@@ -793,21 +810,29 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           } else {
             if (stage_tma) {
               mbar_wait(&sbar[slot], (gu / (uint32_t)D) & 1);  // the unit's TMA tile has landed
+              TR5(1);
+              const unsigned char* src = sring + (size_t)slot * TC_STG_UNIT + prow * 128;
+#pragma unroll
+              for (int i = 0; i < 4; ++i)
+                x[i] = *reinterpret_cast<const float4*>(src + (((4 * ph + i) ^ (prow & 7)) << 4));
+              __syncwarp();
+              if (lane == 0) mbar_arrive(&sempty[slot]);  // this warp is done with the slot
+              TR5(2);
             } else {
               if (D == 1) asm volatile("cp.async.wait_group 0;\n" ::: "memory");
               else if (D == 2) asm volatile("cp.async.wait_group 1;\n" ::: "memory");
               else if (D == 3) asm volatile("cp.async.wait_group 2;\n" ::: "memory");
               else asm volatile("cp.async.wait_group 3;\n" ::: "memory");
               pbar();  // every producer's copies of this unit have landed
-            }
-            TR5(1);
-            const unsigned char* src = sring + (size_t)slot * TC_STG_UNIT + prow * 128;
+              TR5(1);
+              const unsigned char* src = sring + (size_t)slot * TC_STG_UNIT + prow * 128;
 #pragma unroll
-            for (int i = 0; i < 4; ++i)
-              x[i] = *reinterpret_cast<const float4*>(src + (((4 * ph + i) ^ (prow & 7)) << 4));
-            pbar();  // every producer has read the slot: it may be refilled
-            TR5(2);
-            issue(slot);  // unit gu + D
+              for (int i = 0; i < 4; ++i)
+                x[i] = *reinterpret_cast<const float4*>(src + (((4 * ph + i) ^ (prow & 7)) << 4));
+              pbar();  // every producer has read the slot: it may be refilled
+              TR5(2);
+              issue(slot);  // unit gu + D
+            }
           }
           const int kbq = EPK == 16 ? 2 * u + ph : u;
           if (kbq >= nkb) continue;
@@ -1043,6 +1068,35 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         if (tc == 0) TCT(3, clock64());
       }
     }
+  } else if (warp == TC_STG_WARP) {
+    // ===================== staging warp (stage_tma): TMA 2D tiles (32 fp32 x 128 rows) of the
+    // dense fp32 A into the producers' ring, `stg` units ahead; a slot is refilled once all 8
+    // producer warps have read it (sempty), so no producer waits on the refill
+    if (stage_tma && lane == 0) {
+      unsigned char* sring = tc_stage_ring(smem, stages * stage_bytes, g.ln);
+      uint64_t* sbar = tc_stage_bars(smem, stages * stage_bytes, g.ln, stg);
+      uint64_t* sempty = sbar + 4;
+      constexpr int EPK = PREC == TG_PREC_F16X3 ? 32 : 16;
+      const int upt = (nkb * EPK + 31) / 32;
+      uint32_t q = 0;
+      for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        const int y = (t / w.ntn) * TC_BM;
+        for (int u = 0; u < upt; ++u, ++q) {
+          const uint32_t slot = q % (uint32_t)stg;
+          if (q >= (uint32_t)stg) mbar_wait(&sempty[slot], ((q / (uint32_t)stg) - 1u) & 1u);
+          // the producers' generic reads of the slot before the async-proxy write that refills it
+          asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
+          const uint32_t bar = smem_u32(&sbar[slot]);
+          asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(bar), "r"(TC_STG_UNIT)
+                       : "memory");
+          asm volatile(
+              "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], "
+              "[%4];\n" ::"r"(smem_u32(sring + (size_t)slot * TC_STG_UNIT)),
+              "l"(reinterpret_cast<uint64_t>(&tmA)), "r"(u * 32), "r"(y), "r"(bar)
+              : "memory");
+        }
+      }
+    }
   } else if (g.ln) {
     // ===================== epilogue with the fused LayerNorm (G2, Eq. 6: r = LN(W_fc o +
     // b_fc + q), R1; the residual q = [h | 0 | Phi(0)] is already in the accumulator: h
@@ -1188,11 +1242,22 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     const int half = ew >> 2;              // which alternate chunk (with 8 epilogue warps)
     float* stg = reinterpret_cast<float*>(smem + stages * stage_bytes + TC_BAR_BYTES) + ew * (32 * TC_STG_LD);
     const int rq = lane >> 2, cq = lane & 3;  // read-back: row rq + 8i, float4 column cq
+    // the tile's bias (and F16X3 column scales) staged in shared memory before its accumulator
+    // is ready -- no global-load latency inside the chunk loop
+    float* s_eb = reinterpret_cast<float*>(smem + stages * stage_bytes + TC_BAR_BYTES + TC_EPI_XPOSE_BYTES);
+    const int etid = tid - TC_EPI_WARP0 * 32;
     uint32_t tc = 0;
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++tc) {
       const int tm = t / w.ntn, tn = t - tm * w.ntn;
       const int m0 = tm * TC_BM, n0 = tn * BN;
       const uint32_t acc = tc % nbuf;
+      float* sb = s_eb + (tc & 1) * 512;  // [bias 256 | scale 256]; buffer tc & 1 was last read by tile tc - 2
+      for (int i = etid; i < BN; i += TC_EPI_WARPS * 32) {
+        const int c = n0 + i;
+        sb[i] = (g.bias && c < g.N) ? g.bias[c] : 0.f;
+        if (PREC == TG_PREC_F16X3) sb[256 + i] = w.colscale[c];
+      }
+      asm volatile("bar.sync 1, %0;\n" ::"n"(TC_EPI_WARPS * 32) : "memory");
       const int er = m0 + quad * 32 + lane;
       float* orow = nullptr;
       unsigned short* hrow = nullptr;
@@ -1234,9 +1299,9 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         const bool cin = cl < BN && c < g.N;                    // N % 4 == 0: all 4 or none
         const bool cpad = cl < BN && c >= g.N && c < g.ldc_h;  // bf16 zero padding [N, ldc_h)
         float4 b4 = make_float4(0.f, 0.f, 0.f, 0.f);
-        if (cin && g.bias) b4 = *reinterpret_cast<const float4*>(g.bias + c);
+        if (cl < BN) b4 = *reinterpret_cast<const float4*>(sb + cl);  // 0 past N
         float4 s4 = make_float4(1.f, 1.f, 1.f, 1.f);  // F16X3: undo the weight-row scale (exact)
-        if (PREC == TG_PREC_F16X3 && cl < BN) s4 = *reinterpret_cast<const float4*>(w.colscale + n0 + cl);
+        if (PREC == TG_PREC_F16X3 && cl < BN) s4 = *reinterpret_cast<const float4*>(sb + 256 + cl);
 #pragma unroll
         for (int i = 0; i < 4; ++i) {
           const int r = rq + 8 * i;
