@@ -246,22 +246,27 @@ def front_bytes(per, L, k, d_n):
     return b
 
 
-def ideal_time(per_batch, s, mc, peaks, prec):
+def ideal_time(per_batch, s, mc, peaks, prec, g1_l0=1):
     """End-to-end ideal time = sum_b max(F_b / P_tensor, B_b / BW_HBM), from the
-    measured per-batch counters, in both formulations (paper form and absorbed form)."""
+    measured per-batch counters, in both formulations (paper form and absorbed form). g1_l0: the
+    first level whose targets run G1 (2 when the layer-1 query side comes from the per-node
+    table U1, R27)."""
     L, k = mc.n_layers, mc.n_neighbors
     bw = peaks["hbm_gbs"] * 1e9
     pt = tensor_peak(peaks, prec) * 1e12
-    fs, fa, gb = flops_spec(s, mc), flops_absorbed(s, mc)["total"], gather_bytes(s, mc)
+    fab = flops_absorbed(s, mc)
+    fs, fa, gb = flops_spec(s, mc), fab["total"], gather_bytes(s, mc)
     t_spec = t_abs = 0.0
     F_spec = F_abs = B = 0
     for p in per_batch:
         m = sum(p[f"l{l}_misses"] for l in range(1, L + 1))
+        mg1 = sum(p[f"l{l}_misses"] for l in range(g1_l0, L + 1))
+        fab_b = m * (fa - fab["G1"]) + mg1 * fab["G1"]
         bb = m * gb + front_bytes(p, L, k, s.d_n)
         t_spec += max(m * fs / pt, bb / bw)
-        t_abs += max(m * fa / pt, bb / bw)
+        t_abs += max(fab_b / pt, bb / bw)
         F_spec += m * fs
-        F_abs += m * fa
+        F_abs += fab_b
         B += bb
     return {"ideal_ms_paper_form": 1e3 * t_spec, "ideal_ms_absorbed_form": 1e3 * t_abs,
             "flops_paper_form": F_spec, "flops_absorbed_form": F_abs, "bytes": B,
@@ -438,12 +443,18 @@ def measure(args, prec_name, s, flat, mc, ctx_kw, shard, world, rank, local, dis
                                "achieved_absorbed_io": n_targets * absorbed_io / (attn_ms / 1e3) / 1e9,
                                "absorbed_io_bytes_per_target": absorbed_io,
                                "share_of_step": attn_ms / ms_step}
+        # layer-1 query side from the per-node table U1 (R27): G1 runs only for levels >= 2, i.e.
+        # (L - 1) of the L launches per superbatch the attention makes
+        g1_l0 = 2 if stages["proj_k"][1] * L == attn_n * (L - 1) else 1
         for st_name, g in (("proj_k", "G1"), ("proj_v", "G2"), ("ffn1", "G3"), ("ffn2", "G4")):
             t_ms, n_l = stages[st_name]
+            if n_l == 0:
+                continue
+            tg = sum(c[f"l{l}_misses"] for l in range(g1_l0, L + 1)) if g == "G1" else n_targets
             kernels[f"k_gemm_tc {g}" if prec_name != "fp32" else f"k_gemm_simt {g}"] = {
-                "bound": "tensor", "unit": "TFLOP/s", "peak": tpk, "flops_per_target": fa[g], "targets": n_targets,
+                "bound": "tensor", "unit": "TFLOP/s", "peak": tpk, "flops_per_target": fa[g], "targets": tg,
                 "launches": n_l, "avg_launch_us": 1e3 * t_ms / max(1, n_l),
-                "achieved": n_targets * fa[g] / (t_ms / 1e3) / 1e12, "share_of_step": t_ms / ms_step}
+                "achieved": tg * fa[g] / (t_ms / 1e3) / 1e12, "share_of_step": t_ms / ms_step}
         for v in kernels.values():
             v["frac"] = v["achieved"] / v["peak"]
         dom = max(kernels, key=lambda n: kernels[n]["share_of_step"])
@@ -462,7 +473,7 @@ def measure(args, prec_name, s, flat, mc, ctx_kw, shard, world, rank, local, dis
                                                    f"{' / 3 passes' if prec_name == 'tf32x3' else ''}")),
                 "launches": dk["launches"], "avg_launch_us": dk["avg_launch_us"],
                 "share_of_step": dk["share_of_step"]}
-        ideal = ideal_time(per, s, mc, peaks, prec_name)
+        ideal = ideal_time(per, s, mc, peaks, prec_name, g1_l0)
         ideal["measured_ms"] = ms_step
         ideal["frac_paper_form"] = ideal["ideal_ms_paper_form"] / ms_step
         ideal["frac_absorbed_form"] = ideal["ideal_ms_absorbed_form"] / ms_step

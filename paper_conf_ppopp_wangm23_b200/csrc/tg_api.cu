@@ -83,6 +83,12 @@ struct tg_ctx {
   // compute workspace
   int maxC = 0;
   float *u = nullptr, *c = nullptr, *y = nullptr, *r = nullptr, *z = nullptr, *HL = nullptr;
+  // U1 [(V+1) x H*Dp]: the layer-1 query side u = P x_i + b_u of every node (R27). Layer-1
+  // targets' h^(0) is the node's static feature row, so u is a function of the node
+  // alone: computed once at tg_model_load by the same GEMM (row-invariant: the bits G1 would
+  // produce per target); null when it would exceed the budget (G1 per target then)
+  float* u1 = nullptr;
+  int* u1_m = nullptr;
   // bf16 activations (TG_PREC_BF16): c, [LN(y) | h], z with row strides padded to 8
   unsigned short *c_h = nullptr, *rh_h = nullptr, *z_h = nullptr;
   int ld_ch = 0, ld_rh = 0, ld_z = 0;
@@ -234,6 +240,7 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   // level 1: the node-feature rows were gathered densely on the front stream (TMA-fed A);
   // levels >= 2 read layer l-1 embeddings of this superbatch through their row pointers
   // (densifying them here on the layer stream measured no faster: 9.31 vs 9.35 M edges/s)
+  const bool u1 = l == 1 && ctx->u1;  // layer 1: u rows from the per-node table (no G1)
   const bool dense_hs = lv.hs_dense && l == 1;
   GemmArgs g1{};
   g1.err = ctx->err;
@@ -248,15 +255,18 @@ tg_status run_layer(tg_ctx* ctx, int l, cudaStream_t st) {
   g1.ldc = HDp;
   g1.m_dev = m_dev;
   g1.m_max = mmax;
-  {
-    Prof pf(ctx, TG_ST_PROJ_K, st);
-    if (tc) launch_gemm_tc(g1, w.tcP, ctx->cfg.precision, st, dense_hs ? &ctx->ta_hs[ctx->cur_set][l] : nullptr);
-    else launch_gemm_simt(g1, st);
+  if (!u1) {
+    {
+      Prof pf(ctx, TG_ST_PROJ_K, st);
+      if (tc) launch_gemm_tc(g1, w.tcP, ctx->cfg.precision, st, dense_hs ? &ctx->ta_hs[ctx->cur_set][l] : nullptr);
+      else launch_gemm_simt(g1, st);
+    }
+    TRY(launched(ctx));
   }
-  TRY(launched(ctx));
   // attention over the k sampled neighbours
   AttnArgs a{};
-  a.u = ctx->u;
+  a.u = u1 ? ctx->u1 : ctx->u;
+  a.u_row = u1 ? lv.c_node : nullptr;
   a.c = ctx->c;
   a.nb_row = lv.nb_row;
   a.nb_node = lv.nb_node;
@@ -553,7 +563,7 @@ tg_status run_front(tg_ctx* ctx, int S, bool edge_mode, const EdgeSrc& es, int n
     launch_resolve(ra, ctx->err, st);
   }
   TRY(launched(ctx));
-  if (ctx->lv[1].hs_dense) {  // fp32-level modes: G1's A rows of level 1 (node features) made dense
+  if (ctx->lv[1].hs_dense && !ctx->u1) {  // fp32-level modes: G1's A rows of level 1 (node features) made dense
     Prof pf(ctx, TG_ST_RESOLVE, st);
     launch_gather_hs(ra, 1, 1, st);
     TRY(launched(ctx));
@@ -1163,6 +1173,41 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
             attn_make_rows_map(tb, ctx->dtp, ctx->dtp, trows, &m.t) == TG_OK)
           m.valid = 1;
       }
+  }
+  // ---- U1: layer-1 query side of every node, u = P x_i + b_u (R27), by the layer-1 G1 kernel
+  {
+    static const bool u1_env = [] {  // TG_U1=0: G1 per layer-1 target instead (A/B)
+      const char* e = getenv("TG_U1");
+      return !(e && e[0] == '0');
+    }();
+    const long long nv = (long long)ctx->g.V + 1;
+    if (u1_env && nv * HDp * 4 <= (8ll << 30) && nv < (1ll << 31)) {
+      TRY(dalloc(ctx, &ctx->u1, (size_t)nv * HDp));
+      TRY(dalloc(ctx, &ctx->u1_m, 1));
+      launch_set_int(ctx->u1_m, (int)nv, 0);
+      const LayerW& w = ctx->lw[0];
+      GemmArgs g{};
+      g.err = ctx->err;
+      g.a_base0 = ctx->X;
+      g.lda0 = ctx->g.ldn;
+      g.K0 = g.K = dnp;
+      g.B = w.P;
+      g.N = HDp;
+      g.bias = w.bu;
+      g.C = ctx->u1;
+      g.ldc = HDp;
+      g.m_dev = ctx->u1_m;
+      g.m_max = (int)nv;
+      if (cfg->precision == TG_PREC_FP32) {
+        launch_gemm_simt(g, 0);
+      } else {
+        TcTensorA ta;  // fp32-level modes: dense rows staged by TMA, as for the per-target G1
+        if (cfg->precision == TG_PREC_TF32X3 || cfg->precision == TG_PREC_F16X3)
+          TRY(tc_make_tensor_a(ctx->X, 4, ctx->g.ldn, (int)nv, &ta));
+        launch_gemm_tc(g, w.tcP, cfg->precision, 0, ta.valid ? &ta : nullptr);
+      }
+      CK(cudaGetLastError());
+    }
   }
   TRY(dalloc(ctx, &ctx->cnt_total, TG_NCOUNTERS));
   for (int set = 0; set < 2; ++set) {

@@ -243,7 +243,8 @@ void launch_time_encode(const float* omega, const float* phi, const float* table
                         int use_table, const int64_t* delta, int64_t n, float* out, cudaStream_t st);
 
 struct AttnArgs {
-  const float* u;          // [nc x H*Dp]
+  const float* u;          // [nc x H*Dp], or [V+1 x H*Dp] rows selected by u_row
+  const int32_t* u_row;    // if non-null: target p reads u row u_row[p] (level 1: node id, per-node table)
   float* c;                // [nc x H*Dp]
   const float* const* nb_row;
   const int32_t* nb_node;  // mask: node == 0 (R7)
