@@ -108,6 +108,8 @@ struct tg_ctx {
   long long* cnt_sbs[2] = {nullptr, nullptr};
   // front stream + events of the two-set pipeline (stream_edges)
   cudaStream_t fst = nullptr;
+  cudaStream_t lst = nullptr;      // layer stream at the highest priority (TG_LAYER_PRIO=1)
+  cudaEvent_t ev_lend = nullptr;
   cudaEvent_t ev_front[2] = {nullptr, nullptr}, ev_back[2] = {nullptr, nullptr}, ev_in = nullptr, ev_fend = nullptr;
   int* err = nullptr;
   int64_t launches = 0;
@@ -612,8 +614,13 @@ tg_status finish(tg_ctx* ctx, int S, long long* log, int64_t row0, cudaStream_t 
 }
 
 tg_status stream_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, const uint32_t* ts, const int32_t* neg,
-                       int64_t n_edges, int batch, float* scores, long long* log, cudaStream_t st) {
+                       int64_t n_edges, int batch, float* scores, long long* log, cudaStream_t st_in) {
   const int64_t nb = (n_edges + batch - 1) / batch;
+  static const bool prio = [] {  // experiment: layers on a high-priority stream, front on the lowest
+    const char* e = getenv("TG_LAYER_PRIO");
+    return e && e[0] == '1';
+  }();
+  cudaStream_t st = st_in;
   // Two-set pipeline: superbatch i's front half runs on ctx->fst into level set
   // i % 2 as soon as superbatch i-2's layers released that set, overlapping the
   // layers of superbatch i-1 on st. The cache index is only touched by front
@@ -621,6 +628,10 @@ tg_status stream_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, cons
   // every kernel sees the same data as in the serial order.
   CK(cudaEventRecord(ctx->ev_in, st));
   CK(cudaStreamWaitEvent(ctx->fst, ctx->ev_in, 0));
+  if (prio) {
+    st = ctx->lst;
+    CK(cudaStreamWaitEvent(st, ctx->ev_in, 0));
+  }
   int64_t sb = 0;
   for (int64_t b0 = 0, S = 0; b0 < nb; b0 += S, ++sb) {
     S = std::min<int64_t>(ctx->S, nb - b0);
@@ -664,7 +675,11 @@ tg_status stream_edges(tg_ctx* ctx, const int32_t* src, const int32_t* dst, cons
 
   }
   CK(cudaEventRecord(ctx->ev_fend, ctx->fst));  // join the front stream into st
-  CK(cudaStreamWaitEvent(st, ctx->ev_fend, 0));
+  CK(cudaStreamWaitEvent(st_in, ctx->ev_fend, 0));
+  if (prio) {
+    CK(cudaEventRecord(ctx->ev_lend, st));
+    CK(cudaStreamWaitEvent(st_in, ctx->ev_lend, 0));
+  }
   select_set(ctx, 0);
   return TG_OK;
 }
@@ -996,6 +1011,25 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
       w.fa_kb0 = kb0;
     }
   }
+  // ---- superbatch size fitted to whole waves of the value/output projection G2 (the largest GEMM):
+  // with the default S, pick S' in [S/2, S] maximising S' / waves(S'), waves = its N x M tiles of
+  // the top layer's worst-case row count (S' x max_batch_targets) over the 148 SMs, e.g. Reddit:
+  // S = 64 -> 600 tiles = 5 waves (the last holding 8 tiles), S = 63 -> 591 tiles = 4 waves
+  if (cfg->superbatch == 0 && !getenv("TG_SB_DEFAULT") && cfg->precision != TG_PREC_FP32 && ctx->lw[L - 1].tcF.ntn > 0) {
+    const int64_t ntn = ctx->lw[L - 1].tcF.ntn, T = cfg->max_batch_targets;
+    int best = S;
+    double best_r = 0.0;
+    for (int s2 = S; s2 >= std::max(1, S / 2); --s2) {
+      const int64_t tiles = ((int64_t)s2 * T + 127) / 128 * ntn;
+      const double r = (double)s2 / (double)((tiles + 147) / 148);
+      if (r > best_r * 1.0001) {
+        best_r = r;
+        best = s2;
+      }
+    }
+    S = best;
+    ctx->S = S;
+  }
   // ---- affinity score MLP (R10), padded
   {
     const float* Wa1 = ph + d_t;
@@ -1216,7 +1250,11 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
   }
   select_set(ctx, 0);
   if (!ctx->fst) {
-    CK(cudaStreamCreateWithFlags(&ctx->fst, cudaStreamNonBlocking));
+    int plo = 0, phi = 0;
+    CK(cudaDeviceGetStreamPriorityRange(&plo, &phi));
+    CK(cudaStreamCreateWithPriority(&ctx->fst, cudaStreamNonBlocking, plo));
+    CK(cudaStreamCreateWithPriority(&ctx->lst, cudaStreamNonBlocking, phi));
+    CK(cudaEventCreateWithFlags(&ctx->ev_lend, cudaEventDisableTiming));
     for (int i = 0; i < 2; ++i) {
       CK(cudaEventCreateWithFlags(&ctx->ev_front[i], cudaEventDisableTiming));
       CK(cudaEventCreateWithFlags(&ctx->ev_back[i], cudaEventDisableTiming));
@@ -1651,9 +1689,11 @@ void tg_free(tg_ctx* ctx) {
   for (void* p : ctx->owned) cudaFree(p);
   for (void* p : ctx->owned_host) cudaFreeHost(p);
   for (cudaEvent_t e : ctx->ev_pool) cudaEventDestroy(e);
-  for (cudaEvent_t e : {ctx->ev_front[0], ctx->ev_front[1], ctx->ev_back[0], ctx->ev_back[1], ctx->ev_in, ctx->ev_fend})
+  for (cudaEvent_t e : {ctx->ev_front[0], ctx->ev_front[1], ctx->ev_back[0], ctx->ev_back[1], ctx->ev_in, ctx->ev_fend,
+                        ctx->ev_lend})
     if (e) cudaEventDestroy(e);
   if (ctx->fst) cudaStreamDestroy(ctx->fst);
+  if (ctx->lst) cudaStreamDestroy(ctx->lst);
   if (ctx->occ_h) cudaFreeHost(ctx->occ_h);
   if (ctx->stage) cudaFree(ctx->stage);
   delete ctx;
