@@ -169,6 +169,16 @@ tg_status tc_prepare_weights(const float* W, int N, int K, int precision, TcWeig
   }();
   if ((precision == TG_PREC_TF32X3 || precision == TG_PREC_F16X3) && x3_bn > 0 && x3_bn < 256 && N > 256)
     ntn = (N + x3_bn - 1) / x3_bn;
+  // narrow fp32-level GEMMs (N <= 192: G3, G4, the score MLP) run ONE N tile of round16(N) columns
+  // (single-buffered [big | small]): a tf32x3 k-block of 16 K costs about the same (~0.47 us, six
+  // MMAs) at N = 96 and N = 176 (clock64 traces), so two 96-column tiles cost twice the MMA time
+  // and convert A twice (measured: G3 68 -> 55 us, G4 42 -> 36 us per launch; TG_X3_NARROW=2: two)
+  static const int x3_narrow = [] {
+    const char* e = getenv("TG_X3_NARROW");
+    return e ? atoi(e) : 1;
+  }();
+  if ((precision == TG_PREC_TF32X3 || precision == TG_PREC_F16X3) && N <= 256 && N <= x3_bn && x3_narrow >= 1)
+    ntn = std::min(ntn, x3_narrow);
   int BN = (N + ntn - 1) / ntn;
   BN = (BN + 15) & ~15;
   const int kbb = tc_kb_bytes(precision);          // bytes of K per k-block row
