@@ -826,7 +826,10 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     const int v = e ? atoi(e) : 0;
     return v > 0 && v <= kMaxS ? v : 64;
   }();
-  int S = cfg->superbatch ? cfg->superbatch : s_default;
+  // default S: the cost model below picks it in [smax / 8, smax] (smax: the workspace budget);
+  // TG_SB_DEFAULT or cfg->superbatch fix it
+  const bool s_auto = cfg->superbatch == 0 && !getenv("TG_SB_DEFAULT") && cfg->precision != TG_PREC_FP32;
+  int S = cfg->superbatch ? cfg->superbatch : (s_auto ? kMaxS : s_default);
   // per-batch capacities: I_L = targets; I_{l-1} = C_l (k+1) <= I_l (k+1)
   int cap[TG_MAX_LAYERS + 1];
   int64_t cc = cfg->max_batch_targets;
@@ -856,6 +859,7 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
     };
     while (S > 1 && (ws(S) > (40ll << 30) || (int64_t)cap[1] * S > (int64_t)kSbhMaxBlocks * kSbhChunk)) --S;
   }
+  const int smax = S;
   if ((int64_t)cap[1] * S > ((int64_t)1 << 26)) return TG_EINVAL;
   if (cudaSetDevice(ctx->device) != cudaSuccess) return TG_ECUDA;
   ctx->cfg = *cfg;
@@ -1011,19 +1015,40 @@ tg_status tg_model_load(tg_ctx* ctx, const tg_model_cfg* cfg, const float* param
       w.fa_kb0 = kb0;
     }
   }
-  // ---- superbatch size fitted to whole waves of the value/output projection G2 (the largest GEMM):
-  // with the default S, pick S' in [S/2, S] maximising S' / waves(S'), waves = its N x M tiles of
-  // the top layer's worst-case row count (S' x max_batch_targets) over the 148 SMs, e.g. Reddit:
-  // S = 64 -> 600 tiles = 5 waves (the last holding 8 tiles), S = 63 -> 591 tiles = 4 waves
+  // ---- superbatch size from a wave-quantised cost model (default S only): per superbatch, every
+  // projection GEMM of every layer runs ceil(tiles / 148) waves of tiles that each cost nkb k-blocks
+  // of ~0.08 us per MMA instruction (6 per k-block in the fp32-level modes: 0.47 us, clock64 traces;
+  // N <= 176 costs the same as wider tiles), the attention + LayerNorm cost ~8 ns per target and
+  // layer at k = 20, D = 516 (scaled by k D), and ~140 us per superbatch is fixed (front-stream
+  // overlap, launch ramps); rows per layer ~ S x max_batch_targets. S minimises cost / S over
+  // [smax / 8, smax] -- Reddit: S = 94 (G2 882 tiles = 5.96 waves, G3/G4 294 tiles = 1.99 waves),
+  // 51 ms per pass against 54 ms at S = 63 and 64
   if (cfg->superbatch == 0 && !getenv("TG_SB_DEFAULT") && cfg->precision != TG_PREC_FP32 && ctx->lw[L - 1].tcF.ntn > 0) {
-    const int64_t ntn = ctx->lw[L - 1].tcF.ntn, T = cfg->max_batch_targets;
+    const int64_t T = cfg->max_batch_targets;
+    const bool x3 = cfg->precision == TG_PREC_TF32X3 || cfg->precision == TG_PREC_F16X3;
+    const double t_kb = 0.08 * (x3 ? 6 : 4);  // us per k-block
+    static const bool u1_on = [] {
+      const char* e = getenv("TG_U1");
+      return !(e && e[0] == '0');
+    }();
+    const bool u1_will = u1_on && ((long long)ctx->g.V + 1) * HDp * 4 <= (8ll << 30);
+    const double c_t = 8e-3 * ((double)k * Dp) / (20.0 * 516.0);  // us per target and layer
+    auto waves = [](int64_t tiles) { return (double)((tiles + 147) / 148); };
     int best = S;
-    double best_r = 0.0;
-    for (int s2 = S; s2 >= std::max(1, S / 2); --s2) {
-      const int64_t tiles = ((int64_t)s2 * T + 127) / 128 * ntn;
-      const double r = (double)s2 / (double)((tiles + 147) / 148);
-      if (r > best_r * 1.0001) {
-        best_r = r;
+    double best_c = 1e300;
+    for (int s2 = smax; s2 >= std::max(1, smax / 8); --s2) {
+      const int64_t mt = ((int64_t)s2 * T + 127) / 128;
+      double c = 140.0 + (double)L * s2 * T * c_t;
+      for (int l = 0; l < L; ++l) {
+        const LayerW& w = ctx->lw[l];
+        if (!(l == 0 && u1_will)) c += waves(mt * w.tcP.ntn) * w.tcP.nkb * t_kb;
+        c += waves(mt * w.tcF.ntn) * w.tcF.nkb * t_kb;
+        c += waves(mt * w.tcW1.ntn) * w.tcW1.nkb * t_kb;
+        c += waves(mt * w.tcW2.ntn) * w.tcW2.nkb * t_kb;
+      }
+      c /= s2;
+      if (c < best_c * 0.9999) {
+        best_c = c;
         best = s2;
       }
     }
