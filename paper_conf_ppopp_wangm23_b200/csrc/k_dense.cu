@@ -102,7 +102,12 @@ void launch_gemm_simt(const GemmArgs& g, cudaStream_t st) {
 // dense A operand of the merge FFN, Eq. 7) and/or the bf16 merge-FFN
 // input row rh = [LN(y) (Dp) | 0 | h^(l-1) at rh_off (16-byte aligned) | 0] (Eq. 7).
 constexpr int kLnMaxD4 = 256;  // Dp <= 1024 (checked at model load)
-__global__ void __launch_bounds__(256, 4)
+// NJ = ceil(Dp / 128) float4 per lane and row. Two rows per warp iteration (r2): their loads
+// (y rows, the h row pointers, then the h rows) are all issued before either row is reduced,
+// so each warp keeps two rows of memory in flight (the single-row loop exposed the pointer ->
+// h-row dependent latency once per row: 107 us per launch at 50k rows, 2.6 TB/s).
+template <int NJ>
+__global__ void __launch_bounds__(256, 3)
     k_layernorm(const float* __restrict__ y, float* __restrict__ r, int Dp, int dn, int dnp, int de, int dep, int dt,
                 const float* __restrict__ gamma, const float* __restrict__ beta, const int* __restrict__ m_dev,
                 const float* const* __restrict__ hs_rows, const float* __restrict__ phi0,
@@ -129,70 +134,94 @@ __global__ void __launch_bounds__(256, 4)
   const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, nw = (gridDim.x * blockDim.x) >> 5;
   const float D = (float)(dn + de + dt);
   const int nh4 = dnp >> 2;
-  for (int row = warp; row < M; row += nw) {
-    const float4* yr = reinterpret_cast<const float4*>(y + (size_t)row * Dp);
-    const float4* hr = reinterpret_cast<const float4*>(hs_rows[row]);
-    float4 v[8];
-    float sum = 0.f;
+  for (int row0 = warp; row0 < M; row0 += 2 * nw) {
+    const int rows[2] = {row0, row0 + nw};
+    const bool live1 = rows[1] < M;
+    float4 v[2][NJ];
+    const float4* hr[2];
 #pragma unroll
-    for (int j = 0; j < 8; ++j) {
-      const int q = lane + 32 * j;
-      v[j] = make_float4(0.f, 0.f, 0.f, 0.f);
-      if (q < D4) {
-        const float4 a = yr[q];
-        const float4 b = q < nh4 ? hr[q] : s_q[q];  // + q = [h || 0 || Phi(0)] (pads are zero)
-        v[j] = make_float4(a.x + b.x, a.y + b.y, a.z + b.z, a.w + b.w);
-        sum += (v[j].x + v[j].y) + (v[j].z + v[j].w);  // padded columns are exact zeros
+    for (int u = 0; u < 2; ++u) hr[u] = (u == 0 || live1) ? reinterpret_cast<const float4*>(hs_rows[rows[u]]) : nullptr;
+#pragma unroll
+    for (int u = 0; u < 2; ++u) {
+      const float4* yr = reinterpret_cast<const float4*>(y + (size_t)rows[u] * Dp);
+#pragma unroll
+      for (int j = 0; j < NJ; ++j) {
+        const int q = lane + 32 * j;
+        v[u][j] = (q < D4 && (u == 0 || live1)) ? yr[q] : make_float4(0.f, 0.f, 0.f, 0.f);
       }
     }
+    float4 hv[2][2];  // the first 64 float4 of each h row (d_n <= 256), issued with the y loads
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
-    const float mu = sum / D;
-    float var = 0.f;
+    for (int u = 0; u < 2; ++u)
 #pragma unroll
-    for (int j = 0; j < 8; ++j) {
-      const int q = lane + 32 * j;
-      if (q < D4) {
-        const float4 w = s_w[q];
-        const float dx = v[j].x - mu, dy = v[j].y - mu, dz = v[j].z - mu, dw = v[j].w - mu;
-        var = fmaf(w.x * dx, dx, var);
-        var = fmaf(w.y * dy, dy, var);
-        var = fmaf(w.z * dz, dz, var);
-        var = fmaf(w.w * dw, dw, var);
+      for (int j = 0; j < 2; ++j) {
+        const int q = lane + 32 * j;
+        hv[u][j] = (q < nh4 && (u == 0 || live1)) ? hr[u][q] : make_float4(0.f, 0.f, 0.f, 0.f);
       }
-    }
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) var += __shfl_xor_sync(0xffffffffu, var, o);
-    const float rstd = rsqrtf(var / D + 1e-5f);
+    for (int u = 0; u < 2; ++u) {
+      if (u == 1 && !live1) break;
+      const int row = rows[u];
+      float sum = 0.f;
 #pragma unroll
-    for (int j = 0; j < 8; ++j) {
-      const int q = lane + 32 * j;
-      if (q < D4) {
-        const float4 g = s_g[q], b = s_b[q];  // zero on padded columns -> output 0 there
-        const float4 o4 = make_float4(fmaf((v[j].x - mu) * rstd, g.x, b.x), fmaf((v[j].y - mu) * rstd, g.y, b.y),
-                                      fmaf((v[j].z - mu) * rstd, g.z, b.z), fmaf((v[j].w - mu) * rstd, g.w, b.w));
-        if (r) reinterpret_cast<float4*>(r + (size_t)row * ldr)[q] = o4;
-        if (rh) {
-          __nv_bfloat162 lo = __floats2bfloat162_rn(o4.x, o4.y), hi = __floats2bfloat162_rn(o4.z, o4.w);
+      for (int j = 0; j < NJ; ++j) {
+        const int q = lane + 32 * j;
+        if (q < D4) {
+          const float4 b = q < nh4 ? (j < 2 ? hv[u][j < 2 ? j : 0] : hr[u][q]) : s_q[q];  // + q = [h || 0 || Phi(0)]
+          v[u][j] = make_float4(v[u][j].x + b.x, v[u][j].y + b.y, v[u][j].z + b.z, v[u][j].w + b.w);
+          sum += (v[u][j].x + v[u][j].y) + (v[u][j].z + v[u][j].w);  // padded columns are exact zeros
+        }
+      }
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
+      const float mu = sum / D;
+      float var = 0.f;
+#pragma unroll
+      for (int j = 0; j < NJ; ++j) {
+        const int q = lane + 32 * j;
+        if (q < D4) {
+          const float4 w = s_w[q];
+          const float dx = v[u][j].x - mu, dy = v[u][j].y - mu, dz = v[u][j].z - mu, dw = v[u][j].w - mu;
+          var = fmaf(w.x * dx, dx, var);
+          var = fmaf(w.y * dy, dy, var);
+          var = fmaf(w.z * dz, dz, var);
+          var = fmaf(w.w * dw, dw, var);
+        }
+      }
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) var += __shfl_xor_sync(0xffffffffu, var, o);
+      const float rstd = rsqrtf(var / D + 1e-5f);
+#pragma unroll
+      for (int j = 0; j < NJ; ++j) {
+        const int q = lane + 32 * j;
+        if (q < D4) {
+          const float4 g = s_g[q], b = s_b[q];  // zero on padded columns -> output 0 there
+          const float4 o4 = make_float4(fmaf((v[u][j].x - mu) * rstd, g.x, b.x), fmaf((v[u][j].y - mu) * rstd, g.y, b.y),
+                                        fmaf((v[u][j].z - mu) * rstd, g.z, b.z), fmaf((v[u][j].w - mu) * rstd, g.w, b.w));
+          if (r) reinterpret_cast<float4*>(r + (size_t)row * ldr)[q] = o4;
+          if (rh) {
+            __nv_bfloat162 lo = __floats2bfloat162_rn(o4.x, o4.y), hi = __floats2bfloat162_rn(o4.z, o4.w);
+            uint2 pk;
+            pk.x = *reinterpret_cast<uint32_t*>(&lo);
+            pk.y = *reinterpret_cast<uint32_t*>(&hi);
+            *reinterpret_cast<uint2*>(rh + (size_t)row * ldrh + 4 * q) = pk;
+          }
+        }
+      }
+      if (r)  // h^(l-1) after LN(y): the merge FFN's [LN(y) | h] row is dense
+        for (int q = lane, j = 0; q < nh4; q += 32, ++j)
+          reinterpret_cast<float4*>(r + (size_t)row * ldr + Dp)[q] = j < 2 ? hv[u][j & 1] : hr[u][q];
+      if (rh) {  // [Dp, ldrh): zeros, h^(l-1) at rh_off, zeros
+        const int q0 = (rh_off - Dp) >> 2;
+        for (int q = lane; 4 * q < ldrh - Dp; q += 32) {
+          float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
+          if (q >= q0 && q - q0 < nh4) x = hr[u][q - q0];
+          __nv_bfloat162 lo = __floats2bfloat162_rn(x.x, x.y), hi = __floats2bfloat162_rn(x.z, x.w);
           uint2 pk;
           pk.x = *reinterpret_cast<uint32_t*>(&lo);
           pk.y = *reinterpret_cast<uint32_t*>(&hi);
-          *reinterpret_cast<uint2*>(rh + (size_t)row * ldrh + 4 * q) = pk;
+          *reinterpret_cast<uint2*>(rh + (size_t)row * ldrh + Dp + 4 * q) = pk;
         }
-      }
-    }
-    if (r)  // h^(l-1) after LN(y): the merge FFN's [LN(y) | h] row is dense
-      for (int q = lane; q < nh4; q += 32) reinterpret_cast<float4*>(r + (size_t)row * ldr + Dp)[q] = hr[q];
-    if (rh) {  // [Dp, ldrh): zeros, h^(l-1) at rh_off, zeros
-      const int q0 = (rh_off - Dp) >> 2;
-      for (int q = lane; 4 * q < ldrh - Dp; q += 32) {
-        float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
-        if (q >= q0 && q - q0 < nh4) x = hr[q - q0];
-        __nv_bfloat162 lo = __floats2bfloat162_rn(x.x, x.y), hi = __floats2bfloat162_rn(x.z, x.w);
-        uint2 pk;
-        pk.x = *reinterpret_cast<uint32_t*>(&lo);
-        pk.y = *reinterpret_cast<uint32_t*>(&hi);
-        *reinterpret_cast<uint2*>(rh + (size_t)row * ldrh + Dp + 4 * q) = pk;
       }
     }
   }
@@ -202,11 +231,19 @@ void launch_layernorm(const float* y, float* r, int Dp, int dn, int dnp, int de,
                       const float* gamma, const float* beta, const int* m_dev, int m_max,
                       const float* const* hs_rows, const float* phi0, unsigned short* rh, int ldrh, int rh_off,
                       cudaStream_t st) {
-  int blocks = (m_max + 7) / 8;  // 8 warps (rows) per CTA
-  if (blocks > 148 * 4) blocks = 148 * 4;  // one resident wave (4 CTAs / SM at <= 64 registers)
+  int blocks = (m_max + 15) / 16;  // 8 warps per CTA, two rows per warp iteration
+  if (blocks > 148 * 3) blocks = 148 * 3;  // one resident wave (3 CTAs / SM at <= 85 registers)
   if (blocks < 1) blocks = 1;
-  launch_k(k_layernorm, dim3(blocks), dim3(256), 0, st, y, r, Dp, dn, dnp, de, dep, dt, gamma, beta, m_dev, hs_rows,
-           phi0, rh, ldrh, rh_off);
+  const int nj = ((Dp >> 2) + 31) / 32;
+#define TG_LN(NJ)                                                                                              \
+  case NJ:                                                                                                     \
+    launch_k(k_layernorm<NJ>, dim3(blocks), dim3(256), 0, st, y, r, Dp, dn, dnp, de, dep, dt, gamma, beta, m_dev, \
+             hs_rows, phi0, rh, ldrh, rh_off);                                                                 \
+    break;
+  switch (nj) {
+    TG_LN(1) TG_LN(2) TG_LN(3) TG_LN(4) TG_LN(5) TG_LN(6) TG_LN(7) default: TG_LN(8)
+  }
+#undef TG_LN
 }
 
 // -------------------------------------------------------------------- score
