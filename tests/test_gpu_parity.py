@@ -398,6 +398,39 @@ print("ok")
     assert r.returncode == 0 and "ok" in r.stdout, r.stderr[-2000:]
 
 
+@pytest.mark.parametrize("prec", [1, 2, 4])
+def test_layer1_query_table_bitexact_subprocess(prec):
+    """R27: the layer-1 query side u = P x_i + b_u comes from the per-node table U1 built at
+    tg_model_load by the same row-invariant GEMM; with TG_U1=0 every layer-1 target runs G1
+    instead. Scores of a Reddit-shaped stream (tf32x3, bf16, f16x3) must be bit-identical. The
+    toggle is read once per process, hence the subprocesses."""
+    import os
+    import subprocess
+    import sys
+    import tempfile
+    code = r'''
+import sys, numpy as np
+from tests.gpu_helpers import setup, make_ctx
+from tests.test_gpu_parity import _stream_gpu
+cfg, s, flat = setup("reddit", n_edges=6000)
+mc = cfg.model
+ctx = make_ctx(s, flat, mc, precision=int(sys.argv[1]), superbatch=8)
+sc, _ = _stream_gpu(ctx, s, mc.batch)
+np.save(sys.argv[2], np.asarray(sc))
+print("ok")
+'''
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    outs = []
+    with tempfile.TemporaryDirectory() as td:
+        for u1 in ("1", "0"):
+            f = os.path.join(td, f"sc{u1}.npy")
+            r = subprocess.run([sys.executable, "-c", code, str(prec), f], cwd=root, capture_output=True, text=True,
+                               env={**os.environ, "TG_U1": u1}, timeout=600)
+            assert r.returncode == 0 and "ok" in r.stdout, r.stderr[-2000:]
+            outs.append(np.load(f))
+    assert outs[0].shape == outs[1].shape and np.array_equal(outs[0].view(np.uint32), outs[1].view(np.uint32))
+
+
 @pytest.mark.parametrize("S", [1, 16])
 def test_index_rebuild_under_fifo_churn(S):
     """A tiny limit (10 items) makes nearly every layer-1 lookup a miss: ~10^5 inserts into an
