@@ -12,9 +12,10 @@ rows = list(csv.reader(open(sys.argv[1])))
 hdr = next(i for i, r in enumerate(rows) if "Kernel Name" in r)
 h = rows[hdr]
 ik, ig, iv = h.index("Kernel Name"), h.index("Grid Size"), h.index("Metric Value")
+im = h.index("Metric Name") if "Metric Name" in h else None
 L = []
 for r in rows[hdr + 1:]:
-    if len(r) > iv:
+    if len(r) > iv and (im is None or r[im] == "gpu__time_duration.sum"):  # one row per launch
         name = re.sub(r"\(.*", "", r[ik]).replace("void ", "").replace("tg::", "")
         L.append((name, r[ig], float(r[iv]) / 1e3))
 starts = [i for i, x in enumerate(L) if x[0] == "k_dedup"]
