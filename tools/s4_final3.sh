@@ -10,4 +10,4 @@ python tools/kernel_table.py $out/sb_full_$prec.ncu-rep --out $out/kernels_$prec
 python tools/ncu_summary.py $out/sb_full_$prec.ncu-rep --json $out/sb_full_$prec.summary.json > /dev/null
 ncu -i $out/sb_full_$prec.ncu-rep --page source --csv --print-source sass -k regex:k_attn_g > $out/attn_src.csv 2>/dev/null; gzip -f $out/attn_src.csv
 gzip -f $out/launches_$prec.csv; rm -f $out/sb_full_$prec.ncu-rep
-bash tools/sanitize.sh $tag
+[ -n "$SANITIZE" ] && bash tools/sanitize.sh $tag
